@@ -1,0 +1,205 @@
+/*
+ * strings_sched.h -- C ABI of the B200-native Strings scheduler hot path.
+ *
+ * Method: Sengupta, Goswami, Schwan, Pallavi, "Scheduling Multi-tenant Cloud
+ * Workloads on Accelerator-based Systems", SC14.  Citations "P:L<n>" refer to
+ * lines of the paper text; "R-n" to the readings in DESIGN.md §6;
+ * "§4.x" to the scheduler semantics in DESIGN.md §4.
+ *
+ * The library owns device selection (the runtime overrides the
+ * application's cudaSetDevice), merges all tenants of a GPU into one context
+ * (P:L179-185), and co-schedules tenants' H2D / kernel / D2H phases on
+ * the copy engines and on SM partitions of a persistent kernel.
+ *
+ * Conventions
+ *  - Every call returns a strings_status_t (0 = STRINGS_OK, negative = error);
+ *    no call aborts the process.  The last CUDA error seen by the library is
+ *    kept per process (strings_last_cuda_error).
+ *  - All calls are thread-safe.  Tenants are typically distinct host threads.
+ *  - Host buffers are owned by the caller.  Device memory is owned by the
+ *    library (per-GPU arena of resident job slots).
+ *  - Times are ns on the library clock: CLOCK_MONOTONIC since strings_init in
+ *    MEASURED mode, the virtual clock in INJECTED / DECISIONS_ONLY mode.
+ */
+#ifndef STRINGS_SCHED_H
+#define STRINGS_SCHED_H
+
+#include <stdint.h>
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t strings_status_t;
+typedef uint32_t strings_tenant_t;
+typedef uint64_t strings_job_t;
+
+#define STRINGS_OK       0
+#define STRINGS_EINVAL  (-1)  /* bad argument (sizes, class, unknown tenant/job)          */
+#define STRINGS_ENOMEM  (-2)  /* host or device allocation failed                          */
+#define STRINGS_EAGAIN  (-3)  /* not ready / try again                                      */
+#define STRINGS_ECUDA   (-4)  /* CUDA error; see strings_last_cuda_error()                  */
+#define STRINGS_ESTATE  (-5)  /* not initialised, already initialised, or shutting down     */
+#define STRINGS_EFAULT  (-6)  /* a job of this tenant failed (fault localisation)   */
+
+/* Workload-balancing policies (balancer = level 1). */
+#define STRINGS_BAL_GRR      0  /* Global Round Robin                                  */
+#define STRINGS_BAL_GMIN     1  /* fewest bound jobs, ties -> lowest GID            */
+#define STRINGS_BAL_GWTMIN   2  /* load / device weight                                 */
+#define STRINGS_BAL_RTF      3  /* runtime feedback                                 */
+#define STRINGS_BAL_GUF      4  /* GPU-utilisation feedback                             */
+#define STRINGS_BAL_DTF      5  /* data-transfer feedback                               */
+#define STRINGS_BAL_MBF      6  /* memory-bandwidth feedback                            */
+#define STRINGS_BAL_DYNAMIC  7  /* policy arbiter: GMin until feedback, then MBF, P:L311 (R-15) */
+
+/* Device-level dispatch policies (level 2). */
+#define STRINGS_DEV_FIFO 0      /* wake in placement order (baseline)                          */
+#define STRINGS_DEV_LAS  1      /* least attained service, weighted, phase-blind (R-7) */
+#define STRINGS_DEV_PS   2      /* Phase Selection: one per phase, else KL > H2D = D2H */
+
+/* Tenant kernel classes (the paper's workload classes, Table I). */
+#define STRINGS_VSCALE 0        /* y = alpha * x, fp32, n elements          (memory-bound)      */
+#define STRINGS_GEMM   1        /* C = A.B, bf16 in / fp32 out, R repetitions (compute-bound)   */
+#define STRINGS_XFER   2        /* y = fmix32(x ^ seed), u32, n elements    (transfer-heavy)    */
+
+/* Timing modes. */
+#define STRINGS_TIMING_MEASURED        0  /* real clock, real completions                       */
+#define STRINGS_TIMING_INJECTED        1  /* virtual clock from descriptor durations; every
+                                             op still runs on the GPU; decisions bit-exact     */
+#define STRINGS_TIMING_DECISIONS_ONLY  2  /* test-only: decision core without device work;
+                                             D2H buffers are NOT written                        */
+
+typedef struct {
+    int32_t  num_gpus;       /* G logical devices; 0 = number of physical GPUs used             */
+    int32_t  physical_gpus;  /* physical GPUs to use (first N visible); 0 = all visible         */
+    int32_t  balancer;       /* STRINGS_BAL_*                                                   */
+    int32_t  las_admission;  /* 1 = admit pending jobs in weighted-LAS order (R-9)              */
+    int32_t  device_policy;  /* STRINGS_DEV_*                                                   */
+    int32_t  partitions;     /* P KL slots (SM partitions) per device; 0 -> 2                   */
+    int32_t  awake_budget;   /* A woken-unfinished ops per device; 0 -> 2 + P (R-11)            */
+    int32_t  admit_cap;      /* M resident jobs per device; 0 -> 2 * A (R-12)                   */
+    int32_t  joint_select;   /* -1 auto (on for DTF/MBF/DYNAMIC), 0 off, 1 on (R-16)            */
+    int32_t  timing_mode;    /* STRINGS_TIMING_*                                                */
+    uint64_t quantum_ns;     /* LAS epoch Q; 0 -> 1,000,000 (R-5)                               */
+    uint64_t slot_bytes;     /* device bytes per resident job slot; 0 -> 160 MiB                */
+    const char* trace_path;  /* if non-NULL the decision trace is written there at drain/shutdown */
+    int32_t  trace_in_memory;/* 1 = keep the trace for strings_trace_copy                       */
+    int32_t  reserved[7];
+} strings_config_t;
+
+/* Kernel descriptor: which tenant kernel the KL phase runs, and its sizes.
+ * Fixed kernel table, no user function pointers.  H2D / D2H buffer layout:
+ *   VSCALE: h2d = { x[n] fp32 },                 d2h = { y[n] fp32 }
+ *   GEMM:   h2d = { A[m*k] bf16, B[k*n] bf16 },  d2h = { C[m*n] fp32 }  (row-major)
+ *           m % 128 == 0, n % 256 == 0, k % 64 == 0, k <= 256, reps >= 1
+ *   XFER:   h2d = { x[n] u32 },                  d2h = { y[n] u32 }                           */
+typedef struct {
+    uint32_t kclass;         /* STRINGS_VSCALE / STRINGS_GEMM / STRINGS_XFER                  */
+    uint32_t reps;           /* GEMM repetitions R (R-17); ignored otherwise                  */
+    uint64_t n, m, k;        /* sizes (see above)                                             */
+    float    alpha;          /* VSCALE scalar                                                 */
+    uint32_t seed;           /* XFER seed                                                     */
+    uint64_t arrival_ns;     /* INJECTED / DECISIONS_ONLY: virtual arrival time (Eq. 4 inputs);
+                                MEASURED: ignored (arrival = submit time)                     */
+    uint64_t inj_h2d_ns, inj_kl_ns, inj_d2h_ns;  /* injected phase durations (INJECTED modes)   */
+} strings_kernel_desc_t;
+
+typedef struct { void* host; uint64_t bytes; } strings_buf_t;
+
+typedef struct {
+    uint64_t job;
+    uint32_t tenant, seq;
+    int32_t  gid;            /* logical device chosen by the balancer (-1 before PLACE)       */
+    int32_t  status;         /* STRINGS_OK, STRINGS_EAGAIN (not done) or an error             */
+    uint64_t t_arrival, t_place;
+    uint64_t t_start[3], t_done[3];          /* per phase H2D, KL, D2H (library clock)       */
+    int32_t  kl_slot;                        /* logical KL slot                               */
+    int32_t  kl_partition;                   /* physical SM partition that ran the KL        */
+    uint64_t kl_gpu_start_ns, kl_gpu_end_ns; /* %globaltimer stamps of the KL phase          */
+} strings_job_info_t;
+
+typedef struct {
+    uint64_t jobs_submitted, jobs_done, jobs_failed;
+    uint64_t t_first_submit_ns, t_last_done_ns;   /* library clock                              */
+    uint64_t h2d_bytes, d2h_bytes, kernel_bytes, kernel_flop;
+    uint64_t trace_records;
+    uint64_t decisions;                           /* PLACE + WAKE records                       */
+    uint64_t engine_busy_ns[8][3];                /* per logical device (first 8), per engine   */
+    int32_t  num_gpus, physical_gpus, partitions, sms_per_partition;
+} strings_stats_t;
+
+/* Initialise the runtime (gPool creation): enumerate the GPUs,
+ * create one context + H2D/D2H streams per GPU, allocate the resident-slot
+ * arena, launch the persistent dispatcher kernel, start the engine thread.
+ * cfg may be NULL (defaults).  STRINGS_ECUDA if no CUDA device is usable
+ * (except in DECISIONS_ONLY mode).  STRINGS_ESTATE if already initialised.    */
+strings_status_t strings_init(const strings_config_t* cfg);
+
+/* Register a tenant (Request Manager; RCB entry P:L489-515).
+ * weight >= 1 is the tenant priority/weight; max_inflight >= 1 is the number of
+ * its jobs that may be admitted at once (server threads).              */
+strings_status_t strings_register_tenant(uint32_t weight, uint32_t max_inflight,
+                                         strings_tenant_t* out);
+
+/* Submit one job (asynchronous): H2D of the h2d buffers, the KL
+ * phase described by desc, D2H into the d2h buffers.  Jobs of one tenant are
+ * admitted in submission order.  Buffer counts and sizes must match
+ * desc (see strings_kernel_desc_t).  Pinned buffers (strings_host_alloc or
+ * cudaHostRegister'ed) are DMA'd directly; pageable ones are staged (MOT/PMT,
+ * P:L327-329): H2D data is copied at submit, D2H data is copied back before the
+ * job counts as done.  The caller must not read d2h buffers (nor modify pinned
+ * h2d buffers) until strings_sync(tenant) returns.  priority 0 = tenant
+ * weight.  *out receives the job id.                                          */
+strings_status_t strings_submit(strings_tenant_t tenant, const strings_kernel_desc_t* desc,
+                                const strings_buf_t* h2d, int32_t n_h2d,
+                                const strings_buf_t* d2h, int32_t n_d2h,
+                                uint32_t priority, strings_job_t* out);
+
+/* Block until every job this tenant submitted is done (Sync Stream Translator,
+ * never a device-wide sync).  Returns STRINGS_EFAULT if one of
+ * them failed.  In INJECTED mode this also starts virtual-time processing.   */
+strings_status_t strings_sync(strings_tenant_t tenant);
+
+/* Block until every submitted job of every tenant is done; flush the trace.    */
+strings_status_t strings_drain(void);
+
+/* Implicit sync, then remove the tenant (cudaThreadExit path, P:L329, P:L667,
+ * frees its PMT staging; its feedback already reached the SFT).       */
+strings_status_t strings_unregister_tenant(strings_tenant_t tenant);
+
+/* Drain, stop the dispatcher kernel and the engine thread, free everything.   */
+strings_status_t strings_shutdown(void);
+
+/* Pinned host memory for the zero-copy fast path (R-19).                       */
+strings_status_t strings_host_alloc(uint64_t bytes, void** p);
+strings_status_t strings_host_free(void* p);
+
+/* Per-job record (Request Monitor view): GID, phase times, status.     */
+strings_status_t strings_job_info(strings_job_t job, strings_job_info_t* info);
+
+/* Aggregate counters (RMO / FE view).                              */
+strings_status_t strings_get_stats(strings_stats_t* stats);
+
+/* Decision trace, kept when trace_in_memory = 1.              */
+strings_status_t strings_trace_size(uint64_t* bytes);
+strings_status_t strings_trace_copy(char* buf, uint64_t capacity, uint64_t* written);
+
+const char* strings_strerror(strings_status_t s);
+int32_t strings_last_cuda_error(void);
+const char* strings_version(void);
+
+/* Stand-alone tenant kernel launch (outside the scheduler) for kernel-level
+ * parity tests and roofline measurements (SURVEY §8(d) "kernel-level checks").
+ * dev_in / dev_out are device pointers laid out as the H2D / D2H buffers of
+ * desc; ctas = number of CTAs (0 = one per SM); stream = cudaStream_t (NULL =
+ * legacy default).  Asynchronous.                                              */
+strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kernel_desc_t* desc,
+                                       void* const* dev_in, int32_t n_in,
+                                       void* const* dev_out, int32_t n_out,
+                                       int32_t ctas, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STRINGS_SCHED_H */

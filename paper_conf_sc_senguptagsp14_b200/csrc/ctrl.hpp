@@ -1,0 +1,60 @@
+// ctrl.hpp -- host <-> persistent-kernel control block (host-mapped pinned memory).
+//
+// One block per physical GPU.  It carries, per hosted logical device, the
+// device-resident request queue of KL work items (the paper's Dispatcher ->
+// GPU path, replacing the RT-signal wake-up of L697 with a
+// doorbell the GPU polls) and the completion words the GPU writes back
+// (Request Monitor input, L671).
+#pragma once
+#include <cstdint>
+
+#include "tenant_kernels.cuh"
+
+namespace strings_dev {
+
+constexpr int kRing = 256;            // KL ring entries per logical device
+constexpr uint32_t kStop = 0xFFFFFFFFu;
+
+struct __align__(64) KlRing {
+  volatile uint32_t tail;             // number of items published (host writes, GPU reads)
+  uint32_t pad[15];
+  KlItem items[kRing];
+};
+
+struct __align__(32) KlDone {
+  volatile uint32_t seq;              // = item.seq when the item has finished
+  uint32_t partition;
+  uint64_t t_start, t_end;            // %globaltimer ns
+};
+
+// Host-mapped part (cudaHostAlloc mapped): rings + completions + shutdown flag.
+struct HostCtrl {
+  volatile uint32_t shutdown;
+  uint32_t pad[15];
+  // followed by KlRing[L] and KlDone[L][kRing] (sizes depend on L)
+};
+
+// Device-memory part: claim counters and per-partition mailboxes.
+struct __align__(128) PartState {
+  uint32_t gen;                       // item generation published by the leader (kStop = exit)
+  uint32_t done_gen;                  // last generation fully finished by all CTAs
+  uint32_t done_cnt;                  // CTAs finished with the current generation
+  uint32_t ring_idx;
+  uint64_t t_start;
+  KlItem item;
+};
+
+struct DispatchParams {
+  HostCtrl* ctrl;                     // device view of the host-mapped block
+  KlRing* rings;                      // [L]
+  KlDone* done;                       // [L * kRing]
+  uint32_t* heads;                    // [L] device-memory claim counters
+  PartState* parts;                   // [L * P]
+  int L, P;                           // logical devices hosted, partitions per logical device
+};
+
+inline size_t host_ctrl_bytes(int L) {
+  return sizeof(HostCtrl) + sizeof(KlRing) * L + sizeof(KlDone) * kRing * L;
+}
+
+}  // namespace strings_dev

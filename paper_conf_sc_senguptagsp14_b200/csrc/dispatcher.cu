@@ -1,0 +1,177 @@
+// dispatcher.cu -- persistent sm_100a dispatcher kernel and stand-alone launcher.
+//
+// The persistent kernel is the device half of the per-device GPU scheduler
+// (PAPER.md L331-333, L667-673): it pulls KL work items from the
+// device-resident request queue (KL ring, ctrl.hpp) and runs tenant kernel
+// bodies on SM partitions, so tenants' kernels co-run on disjoint SMs while
+// the copy engines stream other tenants' buffers (PS, L819; MBF, L831).
+//
+// Geometry: one CTA per SM (grid = #SMs, 256 threads, ~196 KB smem so GEMM
+// operands fit), split into NP = L*P partitions of contiguous CTAs.  Partition
+// q serves logical device q / P.  Its leader (CTA rank 0, thread 0):
+//   1. waits until the previous item is finished by every CTA (done_gen),
+//   2. polls the ring tail in host memory (ld.acquire.sys, nanosleep back-off)
+//      and claims the next item with a CAS on the device claim counter,
+//   3. copies the item into the partition mailbox and publishes gen+1
+//      (st.release.gpu).
+// Every CTA of the partition waits for the new generation, runs its share of
+// the item, and the last CTA to finish writes the completion word and the
+// %globaltimer stamps back to host memory (st.release.sys).
+#include <cstdio>
+
+#include "ctrl.hpp"
+
+namespace strings_dev {
+
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys(const volatile uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(volatile uint32_t* p, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void partition_of(int b, int G, int NP, int* q, int* start, int* S) {
+  int p = (int)(((long long)b * NP) / G);
+  while (p + 1 < NP && (int)(((long long)(p + 1) * G) / NP) <= b) ++p;
+  while (p > 0 && (int)(((long long)p * G) / NP) > b) --p;
+  *q = p;
+  *start = (int)(((long long)p * G) / NP);
+  *S = (int)(((long long)(p + 1) * G) / NP) - *start;
+}
+
+__global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams p) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ KlItem s_item;
+  __shared__ uint32_t s_gen;
+  GemmSmem sm = carve_smem(smem);
+  const int NP = p.L * p.P;
+  int q, start, S;
+  partition_of(blockIdx.x, gridDim.x, NP, &q, &start, &S);
+  const int rank = blockIdx.x - start;
+  const int ld = q / p.P;
+  PartState* ps = p.parts + q;
+  const uint32_t tmem = cta_setup(sm);
+  uint32_t mma_phase = 0;
+  uint32_t seen = 0;
+  for (;;) {
+    if (threadIdx.x == 0) {
+      if (rank == 0) {
+        while (ld_acquire_gpu(&ps->done_gen) != seen) __nanosleep(32);
+        uint32_t g;
+        uint32_t backoff = 32;
+        for (;;) {
+          const uint32_t tail = ld_acquire_sys(&p.rings[ld].tail);
+          const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&p.heads[ld]);
+          if (h < tail) {
+            if (atomicCAS(&p.heads[ld], h, h + 1) == h) {
+              const KlItem* src = &p.rings[ld].items[h % kRing];
+              const volatile uint4* s4 = reinterpret_cast<const volatile uint4*>(src);
+              uint4* d4 = reinterpret_cast<uint4*>(&ps->item);
+#pragma unroll
+              for (int w = 0; w < (int)(sizeof(KlItem) / 16); ++w) {
+                uint4 v;
+                v.x = s4[w].x; v.y = s4[w].y; v.z = s4[w].z; v.w = s4[w].w;
+                d4[w] = v;
+              }
+              ps->ring_idx = h % kRing;
+              ps->t_start = globaltimer();
+              g = seen + 1;
+              break;
+            }
+            continue;
+          }
+          if (ld_acquire_sys(&p.ctrl->shutdown)) {
+            g = kStop;
+            break;
+          }
+          __nanosleep(backoff);
+          if (backoff < 1024) backoff <<= 1;
+        }
+        st_release_gpu(&ps->gen, g);
+      }
+      uint32_t g;
+      while ((g = ld_acquire_gpu(&ps->gen)) == seen) __nanosleep(32);
+      s_gen = g;
+      if (g != kStop) s_item = ps->item;
+    }
+    __syncthreads();
+    const uint32_t g = s_gen;
+    if (g == kStop) break;
+    seen = g;
+    const KlItem it = s_item;
+    run_item(it, rank, S, sm, tmem, mma_phase);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      const uint32_t old = atomicAdd(&ps->done_cnt, 1u);
+      if (old == (uint32_t)S - 1) {
+        ps->done_cnt = 0;
+        KlDone* d = &p.done[ld * kRing + ps->ring_idx];
+        d->partition = (uint32_t)q;
+        d->t_start = ps->t_start;
+        d->t_end = globaltimer();
+        __threadfence_system();
+        st_release_sys(&d->seq, it.seq);
+        st_release_gpu(&ps->done_gen, seen);
+      }
+    }
+  }
+  cta_teardown(tmem);
+}
+
+// Stand-alone launch of one tenant body on `gridDim.x` CTAs (kernel-level
+// checks outside the scheduler, and KL_MODE_LAUNCH).
+__global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(KlItem it) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  GemmSmem sm = carve_smem(smem);
+  uint32_t tmem = 0, mma_phase = 0;
+  const bool gemm = it.kclass == 1;
+  if (gemm) tmem = cta_setup(sm);
+  run_item(it, blockIdx.x, gridDim.x, sm, tmem, mma_phase);
+  if (gemm) cta_teardown(tmem);
+}
+
+}  // namespace strings_dev
+
+// ----------------------------------------------------------------- host side
+namespace strings {
+
+cudaError_t launch_dispatcher(const strings_dev::DispatchParams& p, int grid, cudaStream_t s) {
+  cudaError_t e = cudaFuncSetAttribute(strings_dev::dispatcher_kernel,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)strings_dev::kSmemGemm);
+  if (e != cudaSuccess) return e;
+  strings_dev::dispatcher_kernel<<<grid, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t s) {
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(strings_dev::oneshot_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)strings_dev::kSmemGemm);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  const uint32_t smem = it.kclass == 1 ? strings_dev::kSmemGemm : 0;
+  strings_dev::oneshot_kernel<<<ctas, strings_dev::kThreads, smem, s>>>(it);
+  return cudaGetLastError();
+}
+
+}  // namespace strings

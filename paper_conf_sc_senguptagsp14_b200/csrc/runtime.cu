@@ -1,0 +1,933 @@
+// runtime.cu -- the C ABI (include/strings_sched.h), the engine thread and the
+// per-GPU executor (copy streams, resident slots, KL ring, persistent kernel).
+//
+// Structure:
+//   API calls (any thread) --> inbox under mu_ --> engine thread
+//   engine thread: drives strings::Core (core.cpp) in one of three timing
+//   modes and implements its Hooks by issuing physical ops at WAKE:
+//     H2D  cudaMemcpyAsync on the logical device's H2D stream + event
+//     KL   KlItem into the logical device's ring (host-mapped), the persistent
+//          dispatcher kernel claims it (dispatcher.cu)
+//     D2H  cudaMemcpyAsync on the D2H stream + event
+#include <cuda_runtime.h>
+#include <time.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <memory>
+#include <mutex>
+#include <queue>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "core.hpp"
+#include "ctrl.hpp"
+#include "../../include/strings_sched.h"
+
+namespace strings {
+cudaError_t launch_dispatcher(const strings_dev::DispatchParams& p, int grid, cudaStream_t s);
+cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t s);
+}  // namespace strings
+
+using strings_dev::HostCtrl;
+using strings_dev::KlDone;
+using strings_dev::KlItem;
+using strings_dev::KlRing;
+using strings_dev::kRing;
+
+namespace {
+
+std::atomic<int32_t> g_last_cuda_error{0};
+
+inline bool cuda_ok(cudaError_t e) {
+  if (e == cudaSuccess) return true;
+  g_last_cuda_error.store((int32_t)e);
+  return false;
+}
+
+uint64_t mono_ns() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return (uint64_t)ts.tv_sec * 1000000000ull + ts.tv_nsec;
+}
+
+constexpr uint64_t kAlign = 256;
+inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
+
+struct HostBuf {
+  void* user = nullptr;     // caller's buffer
+  uint64_t bytes = 0;
+  void* dma = nullptr;      // pinned address used by the copy engine
+  bool staged = false;      // dma is library-owned staging (PMT entry)
+};
+
+struct JobCtx {
+  strings::Job job;
+  strings_kernel_desc_t desc{};
+  std::vector<HostBuf> in, out;
+  int32_t status = STRINGS_EAGAIN;
+  // execution state
+  int slot = -1;                       // resident slot on the logical device
+  uint64_t dev_in[2] = {0, 0}, dev_out = 0;
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+  bool issued[3] = {false, false, false};
+  bool phys_done[3] = {false, false, false};
+  uint32_t kl_seq = 0;
+  int kl_idx = -1;
+  int kl_partition = -1;
+  uint64_t kl_t0 = 0, kl_t1 = 0;
+};
+
+struct Phys;
+
+struct Logical {
+  int gid = 0;
+  Phys* phys = nullptr;
+  int local = 0;                       // index among the logical devices of phys
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  std::vector<cudaStream_t> kl_streams;  // KL_MODE_LAUNCH only
+  int next_kl_stream = 0;
+  uint8_t* arena = nullptr;            // M slots of slot_bytes
+  std::vector<int> free_slots;
+  KlRing* ring = nullptr;              // host pointer
+  KlDone* done = nullptr;              // host pointer, kRing entries
+  uint32_t tail = 0;                   // items published
+  uint32_t completed = 0;              // items whose completion was consumed
+};
+
+struct Phys {
+  int dev = 0;
+  int sms = 0;
+  int L = 0;
+  HostCtrl* ctrl = nullptr;            // host-mapped block
+  void* ctrl_dev = nullptr;
+  uint8_t* dev_state = nullptr;        // heads + parts
+  uint8_t* arena = nullptr;
+  bool arena_owned = false;
+  cudaStream_t kstream = nullptr;
+  bool kernel_running = false;
+  std::vector<cudaEvent_t> ev_pool;
+};
+
+struct Tenant {
+  uint32_t weight = 1, c = 1;
+  uint64_t outstanding = 0;            // submitted, not done
+  uint64_t failed = 0;
+  uint32_t next_seq = 0;
+  bool active = true;
+};
+
+class Runtime;
+Runtime* g_rt = nullptr;
+std::mutex g_init_mu;
+
+class Runtime : public strings::Hooks {
+ public:
+  strings_config_t cfg{};
+  strings::CoreConfig ccfg;
+  int kl_mode = 0;                     // 0 persistent, 1 launch (profiling)
+  std::unique_ptr<strings::Core> core;
+  std::vector<std::unique_ptr<Phys>> phys;
+  std::vector<Logical> logical;
+  std::vector<Tenant> tenants;
+  std::deque<std::unique_ptr<JobCtx>> jobs;   // index = job id
+  std::vector<JobCtx*> inbox;
+  std::mutex mu;
+  std::condition_variable cv_engine, cv_done;
+  std::thread engine;
+  bool stop = false, sealed = false;
+  int32_t fatal = STRINGS_OK;
+  uint64_t t0 = 0;
+  uint64_t submitted = 0, done_count = 0, failed_count = 0;
+  uint64_t first_submit = 0, last_done = 0;
+  uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
+  // in-flight physical ops (measured mode): (job, engine)
+  std::vector<std::pair<JobCtx*, int>> inflight;
+  // virtual DONE events (injected / decisions-only)
+  struct VEv {
+    uint64_t t;
+    strings::Completion c;
+    bool operator>(const VEv& o) const { return t > o.t; }
+  };
+  std::priority_queue<VEv, std::vector<VEv>, std::greater<VEv>> vheap;
+
+  bool virtual_clock() const { return cfg.timing_mode != STRINGS_TIMING_MEASURED; }
+  bool has_gpu() const { return cfg.timing_mode != STRINGS_TIMING_DECISIONS_ONLY; }
+  uint64_t now() const { return mono_ns() - t0; }
+
+  // ------------------------------------------------------------ init/fini
+  strings_status_t init(const strings_config_t* c) {
+    if (c) cfg = *c;
+    if (cfg.partitions <= 0) cfg.partitions = 2;
+    if (cfg.awake_budget <= 0) cfg.awake_budget = 2 + cfg.partitions;
+    if (cfg.admit_cap <= 0) cfg.admit_cap = 2 * cfg.awake_budget;
+    if (cfg.quantum_ns == 0) cfg.quantum_ns = 1000000;
+    if (cfg.slot_bytes == 0) cfg.slot_bytes = 160ull << 20;
+    if (cfg.balancer < 0 || cfg.balancer > 7 || cfg.device_policy < 0 || cfg.device_policy > 2 ||
+        cfg.timing_mode < 0 || cfg.timing_mode > 2)
+      return STRINGS_EINVAL;
+    kl_mode = cfg.reserved[0] == 1 ? 1 : 0;
+    int nphys = 0;
+    if (has_gpu()) {
+      if (!cuda_ok(cudaGetDeviceCount(&nphys)) || nphys <= 0) return STRINGS_ECUDA;
+      if (cfg.physical_gpus > 0) nphys = std::min(nphys, (int)cfg.physical_gpus);
+    }
+    if (cfg.num_gpus <= 0) cfg.num_gpus = has_gpu() ? nphys : 1;
+    if (cfg.joint_select < 0)
+      cfg.joint_select = (cfg.balancer == STRINGS_BAL_DTF || cfg.balancer == STRINGS_BAL_MBF ||
+                          cfg.balancer == STRINGS_BAL_DYNAMIC);
+    ccfg.G = cfg.num_gpus;
+    ccfg.P = cfg.partitions;
+    ccfg.A = cfg.awake_budget;
+    ccfg.M = cfg.admit_cap;
+    ccfg.balancer = cfg.balancer;
+    ccfg.las_admission = cfg.las_admission;
+    ccfg.device_policy = cfg.device_policy;
+    ccfg.joint = cfg.joint_select;
+    ccfg.Q = cfg.quantum_ns;
+    cfg.physical_gpus = nphys;
+    core.reset(new strings::Core(ccfg, this));
+    logical.resize(cfg.num_gpus);
+    for (int g = 0; g < cfg.num_gpus; ++g) logical[g].gid = g;
+    if (has_gpu()) {
+      strings_status_t s = init_gpus(nphys);
+      if (s != STRINGS_OK) {
+        teardown_gpus();
+        return s;
+      }
+    }
+    t0 = mono_ns();
+    engine = std::thread([this] { engine_main(); });
+    return STRINGS_OK;
+  }
+
+  strings_status_t init_gpus(int nphys) {
+    const int G = cfg.num_gpus;
+    for (int p = 0; p < nphys; ++p) {
+      auto ph = std::make_unique<Phys>();
+      ph->dev = p;
+      phys.push_back(std::move(ph));
+    }
+    for (int g = 0; g < G; ++g) {
+      Phys* ph = phys[g % nphys].get();
+      logical[g].phys = ph;
+      logical[g].local = ph->L++;
+    }
+    for (auto& ph : phys) {
+      if (ph->L == 0) continue;
+      if (!cuda_ok(cudaSetDevice(ph->dev))) return STRINGS_ECUDA;
+      cudaDeviceProp prop;
+      if (!cuda_ok(cudaGetDeviceProperties(&prop, ph->dev))) return STRINGS_ECUDA;
+      ph->sms = prop.multiProcessorCount;
+      if (ph->L * cfg.partitions > ph->sms) return STRINGS_EINVAL;
+      // host-mapped control block
+      size_t cb = strings_dev::host_ctrl_bytes(ph->L);
+      void* hp = nullptr;
+      if (!cuda_ok(cudaHostAlloc(&hp, cb, cudaHostAllocMapped | cudaHostAllocPortable)))
+        return STRINGS_ENOMEM;
+      memset(hp, 0, cb);
+      ph->ctrl = static_cast<HostCtrl*>(hp);
+      if (!cuda_ok(cudaHostGetDevicePointer(&ph->ctrl_dev, hp, 0))) return STRINGS_ECUDA;
+      // device state: heads[L] (padded) + parts[L*P]
+      size_t heads_bytes = 128 * (size_t)ph->L;
+      size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
+      if (!cuda_ok(cudaMalloc(&ph->dev_state, heads_bytes + parts_bytes))) return STRINGS_ENOMEM;
+      if (!cuda_ok(cudaMemset(ph->dev_state, 0, heads_bytes + parts_bytes))) return STRINGS_ECUDA;
+      // arena: L logical devices x M slots
+      size_t arena = (size_t)ph->L * cfg.admit_cap * cfg.slot_bytes;
+      if (!cuda_ok(cudaMalloc(&ph->arena, arena))) return STRINGS_ENOMEM;
+      ph->arena_owned = true;
+      if (!cuda_ok(cudaStreamCreateWithFlags(&ph->kstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+      uint8_t* base = static_cast<uint8_t*>(hp) + sizeof(HostCtrl);
+      KlRing* rings = reinterpret_cast<KlRing*>(base);
+      KlDone* dones = reinterpret_cast<KlDone*>(base + sizeof(KlRing) * ph->L);
+      for (auto& lg : logical) {
+        if (lg.phys != ph.get()) continue;
+        if (!cuda_ok(cudaStreamCreateWithFlags(&lg.h2d, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        if (!cuda_ok(cudaStreamCreateWithFlags(&lg.d2h, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        if (kl_mode == 1) {
+          lg.kl_streams.resize(cfg.partitions);
+          for (auto& s : lg.kl_streams)
+            if (!cuda_ok(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        }
+        lg.arena = ph->arena + (size_t)lg.local * cfg.admit_cap * cfg.slot_bytes;
+        for (int s = cfg.admit_cap - 1; s >= 0; --s) lg.free_slots.push_back(s);
+        lg.ring = rings + lg.local;
+        lg.done = dones + (size_t)lg.local * kRing;
+      }
+      for (int i = 0; i < 8 * cfg.awake_budget * ph->L + 16; ++i) {
+        cudaEvent_t e;
+        if (!cuda_ok(cudaEventCreateWithFlags(&e, cudaEventDisableTiming))) return STRINGS_ECUDA;
+        ph->ev_pool.push_back(e);
+      }
+      if (kl_mode == 0) {
+        strings_dev::DispatchParams dp;
+        uint8_t* dbase = static_cast<uint8_t*>(ph->ctrl_dev);
+        dp.ctrl = reinterpret_cast<HostCtrl*>(dbase);
+        dp.rings = reinterpret_cast<KlRing*>(dbase + sizeof(HostCtrl));
+        dp.done = reinterpret_cast<KlDone*>(dbase + sizeof(HostCtrl) + sizeof(KlRing) * ph->L);
+        dp.heads = reinterpret_cast<uint32_t*>(ph->dev_state);
+        dp.parts = reinterpret_cast<strings_dev::PartState*>(ph->dev_state + heads_bytes);
+        dp.L = ph->L;
+        dp.P = cfg.partitions;
+        if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
+        ph->kernel_running = true;
+      }
+    }
+    return STRINGS_OK;
+  }
+
+  void teardown_gpus() {
+    for (auto& ph : phys) {
+      if (ph->L == 0) continue;
+      cudaSetDevice(ph->dev);
+      if (ph->kernel_running) {
+        ph->ctrl->shutdown = 1;
+        std::atomic_thread_fence(std::memory_order_seq_cst);
+        cudaStreamSynchronize(ph->kstream);
+        ph->kernel_running = false;
+      }
+      for (auto& lg : logical) {
+        if (lg.phys != ph.get()) continue;
+        if (lg.h2d) cudaStreamSynchronize(lg.h2d), cudaStreamDestroy(lg.h2d);
+        if (lg.d2h) cudaStreamSynchronize(lg.d2h), cudaStreamDestroy(lg.d2h);
+        for (auto s : lg.kl_streams) cudaStreamSynchronize(s), cudaStreamDestroy(s);
+        lg.h2d = lg.d2h = nullptr;
+        lg.kl_streams.clear();
+      }
+      for (auto e : ph->ev_pool) cudaEventDestroy(e);
+      ph->ev_pool.clear();
+      if (ph->kstream) cudaStreamDestroy(ph->kstream);
+      if (ph->arena && ph->arena_owned) cudaFree(ph->arena);
+      if (ph->dev_state) cudaFree(ph->dev_state);
+      if (ph->ctrl) cudaFreeHost(ph->ctrl);
+      ph->kstream = nullptr;
+      ph->arena = nullptr;
+      ph->dev_state = nullptr;
+      ph->ctrl = nullptr;
+    }
+  }
+
+  // ------------------------------------------------------------- hooks
+  void fail_job(JobCtx* jc) {
+    if (jc->status == STRINGS_EAGAIN || jc->status == STRINGS_OK) jc->status = STRINGS_EFAULT;
+  }
+
+  void on_wake(strings::Job& j, int engine, uint64_t) override {
+    JobCtx* jc = static_cast<JobCtx*>(j.user);
+    if (!has_gpu()) {
+      jc->phys_done[engine] = true;
+      return;
+    }
+    Logical& lg = logical[j.gid];
+    Phys* ph = lg.phys;
+    cudaSetDevice(ph->dev);
+    bool ok = true;
+    if (engine == strings::ENG_H2D) {
+      if (jc->slot < 0) {
+        jc->slot = lg.free_slots.back();
+        lg.free_slots.pop_back();
+        uint8_t* base = lg.arena + (size_t)jc->slot * cfg.slot_bytes;
+        uint64_t off = 0;
+        for (size_t i = 0; i < jc->in.size(); ++i) {
+          jc->dev_in[i] = reinterpret_cast<uint64_t>(base + off);
+          off = align_up(off + jc->in[i].bytes);
+        }
+        jc->dev_out = reinterpret_cast<uint64_t>(base + off);
+      }
+      for (size_t i = 0; i < jc->in.size() && ok; ++i)
+        if (jc->in[i].bytes)
+          ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma,
+                                       jc->in[i].bytes, cudaMemcpyHostToDevice, lg.h2d));
+      jc->ev[engine] = take_event(ph);
+      ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], lg.h2d));
+    } else if (engine == strings::ENG_D2H) {
+      uint64_t off = 0;
+      for (size_t i = 0; i < jc->out.size() && ok; ++i) {
+        if (jc->out[i].bytes)
+          ok = cuda_ok(cudaMemcpyAsync(jc->out[i].dma, reinterpret_cast<void*>(jc->dev_out + off),
+                                       jc->out[i].bytes, cudaMemcpyDeviceToHost, lg.d2h));
+        off = align_up(off + jc->out[i].bytes);
+      }
+      jc->ev[engine] = take_event(ph);
+      ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], lg.d2h));
+    } else {
+      KlItem it;
+      memset(&it, 0, sizeof it);
+      it.kclass = jc->desc.kclass;
+      it.job = j.id;
+      it.in0 = jc->dev_in[0];
+      it.in1 = jc->dev_in[1];
+      it.out0 = jc->dev_out;
+      it.n = jc->desc.n;
+      it.m = jc->desc.m;
+      it.k = jc->desc.k;
+      it.reps = jc->desc.reps ? jc->desc.reps : 1;
+      it.alpha = jc->desc.alpha;
+      it.seed = jc->desc.seed;
+      if (kl_mode == 0) {
+        if (lg.tail - lg.completed >= (uint32_t)kRing) {
+          ok = false;  // cannot happen with A <= kRing; treat as a job fault
+        } else {
+          const uint32_t idx = lg.tail % kRing;
+          it.seq = lg.tail + 1;
+          KlItem* dst = &lg.ring->items[idx];
+          memcpy(dst, &it, sizeof it);
+          jc->kl_seq = it.seq;
+          jc->kl_idx = (int)idx;
+          std::atomic_thread_fence(std::memory_order_seq_cst);
+          lg.tail += 1;
+          lg.ring->tail = lg.tail;
+          std::atomic_thread_fence(std::memory_order_seq_cst);
+        }
+      } else {
+        cudaStream_t s = lg.kl_streams[lg.next_kl_stream];
+        lg.next_kl_stream = (lg.next_kl_stream + 1) % (int)lg.kl_streams.size();
+        int ctas = ph->sms / (ph->L * cfg.partitions);
+        ok = cuda_ok(strings::launch_oneshot(it, ctas, s));
+        jc->ev[engine] = take_event(ph);
+        ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], s));
+      }
+    }
+    jc->issued[engine] = true;
+    if (!ok) {
+      fail_job(jc);
+      jc->phys_done[engine] = true;   // a failed op completes immediately (fault localised)
+    }
+    if (!virtual_clock()) inflight.push_back({jc, engine});
+  }
+
+  void on_start(strings::Job& j, int engine, int slot, uint64_t t) override {
+    if (virtual_clock()) {
+      strings::Completion c{t + j.dur[engine], j.gid, engine, slot, j.id};
+      vheap.push({c.t, c});
+    }
+  }
+
+  void on_job_done(strings::Job& j, uint64_t t) override {
+    JobCtx* jc = static_cast<JobCtx*>(j.user);
+    if (has_gpu()) {
+      Logical& lg = logical[j.gid];
+      for (auto& o : jc->out)
+        if (o.staged && o.bytes) memcpy(o.user, o.dma, o.bytes);
+      for (auto* v : {&jc->in, &jc->out})
+        for (auto& b : *v)
+          if (b.staged && b.dma) {
+            cudaFreeHost(b.dma);
+            b.dma = nullptr;
+          }
+      if (jc->slot >= 0) {
+        lg.free_slots.push_back(jc->slot);
+        jc->slot = -1;
+      }
+    }
+    if (jc->status == STRINGS_EAGAIN) jc->status = STRINGS_OK;
+    Tenant& tn = tenants[j.tenant];
+    tn.outstanding -= 1;
+    if (jc->status != STRINGS_OK) {
+      tn.failed += 1;
+      failed_count += 1;
+    }
+    done_count += 1;
+    last_done = t;
+    cv_done.notify_all();
+  }
+
+  cudaEvent_t take_event(Phys* ph) {
+    if (ph->ev_pool.empty()) {
+      cudaEvent_t e;
+      if (!cuda_ok(cudaEventCreateWithFlags(&e, cudaEventDisableTiming))) return nullptr;
+      return e;
+    }
+    cudaEvent_t e = ph->ev_pool.back();
+    ph->ev_pool.pop_back();
+    return e;
+  }
+  void give_event(JobCtx* jc, int engine) {
+    if (jc->ev[engine]) {
+      logical[jc->job.gid].phys->ev_pool.push_back(jc->ev[engine]);
+      jc->ev[engine] = nullptr;
+    }
+  }
+
+  // Physical completion test of an issued op (non-blocking).
+  bool phys_complete(JobCtx* jc, int engine) {
+    if (jc->phys_done[engine]) return true;
+    if (!jc->issued[engine]) return false;
+    Logical& lg = logical[jc->job.gid];
+    if (engine == strings::ENG_KL && kl_mode == 0) {
+      volatile KlDone* d = &lg.done[jc->kl_idx];
+      if (d->seq != jc->kl_seq) return false;
+      std::atomic_thread_fence(std::memory_order_acquire);
+      jc->kl_partition = (int)d->partition;
+      jc->kl_t0 = d->t_start;
+      jc->kl_t1 = d->t_end;
+      lg.completed += 1;
+      jc->phys_done[engine] = true;
+      return true;
+    }
+    cudaSetDevice(lg.phys->dev);
+    cudaError_t e = cudaEventQuery(jc->ev[engine]);
+    if (e == cudaErrorNotReady) return false;
+    if (e != cudaSuccess) {
+      cuda_ok(e);
+      fail_job(jc);
+    }
+    give_event(jc, engine);
+    jc->phys_done[engine] = true;
+    return true;
+  }
+
+  // ------------------------------------------------------------- engine
+  void take_inbox(std::vector<JobCtx*>& out) {
+    out.swap(inbox);
+    inbox.clear();
+  }
+
+  void engine_main() {
+    std::vector<JobCtx*> news;
+    std::unique_lock<std::mutex> lk(mu);
+    while (!stop) {
+      if (virtual_clock()) {
+        if (!sealed || (inbox.empty() && core->unfinished() == 0)) {
+          cv_engine.wait_for(lk, std::chrono::milliseconds(50));
+          continue;
+        }
+        take_inbox(news);
+        for (JobCtx* jc : news) core->add_job(&jc->job);
+        news.clear();
+        virtual_step(lk);
+      } else {
+        if (inbox.empty() && core->unfinished() == 0) {
+          cv_engine.wait_for(lk, std::chrono::milliseconds(50));
+          continue;
+        }
+        measured_step(lk);
+      }
+    }
+  }
+
+  // One virtual timestamp in INJECTED / DECISIONS_ONLY mode.
+  void virtual_step(std::unique_lock<std::mutex>& lk) {
+    if (core->unfinished() == 0) return;
+    uint64_t t = UINT64_MAX;
+    if (!vheap.empty()) t = vheap.top().t;
+    if (core->has_pending_arrival()) t = std::min(t, core->next_arrival());
+    if (t == UINT64_MAX) {
+      fatal = STRINGS_ESTATE;          // deadlock: cannot happen with A, M >= 1
+      stop = true;
+      cv_done.notify_all();
+      return;
+    }
+    t = std::min(t, core->next_epoch());
+    bool first = true;
+    for (;;) {
+      std::vector<strings::Completion> batch;
+      while (!vheap.empty() && vheap.top().t == t) {
+        batch.push_back(vheap.top().c);
+        vheap.pop();
+      }
+      // release each DONE only after the physical op completed (virtual time
+      // decides, the GPU still does the work)
+      for (auto& c : batch) {
+        JobCtx* jc = jobs[c.job].get();
+        while (!phys_complete(jc, c.engine)) {
+          lk.unlock();
+          std::this_thread::yield();
+          lk.lock();
+        }
+      }
+      core->step(t, std::move(batch), first);
+      first = false;
+      if (vheap.empty() || vheap.top().t != t) break;
+    }
+  }
+
+  // One real-time batch in MEASURED mode.
+  void measured_step(std::unique_lock<std::mutex>& lk) {
+    std::vector<JobCtx*> news;
+    take_inbox(news);
+    uint64_t t = now();
+    if (t <= core->current_time()) t = core->current_time() + 1;
+    for (JobCtx* jc : news) {
+      jc->job.arrival = t;
+      core->add_job(&jc->job);
+    }
+    core->close_epochs_before(t);
+    bool first = true;
+    bool progressed = !news.empty();
+    for (;;) {
+      std::vector<strings::Completion> batch;
+      for (size_t i = 0; i < inflight.size();) {
+        JobCtx* jc = inflight[i].first;
+        int e = inflight[i].second;
+        strings::Job& j = jc->job;
+        // report only ops the core has started: an op queued behind a FIFO
+        // predecessor may finish physically in the same poll; it is reported
+        // in the next iteration, after its START
+        const bool started = j.phase == e && j.slot[e] >= 0;
+        if (started && phys_complete(jc, e)) {
+          batch.push_back({t, j.gid, e, j.slot[e], j.id});
+          inflight[i] = inflight.back();
+          inflight.pop_back();
+        } else {
+          ++i;
+        }
+      }
+      if (batch.empty() && !first) break;
+      if (batch.empty() && !progressed && core->next_epoch() != t) break;
+      core->step(t, std::move(batch), first);
+      first = false;
+      progressed = false;
+    }
+    if (!progressed) {
+      lk.unlock();
+      std::this_thread::yield();
+      lk.lock();
+    }
+  }
+
+  // ------------------------------------------------------------ API impl
+  strings_status_t submit(strings_tenant_t t, const strings_kernel_desc_t* d, const strings_buf_t* h2d,
+                          int32_t n_h2d, const strings_buf_t* d2h, int32_t n_d2h, uint32_t prio,
+                          strings_job_t* out) {
+    if (!d) return STRINGS_EINVAL;
+    std::vector<uint64_t> need_in, need_out;
+    switch (d->kclass) {
+      case STRINGS_VSCALE:
+      case STRINGS_XFER:
+        need_in = {4 * d->n};
+        need_out = {4 * d->n};
+        break;
+      case STRINGS_GEMM:
+        if (d->m == 0 || d->n == 0 || d->k == 0 || d->m % 128 || d->n % 256 || d->k % 64 || d->k > 256 ||
+            d->reps == 0)
+          return STRINGS_EINVAL;
+        need_in = {2 * d->m * d->k, 2 * d->k * d->n};
+        need_out = {4 * d->m * d->n};
+        break;
+      default:
+        return STRINGS_EINVAL;
+    }
+    if (n_h2d != (int32_t)need_in.size() || n_d2h != (int32_t)need_out.size()) return STRINGS_EINVAL;
+    uint64_t slot_need = 0;
+    for (int i = 0; i < n_h2d; ++i) {
+      if (h2d[i].bytes != need_in[i] || (h2d[i].bytes && !h2d[i].host)) return STRINGS_EINVAL;
+      slot_need = align_up(slot_need + h2d[i].bytes);
+    }
+    for (int i = 0; i < n_d2h; ++i) {
+      if (d2h[i].bytes != need_out[i] || (d2h[i].bytes && !d2h[i].host)) return STRINGS_EINVAL;
+      slot_need = align_up(slot_need + d2h[i].bytes);
+    }
+    if (slot_need > cfg.slot_bytes) return STRINGS_EINVAL;
+    auto jc = std::make_unique<JobCtx>();
+    jc->desc = *d;
+    // PMT: stage pageable buffers through pinned memory (MOT)
+    auto prep = [&](const strings_buf_t& b, bool is_in, HostBuf& hb) -> strings_status_t {
+      hb.user = b.host;
+      hb.bytes = b.bytes;
+      hb.dma = b.host;
+      if (!has_gpu() || b.bytes == 0) return STRINGS_OK;
+      cudaPointerAttributes a;
+      cudaError_t e = cudaPointerGetAttributes(&a, b.host);
+      if (e != cudaSuccess) cudaGetLastError();
+      bool pinned = e == cudaSuccess && a.type == cudaMemoryTypeHost;
+      if (pinned) return STRINGS_OK;
+      void* p = nullptr;
+      if (!cuda_ok(cudaHostAlloc(&p, b.bytes, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+      if (is_in) memcpy(p, b.host, b.bytes);
+      hb.dma = p;
+      hb.staged = true;
+      return STRINGS_OK;
+    };
+    jc->in.resize(n_h2d);
+    jc->out.resize(n_d2h);
+    for (int i = 0; i < n_h2d; ++i)
+      if (strings_status_t s = prep(h2d[i], true, jc->in[i])) return s;
+    for (int i = 0; i < n_d2h; ++i)
+      if (strings_status_t s = prep(d2h[i], false, jc->out[i])) return s;
+    std::lock_guard<std::mutex> g(mu);
+    if (fatal != STRINGS_OK) return fatal;
+    if (t >= tenants.size() || !tenants[t].active) return STRINGS_EINVAL;
+    if (virtual_clock() && sealed && d->arrival_ns < core->current_time()) return STRINGS_EINVAL;
+    strings::Job& j = jc->job;
+    j.id = jobs.size();
+    j.tenant = t;
+    j.seq = tenants[t].next_seq++;
+    j.prio = prio ? prio : tenants[t].weight;
+    j.kclass = (int)d->kclass;
+    j.arrival = virtual_clock() ? d->arrival_ns : 0;
+    for (int i = 0; i < n_h2d; ++i) j.h2d_bytes += h2d[i].bytes;
+    for (int i = 0; i < n_d2h; ++i) j.d2h_bytes += d2h[i].bytes;
+    strings::class_bytes_flop(j.kclass, d->n, d->m, d->k, d->reps ? d->reps : 1, &j.hbm_bytes, &j.flop);
+    j.dur[0] = d->inj_h2d_ns;
+    j.dur[1] = d->inj_kl_ns;
+    j.dur[2] = d->inj_d2h_ns;
+    j.user = jc.get();
+    tenants[t].outstanding += 1;
+    submitted += 1;
+    if (submitted == 1) first_submit = virtual_clock() ? j.arrival : now();
+    h2d_total += j.h2d_bytes;
+    d2h_total += j.d2h_bytes;
+    kbytes_total += j.hbm_bytes;
+    kflop_total += j.flop;
+    if (out) *out = j.id;
+    inbox.push_back(jc.get());
+    jobs.push_back(std::move(jc));
+    cv_engine.notify_all();
+    return STRINGS_OK;
+  }
+
+  strings_status_t wait_tenant(int64_t t) {
+    std::unique_lock<std::mutex> lk(mu);
+    sealed = true;
+    cv_engine.notify_all();
+    for (;;) {
+      if (fatal != STRINGS_OK) return fatal;
+      uint64_t out = 0, failed = 0;
+      if (t < 0) {
+        for (auto& tn : tenants) out += tn.outstanding, failed += tn.failed;
+      } else {
+        out = tenants[t].outstanding;
+        failed = tenants[t].failed;
+      }
+      if (out == 0) return failed ? STRINGS_EFAULT : STRINGS_OK;
+      cv_done.wait_for(lk, std::chrono::milliseconds(20));
+    }
+  }
+
+  void flush_trace() {
+    if (!cfg.trace_path) return;
+    FILE* f = fopen(cfg.trace_path, "w");
+    if (!f) return;
+    fwrite(core->trace().data(), 1, core->trace().size(), f);
+    fclose(f);
+  }
+
+  void shutdown() {
+    {
+      std::lock_guard<std::mutex> g(mu);
+      stop = true;
+      cv_engine.notify_all();
+    }
+    if (engine.joinable()) engine.join();
+    flush_trace();
+    if (has_gpu()) teardown_gpus();
+  }
+};
+
+}  // namespace
+
+// =================================================================== C ABI
+extern "C" {
+
+strings_status_t strings_init(const strings_config_t* cfg) {
+  std::lock_guard<std::mutex> g(g_init_mu);
+  if (g_rt) return STRINGS_ESTATE;
+  auto* rt = new Runtime();
+  strings_status_t s = rt->init(cfg);
+  if (s != STRINGS_OK) {
+    delete rt;
+    return s;
+  }
+  g_rt = rt;
+  return STRINGS_OK;
+}
+
+strings_status_t strings_register_tenant(uint32_t weight, uint32_t max_inflight, strings_tenant_t* out) {
+  if (!g_rt) return STRINGS_ESTATE;
+  if (weight == 0 || max_inflight == 0 || !out) return STRINGS_EINVAL;
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  Tenant t;
+  t.weight = weight;
+  t.c = max_inflight;
+  g_rt->tenants.push_back(t);
+  int id = g_rt->core->add_tenant(weight, max_inflight);
+  *out = (strings_tenant_t)id;
+  return STRINGS_OK;
+}
+
+strings_status_t strings_submit(strings_tenant_t tenant, const strings_kernel_desc_t* desc,
+                                const strings_buf_t* h2d, int32_t n_h2d, const strings_buf_t* d2h,
+                                int32_t n_d2h, uint32_t priority, strings_job_t* out) {
+  if (!g_rt) return STRINGS_ESTATE;
+  return g_rt->submit(tenant, desc, h2d, n_h2d, d2h, n_d2h, priority, out);
+}
+
+strings_status_t strings_sync(strings_tenant_t tenant) {
+  if (!g_rt) return STRINGS_ESTATE;
+  {
+    std::lock_guard<std::mutex> g(g_rt->mu);
+    if (tenant >= g_rt->tenants.size()) return STRINGS_EINVAL;
+  }
+  return g_rt->wait_tenant((int64_t)tenant);
+}
+
+strings_status_t strings_drain(void) {
+  if (!g_rt) return STRINGS_ESTATE;
+  strings_status_t s = g_rt->wait_tenant(-1);
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  g_rt->flush_trace();
+  return s;
+}
+
+strings_status_t strings_unregister_tenant(strings_tenant_t tenant) {
+  if (!g_rt) return STRINGS_ESTATE;
+  strings_status_t s = strings_sync(tenant);
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  if (tenant < g_rt->tenants.size()) g_rt->tenants[tenant].active = false;
+  return s == STRINGS_EFAULT ? s : STRINGS_OK;
+}
+
+strings_status_t strings_shutdown(void) {
+  std::lock_guard<std::mutex> g(g_init_mu);
+  if (!g_rt) return STRINGS_ESTATE;
+  g_rt->wait_tenant(-1);
+  g_rt->shutdown();
+  delete g_rt;
+  g_rt = nullptr;
+  return STRINGS_OK;
+}
+
+strings_status_t strings_host_alloc(uint64_t bytes, void** p) {
+  if (!p) return STRINGS_EINVAL;
+  if (!cuda_ok(cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+  return STRINGS_OK;
+}
+
+strings_status_t strings_host_free(void* p) {
+  if (!p) return STRINGS_OK;
+  return cuda_ok(cudaFreeHost(p)) ? STRINGS_OK : STRINGS_ECUDA;
+}
+
+strings_status_t strings_job_info(strings_job_t job, strings_job_info_t* info) {
+  if (!g_rt) return STRINGS_ESTATE;
+  if (!info) return STRINGS_EINVAL;
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  if (job >= g_rt->jobs.size()) return STRINGS_EINVAL;
+  JobCtx* jc = g_rt->jobs[job].get();
+  const strings::Job& j = jc->job;
+  memset(info, 0, sizeof *info);
+  info->job = j.id;
+  info->tenant = j.tenant;
+  info->seq = j.seq;
+  info->gid = j.placed ? j.gid : -1;
+  info->status = jc->status;
+  info->t_arrival = j.arrival;
+  info->t_place = j.t_place;
+  for (int x = 0; x < 3; ++x) {
+    info->t_start[x] = j.start[x];
+    info->t_done[x] = j.done[x];
+  }
+  info->kl_slot = j.slot[1];
+  info->kl_partition = jc->kl_partition;
+  info->kl_gpu_start_ns = jc->kl_t0;
+  info->kl_gpu_end_ns = jc->kl_t1;
+  return STRINGS_OK;
+}
+
+strings_status_t strings_get_stats(strings_stats_t* st) {
+  if (!g_rt) return STRINGS_ESTATE;
+  if (!st) return STRINGS_EINVAL;
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  memset(st, 0, sizeof *st);
+  Runtime& r = *g_rt;
+  st->jobs_submitted = r.submitted;
+  st->jobs_done = r.done_count;
+  st->jobs_failed = r.failed_count;
+  st->t_first_submit_ns = r.first_submit;
+  st->t_last_done_ns = r.last_done;
+  st->h2d_bytes = r.h2d_total;
+  st->d2h_bytes = r.d2h_total;
+  st->kernel_bytes = r.kbytes_total;
+  st->kernel_flop = r.kflop_total;
+  st->trace_records = r.core->trace_records();
+  st->decisions = r.core->decisions();
+  for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
+    for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
+  st->num_gpus = r.cfg.num_gpus;
+  st->physical_gpus = r.cfg.physical_gpus;
+  st->partitions = r.cfg.partitions;
+  if (!r.phys.empty() && r.phys[0]->L > 0) st->sms_per_partition = r.phys[0]->sms / (r.phys[0]->L * r.cfg.partitions);
+  return STRINGS_OK;
+}
+
+strings_status_t strings_trace_size(uint64_t* bytes) {
+  if (!g_rt) return STRINGS_ESTATE;
+  if (!bytes) return STRINGS_EINVAL;
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  *bytes = g_rt->core->trace().size();
+  return STRINGS_OK;
+}
+
+strings_status_t strings_trace_copy(char* buf, uint64_t capacity, uint64_t* written) {
+  if (!g_rt) return STRINGS_ESTATE;
+  if (!buf && capacity) return STRINGS_EINVAL;
+  std::lock_guard<std::mutex> g(g_rt->mu);
+  const std::string& t = g_rt->core->trace();
+  uint64_t n = std::min<uint64_t>(capacity, t.size());
+  memcpy(buf, t.data(), n);
+  if (written) *written = n;
+  return n == t.size() ? STRINGS_OK : STRINGS_EAGAIN;
+}
+
+const char* strings_strerror(strings_status_t s) {
+  switch (s) {
+    case STRINGS_OK: return "ok";
+    case STRINGS_EINVAL: return "invalid argument";
+    case STRINGS_ENOMEM: return "out of memory";
+    case STRINGS_EAGAIN: return "not ready";
+    case STRINGS_ECUDA: return "CUDA error";
+    case STRINGS_ESTATE: return "bad library state";
+    case STRINGS_EFAULT: return "a job of this tenant failed";
+  }
+  return "unknown status";
+}
+
+int32_t strings_last_cuda_error(void) { return g_last_cuda_error.load(); }
+
+const char* strings_version(void) { return "strings-b200 0.1 (sm_100a)"; }
+
+strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kernel_desc_t* desc,
+                                       void* const* dev_in, int32_t n_in, void* const* dev_out,
+                                       int32_t n_out, int32_t ctas, void* stream) {
+  if (!desc || !dev_in || !dev_out || n_out < 1) return STRINGS_EINVAL;
+  if (desc->kclass == STRINGS_GEMM) {
+    if (n_in < 2 || desc->m % 128 || desc->n % 256 || desc->k % 64 || desc->k > 256 || desc->k == 0 ||
+        desc->reps == 0)
+      return STRINGS_EINVAL;
+  } else if (desc->kclass != STRINGS_VSCALE && desc->kclass != STRINGS_XFER) {
+    return STRINGS_EINVAL;
+  } else if (n_in < 1) {
+    return STRINGS_EINVAL;
+  }
+  if (!cuda_ok(cudaSetDevice(physical_gpu))) return STRINGS_ECUDA;
+  if (ctas <= 0) {
+    cudaDeviceProp prop;
+    if (!cuda_ok(cudaGetDeviceProperties(&prop, physical_gpu))) return STRINGS_ECUDA;
+    ctas = prop.multiProcessorCount;
+  }
+  KlItem it;
+  memset(&it, 0, sizeof it);
+  it.kclass = desc->kclass;
+  it.in0 = reinterpret_cast<uint64_t>(dev_in[0]);
+  it.in1 = n_in > 1 ? reinterpret_cast<uint64_t>(dev_in[1]) : 0;
+  it.out0 = reinterpret_cast<uint64_t>(dev_out[0]);
+  it.n = desc->n;
+  it.m = desc->m;
+  it.k = desc->k;
+  it.reps = desc->reps ? desc->reps : 1;
+  it.alpha = desc->alpha;
+  it.seed = desc->seed;
+  return cuda_ok(strings::launch_oneshot(it, ctas, static_cast<cudaStream_t>(stream))) ? STRINGS_OK
+                                                                                      : STRINGS_ECUDA;
+}
+
+}  // extern "C"

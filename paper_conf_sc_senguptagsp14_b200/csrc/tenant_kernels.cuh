@@ -1,0 +1,325 @@
+// tenant_kernels.cuh -- the three tenant kernel classes as device functions.
+//
+// Each body runs on a group of S CTAs (one SM partition of the persistent
+// dispatcher, or a stand-alone grid); `rank` is this CTA's index in the group.
+// Block = 256 threads.  Classes follow the paper's workload classes (Table I,
+// PAPER.md L767-815) as made concrete in SURVEY.md §8(d):
+//   VSCALE  y = alpha * x            fp32, one __fmul_rn per element (R-23)
+//   XFER    y = fmix32(x ^ seed)     u32 (MurmurHash3 finaliser)
+//   GEMM    C = A . B, R repetitions bf16 -> fp32, tcgen05 + TMEM (R-17, R-22)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace strings_dev {
+
+constexpr int kThreads = 256;
+
+// One KL work item (also the layout of the host-mapped KL ring entries).
+struct __align__(16) KlItem {
+  uint32_t seq;          // claim number (1-based, monotone per ring); written last by the host
+  uint32_t kclass;
+  uint64_t job;
+  uint64_t in0, in1, out0;   // device pointers
+  uint64_t n, m, k;
+  uint32_t reps;
+  float alpha;
+  uint32_t seed;
+  uint32_t pad;
+};
+static_assert(sizeof(KlItem) == 80, "KlItem layout");
+
+// ---------------------------------------------------------------- streaming
+__device__ __forceinline__ uint32_t fmix32(uint32_t h) {
+  h ^= h >> 16;
+  h *= 0x85EBCA6Bu;
+  h ^= h >> 13;
+  h *= 0xC2B2AE35u;
+  h ^= h >> 16;
+  return h;
+}
+
+__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_stream(uint4* p, uint4 v) {
+  asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1,%2,%3,%4};"
+               :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+template <int KCLASS>
+__device__ __forceinline__ uint32_t elem_op(uint32_t x, float alpha, uint32_t seed) {
+  if constexpr (KCLASS == 0) return __float_as_uint(__fmul_rn(__uint_as_float(x), alpha));
+  else return fmix32(x ^ seed);
+}
+
+// Vectorised grid-stride stream over the group's CTAs: 8 independent 16-B
+// loads in flight per thread (32 KB per CTA) to cover HBM latency.
+template <int KCLASS>
+__device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
+                            float alpha, uint32_t seed, int rank, int S) {
+  constexpr int U = 8;
+  const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x;
+  const uint64_t nthreads = (uint64_t)S * kThreads;
+  const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
+  uint64_t nvec = aligned ? n / 4 : 0;
+  const uint4* xv = reinterpret_cast<const uint4*>(x);
+  uint4* yv = reinterpret_cast<uint4*>(y);
+  uint64_t i = tid;
+  for (; i + (U - 1) * nthreads < nvec; i += U * nthreads) {
+    uint4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) v[u] = ld_stream(xv + i + u * nthreads);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      v[u].x = elem_op<KCLASS>(v[u].x, alpha, seed);
+      v[u].y = elem_op<KCLASS>(v[u].y, alpha, seed);
+      v[u].z = elem_op<KCLASS>(v[u].z, alpha, seed);
+      v[u].w = elem_op<KCLASS>(v[u].w, alpha, seed);
+      st_stream(yv + i + u * nthreads, v[u]);
+    }
+  }
+  for (; i < nvec; i += nthreads) {
+    uint4 v = ld_stream(xv + i);
+    v.x = elem_op<KCLASS>(v.x, alpha, seed);
+    v.y = elem_op<KCLASS>(v.y, alpha, seed);
+    v.z = elem_op<KCLASS>(v.z, alpha, seed);
+    v.w = elem_op<KCLASS>(v.w, alpha, seed);
+    st_stream(yv + i, v);
+  }
+  for (uint64_t e = nvec * 4 + tid; e < n; e += nthreads) y[e] = elem_op<KCLASS>(x[e], alpha, seed);
+}
+
+// --------------------------------------------------------------------- GEMM
+// Tile 128 x 256 (M x N) per CTA, whole K (<= 256) resident in shared memory
+// in the UMMA canonical K-major SWIZZLE_NONE layout: a core matrix is 8 rows x
+// 16 B (8 bf16 along K) stored contiguously (128 B).
+//   A tile: core (row-group g in 0..15, k-chunk c) at (c*16 + g)*128   -> SBO = 128, LBO = 2048
+//   B tile: core (n-group g in 0..31, k-chunk c)   at (c*32 + g)*128   -> SBO = 128, LBO = 4096
+// (B is transposed while loading: smem holds B^T, K-major.)
+constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
+constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
+constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
+constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 64;     // + mbarrier / tmem slot
+constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// Shared-memory matrix descriptor (sm_100 UMMA): start>>4 [0,14), LBO>>4 [16,30),
+// SBO>>4 [32,46), version=1 [46,48), base offset 0, layout SWIZZLE_NONE (0) [61,64).
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
+  d |= (uint64_t)1 << 46;
+  return d;
+}
+
+// Instruction descriptor kind::f16: D=f32 [4,6)=1, A=bf16 [7,10)=1, B=bf16 [10,13)=1,
+// A,B K-major (bits 15,16 = 0), N>>3 at [17,23), M>>4 at [24,29).
+__host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t a = smem_u32(bar);
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}"
+      :: "r"(a), "r"(parity) : "memory");
+}
+
+__device__ __forceinline__ void tmem_alloc(uint32_t* slot_smem, uint32_t cols) {
+  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+               :: "r"(smem_u32(slot_smem)), "r"(cols) : "memory");
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t taddr, uint32_t cols) {
+  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(taddr), "r"(cols) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+
+__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+      :: "r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(accumulate) : "memory");
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+               :: "r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]),
+        "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]),
+        "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+struct GemmSmem {
+  uint8_t* a;          // kSmemA bytes, 128-B aligned
+  uint8_t* b;          // kSmemB bytes
+  uint64_t* bar;       // MMA-completion mbarrier
+  uint32_t* tmem_slot; // TMEM base written by tcgen05.alloc
+};
+
+// Load the A tile (rows m0..m0+127, all K) and B^T (cols n0..n0+255, all K)
+// into the canonical layouts above.  All 256 threads participate.
+__device__ inline void gemm_load_tile(const GemmSmem& sm, const uint16_t* __restrict__ A,
+                               const uint16_t* __restrict__ B, uint64_t N, uint64_t K, uint64_t m0,
+                               uint64_t n0) {
+  const int kchunks = (int)(K / 8);
+  // A: 16-B chunks (row r, k-chunk c) -> core (c, r/8), row r%8
+  for (int idx = threadIdx.x; idx < kTileM * kchunks; idx += kThreads) {
+    int r = idx / kchunks, c = idx % kchunks;
+    uint4 v = *reinterpret_cast<const uint4*>(A + (m0 + r) * K + (uint64_t)c * 8);
+    *reinterpret_cast<uint4*>(sm.a + ((c * 16 + (r >> 3)) * 128 + (r & 7) * 16)) = v;
+  }
+  // B^T: read B[k][n0 + 8q .. +7] (16 B along N), scatter to rows n of the K-major tile
+  for (int idx = threadIdx.x; idx < (int)K * (kTileN / 8); idx += kThreads) {
+    int k = idx / (kTileN / 8), q = idx % (kTileN / 8);
+    uint4 v = *reinterpret_cast<const uint4*>(B + (uint64_t)k * N + n0 + (uint64_t)q * 8);
+    const uint16_t* e = reinterpret_cast<const uint16_t*>(&v);
+    int c = k >> 3, kk = k & 7;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+      int n = q * 8 + t;
+      *reinterpret_cast<uint16_t*>(sm.b + ((c * 32 + (n >> 3)) * 128 + (n & 7) * 16 + kk * 2)) = e[t];
+    }
+  }
+  // make generic-proxy smem writes visible to the tensor core (async proxy)
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncthreads();
+}
+
+// Units u = tile * R + rep, tile = (mt, nt); this CTA takes the contiguous
+// chunk [rank*U/S, (rank+1)*U/S).  Each repetition is a full 16-MMA chain into
+// the TMEM accumulator; C is written from repetition R-1 (R-17).
+__device__ inline void gemm_body(const uint16_t* __restrict__ A, const uint16_t* __restrict__ B,
+                          float* __restrict__ C, uint64_t M, uint64_t N, uint64_t K, uint32_t R,
+                          int rank, int S, const GemmSmem& sm, uint32_t tmem_base,
+                          uint32_t& mma_phase) {
+  const uint64_t tiles_n = N / kTileN, tiles = (M / kTileM) * tiles_n;
+  const uint64_t U = tiles * R;
+  const uint64_t u0 = (U * rank) / S, u1 = (U * (rank + 1)) / S;
+  const uint32_t idesc = umma_idesc_bf16(kTileM, kTileN);
+  const uint32_t a_base = smem_u32(sm.a), b_base = smem_u32(sm.b);
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  uint64_t u = u0;
+  while (u < u1) {
+    const uint64_t tile = u / R;
+    const uint64_t last = min(u1, (tile + 1) * R);        // exclusive end of this tile's run
+    const uint64_t mt = tile / tiles_n, nt = tile % tiles_n;
+    gemm_load_tile(sm, A, B, N, K, mt * kTileM, nt * kTileN);
+    if (threadIdx.x == 0) {
+      tc_fence_after();
+      for (uint64_t v = u; v < last; ++v) {
+        for (uint32_t ks = 0; ks < K / 16; ++ks) {
+          uint64_t da = umma_desc(a_base + ks * 2 * 2048, 2048, 128);
+          uint64_t db = umma_desc(b_base + ks * 2 * 4096, 4096, 128);
+          umma_bf16(tmem_base, da, db, idesc, ks > 0 ? 1u : 0u);
+        }
+      }
+      umma_commit(sm.bar);            // arrives when every MMA above has completed
+    }
+    __syncwarp();
+    mbar_wait(sm.bar, mma_phase);
+    mma_phase ^= 1;
+    tc_fence_after();
+    if ((last - 1) % R == R - 1) {    // this run contains the final repetition: epilogue
+      const int lane_base = (warp & 3) * 32;
+      const int col0 = (warp >> 2) * 128;
+      const uint64_t row = mt * kTileM + lane_base + lane;
+      float* crow = C + row * N + nt * kTileN;
+#pragma unroll 1
+      for (int cc = 0; cc < 128; cc += 32) {
+        uint32_t r[32];
+        tmem_ld32(tmem_base + ((uint32_t)lane_base << 16) + (uint32_t)(col0 + cc), r);
+        float4* dst = reinterpret_cast<float4*>(crow + col0 + cc);
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          dst[q] = make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]),
+                               __uint_as_float(r[4 * q + 2]), __uint_as_float(r[4 * q + 3]));
+      }
+    }
+    tc_fence_before();
+    __syncthreads();                  // smem and TMEM free for the next run
+    u = last;
+  }
+}
+
+// Run one work item on this CTA (rank of S).
+__device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, const GemmSmem& sm,
+                                         uint32_t tmem_base, uint32_t& mma_phase) {
+  switch (it.kclass) {
+    case 0:
+      stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
+                     it.n, it.alpha, it.seed, rank, S);
+      break;
+    case 2:
+      stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
+                     it.n, it.alpha, it.seed, rank, S);
+      break;
+    case 1:
+      gemm_body(reinterpret_cast<const uint16_t*>(it.in0), reinterpret_cast<const uint16_t*>(it.in1),
+                reinterpret_cast<float*>(it.out0), it.m, it.n, it.k, it.reps, rank, S, sm, tmem_base,
+                mma_phase);
+      break;
+  }
+}
+
+__device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
+  GemmSmem s;
+  s.a = base;
+  s.b = base + kSmemA;
+  s.bar = reinterpret_cast<uint64_t*>(base + kSmemA + kSmemB);
+  s.tmem_slot = reinterpret_cast<uint32_t*>(base + kSmemA + kSmemB + 16);
+  return s;
+}
+
+// CTA prologue / epilogue shared by every kernel that may run a GEMM item.
+__device__ __forceinline__ uint32_t cta_setup(const GemmSmem& sm) {
+  if (threadIdx.x / 32 == 0) tmem_alloc(sm.tmem_slot, kTmemCols);
+  if (threadIdx.x == 32) {
+    mbar_init(sm.bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  return *sm.tmem_slot;
+}
+__device__ __forceinline__ void cta_teardown(uint32_t tmem_base) {
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (threadIdx.x / 32 == 0) tmem_dealloc(tmem_base, kTmemCols);
+}
+
+}  // namespace strings_dev

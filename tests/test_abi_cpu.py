@@ -1,0 +1,143 @@
+"""C-ABI library on a host without a GPU: symbols, loud failure, host-logic parity.
+
+The decision core (C++, libstrings_sched.so) is host logic; DECISIONS_ONLY mode
+replays it without any device work so its traces can be compared with the
+independent CPU oracle here.  Product timing modes must fail loudly (ECUDA)
+when no CUDA device exists.
+"""
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+import pytest
+
+import strings_workload as W
+from oracle import invariants
+from oracle.des import run_oracle
+from paper_conf_sc_senguptagsp14_b200 import strings as S
+from paper_conf_sc_senguptagsp14_b200.runner import run_workload
+
+
+def _has_gpu():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except Exception:
+        return False
+
+
+def test_library_exports_every_declared_symbol():
+    declared = S.declared_symbols()
+    assert len(declared) >= 17
+    out = subprocess.run(["nm", "-D", "--defined-only", S.LIB_PATH], capture_output=True, text=True,
+                         check=True).stdout
+    exported = {ln.split()[-1] for ln in out.splitlines() if " T " in ln}
+    missing = [s for s in declared if s not in exported]
+    assert missing == []
+    for s in declared:
+        assert hasattr(S.lib, s)
+
+
+def test_version_and_strerror():
+    assert "sm_100a" in S.version()
+    assert S.strerror(S.EINVAL) == "invalid argument"
+    assert S.strerror(S.EFAULT).startswith("a job")
+
+
+@pytest.mark.skipif(_has_gpu(), reason="checks the no-GPU failure path")
+def test_product_modes_fail_loudly_without_gpu():
+    for mode in (S.MEASURED, S.INJECTED):
+        with pytest.raises(S.StringsError) as e:
+            S.init(timing_mode=mode)
+        assert e.value.status == S.ECUDA
+
+
+def test_calls_before_init_are_rejected():
+    assert S.lib.strings_sync(0) == S.ESTATE
+    assert S.lib.strings_drain() == S.ESTATE
+    assert S.lib.strings_shutdown() == S.ESTATE
+
+
+def test_argument_validation():
+    S.init(num_gpus=1, timing_mode=S.DECISIONS_ONLY)
+    try:
+        t = S.register_tenant(1, 1)
+        x = np.zeros(16, np.float32)
+        y = np.zeros(16, np.float32)
+        with pytest.raises(S.StringsError):                      # wrong byte count
+            S.submit(t, S.make_desc(S.VSCALE, n=8), [x], [y])
+        with pytest.raises(S.StringsError):                      # unknown tenant
+            S.submit(t + 5, S.make_desc(S.VSCALE, n=16), [x], [y])
+        a = np.zeros((128, 64), np.uint16)
+        b = np.zeros((64, 200), np.uint16)
+        c = np.zeros((128, 200), np.float32)
+        with pytest.raises(S.StringsError):                      # n % 256 != 0
+            S.submit(t, S.make_desc(S.GEMM, m=128, n=200, k=64), [a, b], [c])
+        with pytest.raises(S.StringsError):                      # missing buffer
+            S.submit(t, S.make_desc(S.GEMM, m=128, n=256, k=64), [a], [c])
+        with pytest.raises(S.StringsError):
+            S.submit(t, S.make_desc(7, n=16), [x], [y])
+        assert S.sync(t) == S.OK
+        with pytest.raises(S.StringsError):
+            S.register_tenant(0, 1)
+    finally:
+        S.shutdown()
+    with pytest.raises(S.StringsError):
+        S.init(balancer=11, timing_mode=S.DECISIONS_ONLY)
+
+
+@pytest.mark.parametrize("name", list(W.CONFIGS))
+def test_decision_core_trace_matches_oracle_on_configs(name):
+    wl = W.CONFIGS[name]()
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+    assert r.status == S.OK
+    assert r.trace == o.trace
+    assert r.stats.jobs_done == len(wl.jobs)
+
+
+@pytest.mark.parametrize("seed", range(150))
+def test_decision_core_trace_matches_oracle_on_random_workloads(seed):
+    wl = W.random_workload(seed)
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+    assert r.trace == o.trace
+
+
+def test_decision_core_job_records_match_oracle():
+    wl = W.config_c4(jobs_per_tenant=4)
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+    for j, info in zip(o.jobs, r.infos):
+        assert info.gid == j.gid
+        assert list(info.t_start) == j.start and list(info.t_done) == j.done
+        assert info.status == S.OK
+    assert invariants.check(r.trace, wl) == []
+
+
+def test_trace_file_written(tmp_path):
+    wl = W.config_c1()
+    p = tmp_path / "trace.txt"
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY, trace_path=str(p))
+    assert p.read_text().splitlines() == r.trace
+
+
+def test_sync_per_tenant_and_unregister():
+    S.init(num_gpus=2, timing_mode=S.DECISIONS_ONLY)
+    try:
+        ts = [S.register_tenant(1, 1) for _ in range(3)]
+        dummy = np.zeros(16, np.uint8)
+        for t in ts:
+            for s in range(4):
+                d = S.make_desc(S.VSCALE, n=1 << 20, arrival_ns=0, inj=(1000 * (t + 1), 500, 1000))
+                S.submit(t, d, [S.HostRef(dummy.ctypes.data, 4 << 20)], [S.HostRef(dummy.ctypes.data, 4 << 20)])
+        assert S.sync(ts[0]) == S.OK
+        assert S.unregister_tenant(ts[1]) == S.OK
+        with pytest.raises(S.StringsError):
+            S.submit(ts[1], S.make_desc(S.VSCALE, n=4), [np.zeros(4, np.float32)], [np.zeros(4, np.float32)])
+        assert S.drain() == S.OK
+        st = S.stats()
+        assert st.jobs_done == 12 and st.jobs_failed == 0
+    finally:
+        S.shutdown()
