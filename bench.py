@@ -1,0 +1,457 @@
+#!/usr/bin/env python
+"""Benchmark: tenant jobs/sec of the Strings scheduler hot path on B200.
+
+Workload (BASELINE.json configs[1], the single-GPU config):
+C2 = 16 tenants (8 GEMM 256^3 R=64 + 8 XFER 2^24 u32), 8 jobs each, DTF
+placement (joint selection), PS dispatch, MEASURED timing.  One "step" = the
+whole hot path (submit -> balancer -> H2D -> persistent-kernel KL -> D2H ->
+completion) over the 128 jobs of one C2 batch.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+
+N > 1 runs under torchrun, one process per GPU; tenants are independent, so
+each rank runs its own C2 batch on its own GPU (weak scaling, no collective
+on the data path; rank timings are combined with a max over a CPU group).
+
+JSON line keys beyond the base contract:
+  roofline         dominant resource of the step = the host link (copy engines)
+  overlapped_roofline   T*_d / span per SURVEY.md §8(d) with the measured peaks
+  kernel_rooflines tenant kernels timed stand-alone (HBM GB/s, tensor TFLOP/s)
+  static_baseline  one process per tenant, synchronous copies (reading R-18)
+  cpu_baseline     the oracle (oracle/) on a bounded sample, on the host cores
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "tenant jobs/sec (8xB200) vs static CUDA provisioning; Jain fairness"
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="strings", choices=["strings", "reference"])
+    p.add_argument("--jobs-per-tenant", type=int, default=8)
+    p.add_argument("--no-static", action="store_true")
+    p.add_argument("--no-kernels", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--kl-mode", type=int, default=0, help="0 persistent dispatcher, 1 per-job launches (ncu)")
+    p.add_argument("--trace-out", default=None)
+    return p.parse_args()
+
+
+# ----------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except FileNotFoundError:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            self.p.wait(timeout=10)
+
+    def summary(self) -> dict:
+        self.f.seek(0)
+        rows = [r.split(",") for r in self.f.read().strip().splitlines() if r.strip()]
+        sm = [float(r[1]) for r in rows if len(r) > 8 and r[1].strip().replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) > 8 and r[2].strip().replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            if len(r) > 8:
+                for n, v in zip(names, r[5:9]):
+                    if v.strip().lower() == "active":
+                        reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+# ------------------------------------------------------------- peaks
+def measured_peaks() -> dict:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained"), "source": "MEASURED_PEAKS.json"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+            "source": "fallback (B200_PROFILING.md)"}
+
+
+def host_link_peaks(torch, nbytes=256 << 20, iters=5) -> dict:
+    """Pinned H2D, D2H and concurrent bidirectional copy bandwidth (GB/s),
+    plain cudaMemcpyAsync through torch on dedicated streams."""
+    h_in = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    h_out = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    d_a = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d_b = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+
+    def timed(fn):
+        best = None
+        for _ in range(iters + 1):
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            fn()
+            torch.cuda.synchronize()
+            dt = time.perf_counter() - t
+            best = dt if best is None else min(best, dt)
+        return best
+
+    def h2d():
+        with torch.cuda.stream(s1):
+            d_a.copy_(h_in, non_blocking=True)
+
+    def d2h():
+        with torch.cuda.stream(s2):
+            h_out.copy_(d_b, non_blocking=True)
+
+    def both():
+        h2d()
+        d2h()
+    r = {"h2d_gbs": nbytes / timed(h2d) / 1e9, "d2h_gbs": nbytes / timed(d2h) / 1e9}
+    r["bidir_gbs"] = 2 * nbytes / timed(both) / 1e9
+    del h_in, h_out, d_a, d_b
+    return r
+
+
+def kernel_rooflines(torch, S, peaks) -> list:
+    """Tenant kernels stand-alone (same device bodies as the dispatcher) on the
+    whole GPU; CUDA events on the launching stream; inputs > L2."""
+    out = []
+    st = torch.cuda.current_stream()
+
+    def time_launch(desc, ins, outs, iters=10):
+        S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs],
+                        stream=st.cuda_stream)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        for _ in range(iters):
+            S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs],
+                            stream=st.cuda_stream)
+        e1.record(st)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / 1e3 / iters
+
+    n = 1 << 28
+    x = torch.empty(n, dtype=torch.float32, device="cuda").uniform_(-1, 1)
+    y = torch.empty_like(x)
+    for cls, name in ((S.VSCALE, "VSCALE"), (S.XFER, "XFER")):
+        t = time_launch(S.make_desc(cls, n=n, alpha=1.001, seed=7), [x], [y])
+        gbs = 8 * n / t / 1e9
+        out.append({"kernel": name, "bound": "hbm", "size": f"n=2^28 ({8 * n >> 20} MiB moved)",
+                    "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                    "frac": round(gbs / peaks["hbm_gbs"], 4), "ms": round(t * 1e3, 4)})
+    del x, y
+    m, nn, k, reps = 128 * 148, 256, 256, 64
+    a = torch.randint(-2, 3, (m, k), device="cuda").to(torch.bfloat16)
+    b = torch.randint(-2, 3, (k, nn), device="cuda").to(torch.bfloat16)
+    c = torch.empty((m, nn), dtype=torch.float32, device="cuda")
+    t = time_launch(S.make_desc(S.GEMM, m=m, n=nn, k=k, reps=reps), [a, b], [c], iters=5)
+    tf = 2 * m * nn * k * reps / t / 1e12
+    out.append({"kernel": "GEMM", "bound": "tensor", "size": f"{m}x{nn}x{k} x R={reps} (148 tiles)",
+                "achieved": round(tf, 1), "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
+                "frac": round(tf / peaks["bf16_tflops"], 4), "ms": round(t * 1e3, 4)})
+    ref = (a.float() @ b.float())
+    assert torch.equal(c, ref), "GEMM roofline run produced a wrong result"
+    del a, b, c, ref
+    torch.cuda.empty_cache()
+    return out
+
+
+# ------------------------------------------------------- strings arm
+def tstar_device(wl, link, hbm_gbs, tflops) -> float:
+    """Overlapped roofline T*_d (s) for one device running all of wl."""
+    import strings_workload as W
+    bh, bd = link["h2d_gbs"] * 1e9, link["d2h_gbs"] * 1e9
+    bb = link["bidir_gbs"] * 1e9
+    h2d = sum(sum(j.h2d_sizes()) for j in wl.jobs)
+    d2h = sum(sum(j.d2h_sizes()) for j in wl.jobs)
+    hbm = flop = 0
+    chains = {}
+    for j in wl.jobs:
+        if j.kclass == W.GEMM:
+            jb = 2 * j.m * j.k + 2 * j.k * j.n + 4 * j.m * j.n
+            jf = 2 * j.m * j.n * j.k * j.reps
+        else:
+            jb, jf = 8 * j.n, 0
+        hbm += jb
+        flop += jf
+        kl = max(jb / (hbm_gbs * 1e9), jf / (tflops * 1e12 / 2))   # a KL slot has half the SMs (P=2)
+        chains[j.tenant] = chains.get(j.tenant, 0.0) + sum(j.h2d_sizes()) / bh + kl + sum(j.d2h_sizes()) / bd
+    terms = {"h2d": h2d / bh, "d2h": d2h / bd, "bidir": (h2d + d2h) / bb,
+             "hbm": (hbm + h2d + d2h) / (hbm_gbs * 1e9), "tensor": flop / (tflops * 1e12),
+             "chain": max(chains.values())}
+    return max(terms.values()), terms
+
+
+def run_strings(args, rank, world, torch, gloo):
+    import numpy as np
+
+    import strings_workload as W
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+
+    peaks = measured_peaks()
+    link = host_link_peaks(torch)
+    krl = [] if args.no_kernels else kernel_rooflines(torch, S, peaks)
+    torch.cuda.synchronize()
+
+    wl = W.config_c2(jobs_per_tenant=args.jobs_per_tenant)
+    cfg = wl.config.resolved()
+    # inputs resident in pinned host memory before timing (the H2D phase is part of the job, S4)
+    ins, outs = [], []
+    for spec in wl.jobs:
+        src = W.job_inputs(spec)
+        pins = []
+        for a in src:
+            p = torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory()
+            pins.append(p)
+        ins.append(pins)
+        outs.append([torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
+    S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1, kl_mode=args.kl_mode,
+                       trace_in_memory=True)
+    # the persistent dispatcher now owns every SM: no torch kernels, no device-wide sync until shutdown
+    tenants = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+    stream = torch.cuda.Stream()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+
+    def one_step():
+        for i, spec in enumerate(wl.jobs):
+            S.submit_spec(tenants[spec.tenant], spec, ins[i], outs[i])
+        st = S.drain()
+        assert st == S.OK, S.strerror(st)
+
+    for _ in range(args.warmup):
+        one_step()
+    trace_start = len(S.trace())
+    gloo_barrier(gloo)
+    stream.synchronize()
+    with ClockSampler(int(os.environ.get("LOCAL_RANK", 0)) if world > 1 else 0) as clk:
+        ev0.record(stream)
+        t_wall = time.perf_counter()
+        for _ in range(args.steps):
+            one_step()
+        ev1.record(stream)
+        ev1.synchronize()
+        t_wall = time.perf_counter() - t_wall
+    gloo_barrier(gloo)
+    dt = ev0.elapsed_time(ev1) / 1e3
+    stats = S.stats()
+    trace = S.trace()[trace_start:]
+    infos = [S.job_info(i) for i in range(len(wl.jobs) * (args.warmup + args.steps))]
+    jobs_step = len(wl.jobs)
+    # e2e: the same workload through the public API from pageable numpy arrays
+    # (PMT staging + copy-back inside the timed region), one step
+    e2e = None
+    if not args.no_e2e:
+        np_ins = [[a.numpy().copy() for a in row] for row in ins]
+        np_outs = [[np.empty(o.numel(), dtype=np.uint8) for o in row] for row in outs]
+        t = time.perf_counter()
+        for i, spec in enumerate(wl.jobs):
+            S.submit_spec(tenants[spec.tenant], spec, np_ins[i], np_outs[i])
+        assert S.drain() == S.OK
+        e2e_dt = time.perf_counter() - t
+        e2e = {"value": round(jobs_step * world / max_over(gloo, e2e_dt), 3), "unit": "jobs/s",
+               "h2d_bytes_per_step": int(sum(sum(j.h2d_sizes()) for j in wl.jobs)),
+               "d2h_bytes_per_step": int(sum(sum(j.d2h_sizes()) for j in wl.jobs)),
+               "host_buffers": "pageable numpy (staged through the library's pinned PMT)"}
+    S.shutdown()
+    torch.cuda.synchronize()
+    # output parity on the last step's results (oracle, sampled)
+    from oracle import kernels as K
+    rng = np.random.default_rng(rank)
+    for i in (0, 1, len(wl.jobs) - 1):
+        spec = wl.jobs[i]
+        src = W.job_inputs(spec)
+        got = outs[i][0].numpy()
+        if spec.kclass == W.GEMM:
+            ref = K.gemm(src[0], src[1])
+            err = np.max(np.abs(got.view(np.float32).reshape(ref.shape).astype(np.float64) - ref)) / np.max(np.abs(ref))
+            assert err <= 1e-5, err
+        else:
+            idx = rng.integers(0, spec.n, 4096)
+            assert np.array_equal(got.view(np.uint32)[idx], K.xfer(src[0][idx], spec.seed))
+    dt_max = max_over(gloo, dt)
+    value = jobs_step * args.steps * world / dt_max
+    # per-step spans from the trace -> overlapped roofline fraction
+    span_step = dt / args.steps
+    tstar, terms = tstar_device(wl, link, peaks["hbm_gbs"], peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"])
+    moved = sum(sum(j.h2d_sizes()) + sum(j.d2h_sizes()) for j in wl.jobs)
+    link_gbs = moved / span_step / 1e9
+    # Jain fairness over tenants (reading R-2): x_i = 1 / mean latency (equal weights, c_t = 1)
+    lat = {}
+    last = infos[-jobs_step * args.steps:]
+    for inf in last:
+        lat.setdefault(inf.tenant, []).append(inf.t_done[2] - inf.t_arrival)
+    xs = [1.0 / statistics.mean(v) for v in lat.values()]
+    jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+    kl_items = jobs_step * args.steps
+    res = {
+        "metric": METRIC, "value": round(value, 3), "unit": "jobs/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt_max / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16/f32/u32",
+        "data": "synthetic (seeded; strings_workload)",
+        "config": {"workload": "C2: 16 tenants (8 GEMM 256^3 R=64, 8 XFER 2^24 u32) x 8 jobs, 1 B200 per rank, "
+                               "DTF joint placement, PS dispatch, measured timing",
+                   "jobs_per_step_per_gpu": jobs_step, "partitions": cfg.partitions,
+                   "awake_budget": cfg.awake_budget, "admit_cap": cfg.admit_cap,
+                   "l2": "inputs larger than L2 (4 GiB H2D + 4 GiB D2H per step)",
+                   "kl_mode": "persistent dispatcher" if args.kl_mode == 0 else "per-job launches",
+                   "parallelism": f"placement only, {world} rank(s) x 1 GPU"},
+        "roofline": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(link["bidir_gbs"], 2),
+                     "unit": "GB/s", "frac": round(link_gbs / link["bidir_gbs"], 4), "traffic": None,
+                     "resource": "copy engines H2D+D2H (the step's dominant resource)",
+                     "peak_source": "measured in this run: concurrent pinned H2D+D2H cudaMemcpyAsync 256 MiB"},
+        "overlapped_roofline": {"tstar_ms": round(tstar * 1e3, 3), "span_ms": round(span_step * 1e3, 3),
+                                "frac": round(tstar / span_step, 4),
+                                "terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()}},
+        "host_link": {k: round(v, 2) for k, v in link.items()},
+        "kernel_rooflines": krl,
+        "jain": round(jain, 4),
+        "gpu_launches": kl_items,
+        "gpu_launches_note": "KL work items executed by the persistent dispatcher kernel (launched once at init)"
+                             if args.kl_mode == 0 else "per-job tenant kernel launches",
+        "clocks": clk.summary(),
+        "decisions_per_step": (stats.decisions // (args.warmup + args.steps + (0 if args.no_e2e else 1))),
+        "wall_s": round(t_wall, 4),
+    }
+    if e2e:
+        res["e2e"] = e2e
+    if args.trace_out and rank == 0:
+        with open(args.trace_out, "w") as f:
+            f.write("\n".join(trace) + "\n")
+    return res, wl
+
+
+def max_over(gloo, x: float) -> float:
+    if gloo is None:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
+    return float(t.item())
+
+
+def gloo_barrier(gloo):
+    if gloo is not None:
+        import torch.distributed as dist
+        dist.barrier(group=gloo)
+
+
+# --------------------------------------------------------------- baselines
+def cpu_baseline(wl, sample_jobs: int = 16) -> dict:
+    """The oracle (as it stands) on a bounded sample of the workload on the host:
+    per job a host copy in, the oracle kernel, a host copy out; BLAS limited to
+    one thread.  Plus the oracle DES on the whole workload."""
+    import numpy as np
+    from threadpoolctl import threadpool_limits
+
+    import strings_workload as W
+    from oracle import kernels as K
+    from oracle.des import run_oracle
+
+    sample = wl.jobs[:sample_jobs]
+    data = [W.job_inputs(s) for s in sample]
+    with threadpool_limits(limits=1):
+        t = time.perf_counter()
+        for s, ins in zip(sample, data):
+            staged = [np.copy(a) for a in ins]
+            outs = K.run_job(s, staged)
+            _ = [np.copy(o) for o in outs]
+        dt = time.perf_counter() - t
+        t2 = time.perf_counter()
+        run_oracle(wl)
+        des = time.perf_counter() - t2
+    return {"value": round(len(sample) / dt, 3), "unit": "jobs/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {len(sample)} jobs of C2 (one per tenant): copy-in, oracle kernel, copy-out",
+            "des_s_full_workload": round(des, 3)}
+
+
+def run_reference(args):
+    """--impl reference: the oracle as it stands on the host cores, same config/metric."""
+    import strings_workload as W
+    wl = W.config_c2(jobs_per_tenant=args.jobs_per_tenant)
+    for _ in range(args.warmup):
+        cpu_baseline(wl, sample_jobs=4)
+    vals = []
+    t = time.perf_counter()
+    for _ in range(args.steps):
+        vals.append(cpu_baseline(wl, sample_jobs=16)["value"])
+    dt = time.perf_counter() - t
+    v = statistics.median(vals)
+    line = {"metric": METRIC, "value": v, "unit": "jobs/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64/f32/u32 (numpy)", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": "C2 (16 tenants, 8 GEMM 256^3 R=64 + 8 XFER 2^24), oracle on the host"},
+            "cpu_baseline": {"value": v, "unit": "jobs/s", "cores": 1, "kind": "oracle",
+                             "sample": "16 jobs of C2 per step (one per tenant)"},
+            "e2e": {"value": v, "unit": "jobs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if args.impl == "reference":
+        if rank == 0:
+            run_reference(args)
+        return
+    if world > 1:
+        os.environ["CUDA_VISIBLE_DEVICES"] = os.environ.get("LOCAL_RANK", str(rank))
+    import torch
+    gloo = None
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(0)
+        dist.init_process_group("nccl", device_id=torch.device("cuda:0"))
+        gloo = dist.new_group(backend="gloo")
+    res, wl = run_strings(args, rank, world, torch, gloo)
+    if rank == 0:
+        if world == 1 and not args.no_static:
+            from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
+            sb = run_static(wl, num_gpus=1)
+            res["static_baseline"] = sb
+            res["speedup_vs_static"] = round(res["value"] / sb["value"], 3)
+        if world == 1:
+            res["cpu_baseline"] = cpu_baseline(wl)
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

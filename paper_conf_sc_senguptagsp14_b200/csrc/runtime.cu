@@ -116,6 +116,48 @@ struct Phys {
   std::vector<cudaEvent_t> ev_pool;
 };
 
+// Pinned staging buffers for pageable caller memory (the paper's PMT).
+// Buffers are recycled by power-of-two size class and released only at
+// shutdown: cudaFreeHost may synchronise the device, which would wait forever
+// on the persistent dispatcher kernel.
+class StagingPool {
+ public:
+  void* get(uint64_t bytes) {
+    const int c = cls(bytes);
+    std::lock_guard<std::mutex> g(mu_);
+    auto& fl = free_[c];
+    if (!fl.empty()) {
+      void* p = fl.back();
+      fl.pop_back();
+      return p;
+    }
+    void* p = nullptr;
+    if (!cuda_ok(cudaHostAlloc(&p, (size_t)1 << c, cudaHostAllocPortable))) return nullptr;
+    all_.push_back(p);
+    return p;
+  }
+  void put(void* p, uint64_t bytes) {
+    std::lock_guard<std::mutex> g(mu_);
+    free_[cls(bytes)].push_back(p);
+  }
+  void release_all() {
+    std::lock_guard<std::mutex> g(mu_);
+    for (void* p : all_) cudaFreeHost(p);
+    all_.clear();
+    for (auto& f : free_) f.clear();
+  }
+
+ private:
+  static int cls(uint64_t b) {
+    int c = 12;
+    while (((uint64_t)1 << c) < b) ++c;
+    return c;
+  }
+  std::mutex mu_;
+  std::vector<void*> free_[64];
+  std::vector<void*> all_;
+};
+
 struct Tenant {
   uint32_t weight = 1, c = 1;
   uint64_t outstanding = 0;            // submitted, not done
@@ -157,6 +199,8 @@ class Runtime : public strings::Hooks {
     bool operator>(const VEv& o) const { return t > o.t; }
   };
   std::priority_queue<VEv, std::vector<VEv>, std::greater<VEv>> vheap;
+  StagingPool staging;
+  std::vector<void*> deferred_host_free;   // strings_host_free while the dispatcher runs
 
   bool virtual_clock() const { return cfg.timing_mode != STRINGS_TIMING_MEASURED; }
   bool has_gpu() const { return cfg.timing_mode != STRINGS_TIMING_DECISIONS_ONLY; }
@@ -240,6 +284,7 @@ class Runtime : public strings::Hooks {
       size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
       if (!cuda_ok(cudaMalloc(&ph->dev_state, heads_bytes + parts_bytes))) return STRINGS_ENOMEM;
       if (!cuda_ok(cudaMemset(ph->dev_state, 0, heads_bytes + parts_bytes))) return STRINGS_ECUDA;
+      if (!cuda_ok(cudaDeviceSynchronize())) return STRINGS_ECUDA;   // zeroed before the dispatcher starts
       // arena: L logical devices x M slots
       size_t arena = (size_t)ph->L * cfg.admit_cap * cfg.slot_bytes;
       if (!cuda_ok(cudaMalloc(&ph->arena, arena))) return STRINGS_ENOMEM;
@@ -420,7 +465,7 @@ class Runtime : public strings::Hooks {
       for (auto* v : {&jc->in, &jc->out})
         for (auto& b : *v)
           if (b.staged && b.dma) {
-            cudaFreeHost(b.dma);
+            staging.put(b.dma, b.bytes);
             b.dma = nullptr;
           }
       if (jc->slot >= 0) {
@@ -640,8 +685,8 @@ class Runtime : public strings::Hooks {
       if (e != cudaSuccess) cudaGetLastError();
       bool pinned = e == cudaSuccess && a.type == cudaMemoryTypeHost;
       if (pinned) return STRINGS_OK;
-      void* p = nullptr;
-      if (!cuda_ok(cudaHostAlloc(&p, b.bytes, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+      void* p = staging.get(b.bytes);
+      if (!p) return STRINGS_ENOMEM;
       if (is_in) memcpy(p, b.host, b.bytes);
       hb.dma = p;
       hb.staged = true;
@@ -719,7 +764,12 @@ class Runtime : public strings::Hooks {
     }
     if (engine.joinable()) engine.join();
     flush_trace();
-    if (has_gpu()) teardown_gpus();
+    if (has_gpu()) {
+      teardown_gpus();
+      staging.release_all();
+      for (void* p : deferred_host_free) cudaFreeHost(p);
+      deferred_host_free.clear();
+    }
   }
 };
 
@@ -804,6 +854,14 @@ strings_status_t strings_host_alloc(uint64_t bytes, void** p) {
 
 strings_status_t strings_host_free(void* p) {
   if (!p) return STRINGS_OK;
+  {
+    std::lock_guard<std::mutex> g(g_init_mu);
+    if (g_rt && g_rt->has_gpu()) {          // freeing pinned memory may synchronise the device:
+      std::lock_guard<std::mutex> g2(g_rt->mu);   // defer until the dispatcher has stopped
+      g_rt->deferred_host_free.push_back(p);
+      return STRINGS_OK;
+    }
+  }
   return cuda_ok(cudaFreeHost(p)) ? STRINGS_OK : STRINGS_ECUDA;
 }
 

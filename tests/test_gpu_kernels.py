@@ -1,0 +1,105 @@
+"""Tenant kernel parity on the B200 (stand-alone launches through the C ABI).
+
+Each kernel is launched through ``strings_kernel_launch`` (the same device
+bodies the persistent dispatcher runs) on torch-allocated device memory and
+compared element by element with the CPU oracle (oracle/kernels.py):
+VSCALE and XFER bit-exact, GEMM bit-exact on integer-valued inputs and within
+1e-5 normwise relative error on random inputs (reading R-22).
+"""
+import numpy as np
+import pytest
+
+import strings_workload as W
+from oracle import kernels as K
+from paper_conf_sc_senguptagsp14_b200 import strings as S
+
+pytestmark = pytest.mark.gpu
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _launch(desc, ins, outs, ctas=0):
+    torch = _torch()
+    dev_in = [torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in ins]
+    dev_out = [torch.zeros(o.nbytes, dtype=torch.uint8, device="cuda") for o in outs]
+    S.kernel_launch(0, desc, [t.data_ptr() for t in dev_in], [t.data_ptr() for t in dev_out], ctas=ctas,
+                    stream=torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    return [t.cpu().numpy().view(o.dtype).reshape(o.shape) for t, o in zip(dev_out, outs)]
+
+
+@pytest.mark.parametrize("n", [0, 1, 3, 4, 5, 1023, 4097, 65536 + 7, (1 << 20) + 3, 1 << 24])
+@pytest.mark.parametrize("ctas", [0, 1, 37])
+def test_vscale_bit_exact(n, ctas):
+    rng = np.random.default_rng(n + 17)
+    x = rng.uniform(-1, 1, n).astype(np.float32)
+    if n > 8:
+        x[:4] = np.array([1e-45, -2.0 ** -126, 3.4e38, -0.0], dtype=np.float32)   # denormal, huge, -0
+    a = 1.0 + 2.0 ** -10
+    (y,) = _launch(S.make_desc(S.VSCALE, n=n, alpha=a), [x], [np.zeros(n, np.float32)], ctas)
+    assert np.array_equal(y.view(np.uint32), K.vscale(x, a).view(np.uint32))
+
+
+@pytest.mark.parametrize("n", [0, 1, 7, 4096, 65537, (1 << 22) + 1])
+def test_xfer_bit_exact(n):
+    rng = np.random.default_rng(n + 3)
+    x = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    seed = 0xDEADBEEF
+    (y,) = _launch(S.make_desc(S.XFER, n=n, seed=seed), [x], [np.zeros(n, np.uint32)])
+    assert np.array_equal(y, K.xfer(x, seed))
+
+
+def test_streaming_unaligned_pointers():
+    torch = _torch()
+    n = 10_001
+    x = np.random.default_rng(1).uniform(-1, 1, n + 1).astype(np.float32)
+    dx = torch.from_numpy(x).cuda()
+    dy = torch.zeros(n + 1, dtype=torch.float32, device="cuda")
+    S.kernel_launch(0, S.make_desc(S.VSCALE, n=n, alpha=3.0), [dx.data_ptr() + 4], [dy.data_ptr() + 4],
+                    stream=torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    assert np.array_equal(dy.cpu().numpy()[1:].view(np.uint32), K.vscale(x[1:], 3.0).view(np.uint32))
+
+
+def _gemm_inputs(m, n, k, seed, int_valued):
+    rng = np.random.default_rng(seed)
+    if int_valued:
+        a = rng.integers(-2, 3, (m, k)).astype(np.float32)
+        b = rng.integers(-2, 3, (k, n)).astype(np.float32)
+    else:
+        a = rng.uniform(-1, 1, (m, k)).astype(np.float32)
+        b = rng.uniform(-1, 1, (k, n)).astype(np.float32)
+    return W.f32_to_bf16_bits(a), W.f32_to_bf16_bits(b)
+
+
+@pytest.mark.parametrize("m,n,k", [(128, 256, 64), (256, 256, 256), (384, 512, 128), (128, 768, 192)])
+@pytest.mark.parametrize("reps,ctas", [(1, 0), (3, 2), (64, 5), (7, 148)])
+def test_gemm_integer_inputs_bit_exact(m, n, k, reps, ctas):
+    a, b = _gemm_inputs(m, n, k, m * 7 + n + k, True)
+    (c,) = _launch(S.make_desc(S.GEMM, m=m, n=n, k=k, reps=reps), [a, b], [np.zeros((m, n), np.float32)], ctas)
+    assert np.array_equal(c, K.gemm(a, b))
+
+
+@pytest.mark.parametrize("m,n,k", [(128, 256, 64), (256, 256, 256), (512, 256, 256)])
+def test_gemm_random_inputs_within_tolerance(m, n, k):
+    a, b = _gemm_inputs(m, n, k, 99 + m, False)
+    (c,) = _launch(S.make_desc(S.GEMM, m=m, n=n, k=k, reps=2), [a, b], [np.zeros((m, n), np.float32)])
+    ref = K.gemm(a, b)
+    err = np.max(np.abs(c.astype(np.float64) - ref)) / np.max(np.abs(ref))
+    assert err <= 1e-5, err
+
+
+def test_gemm_structured_operands_catch_layout_errors():
+    # A = I-like selector, B = arange: C rows must pick exact B rows (catches
+    # transposed / mis-strided smem layouts that random data might average out)
+    m, n, k = 128, 256, 128
+    a = np.zeros((m, k), np.float32)
+    for i in range(m):
+        a[i, (i * 5) % k] = 1.0
+    b = (np.arange(k * n) % 251 - 125).astype(np.float32).reshape(k, n)
+    ab, bb = W.f32_to_bf16_bits(a), W.f32_to_bf16_bits(b)
+    (c,) = _launch(S.make_desc(S.GEMM, m=m, n=n, k=k, reps=1), [ab, bb], [np.zeros((m, n), np.float32)])
+    assert np.array_equal(c, K.gemm(ab, bb))

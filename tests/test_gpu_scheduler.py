@@ -1,0 +1,115 @@
+"""Scheduler parity on the B200: decision traces and tenant outputs vs the oracle.
+
+INJECTED mode: every op runs on the GPU (copy engines + persistent dispatcher
+kernel) while decisions follow the virtual clock, so the trace must be
+byte-identical to the oracle's and every output must match the oracle's CPU
+kernels (bit-exact VSCALE/XFER/int GEMM, 1e-5 for random GEMM).
+MEASURED mode: real clock; the trace must satisfy invariants I1-I5 and the
+outputs must still be exact.
+"""
+import numpy as np
+import pytest
+
+import strings_workload as W
+from oracle import invariants
+from oracle import kernels as K
+from oracle.des import run_oracle
+from paper_conf_sc_senguptagsp14_b200 import strings as S
+from paper_conf_sc_senguptagsp14_b200.runner import run_workload
+
+pytestmark = pytest.mark.gpu
+
+
+def check_outputs(wl, res, sample=None):
+    for i, spec in enumerate(wl.jobs):
+        ins = W.job_inputs(spec)
+        want = K.run_job(spec, ins)
+        for got, ref in zip(res.outputs[i], want):
+            if spec.kclass == W.GEMM and not spec.int_valued:
+                err = np.max(np.abs(got.astype(np.float64) - ref)) / max(1e-30, np.max(np.abs(ref)))
+                assert err <= 1e-5, (i, err)
+            else:
+                assert np.array_equal(got.view(np.uint32) if got.dtype == np.float32 else got,
+                                      ref.view(np.uint32) if ref.dtype == np.float32 else ref), i
+    for info in res.infos:
+        assert info.status == S.OK
+
+
+def test_c1_injected_trace_and_outputs_match_oracle():
+    wl = W.config_c1()
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.INJECTED)
+    assert r.status == S.OK
+    assert r.trace == o.trace
+    check_outputs(wl, r)
+
+
+def test_c1_integer_gemm_injected_bit_exact():
+    wl = W.config_c1(int_valued=True, reps=3)
+    r = run_workload(wl, timing_mode=S.INJECTED)
+    assert r.trace == run_oracle(wl).trace
+    check_outputs(wl, r)
+
+
+@pytest.mark.parametrize("name,kw", [("C2", dict(scale=64, jobs_per_tenant=3)), ("C3", dict(scale=4)),
+                                     ("C4", dict(scale=64, jobs_per_tenant=3)),
+                                     ("C5", dict(scale=64, jobs_per_tenant=5))])
+def test_configs_injected_on_logical_devices(name, kw):
+    # G logical devices share the one physical GPU: decisions
+    # depend only on virtual time, so G = 2/4/8 parity is checked on one B200.
+    wl = W.CONFIGS[name](**kw)
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.INJECTED)
+    assert r.status == S.OK
+    assert r.trace == o.trace
+    check_outputs(wl, r)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_workloads_injected(seed):
+    wl = W.random_workload(seed, max_gpus=3)
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.INJECTED)
+    assert r.trace == o.trace
+    check_outputs(wl, r)
+
+
+@pytest.mark.parametrize("name,kw", [("C1", {}), ("C2", dict(scale=16, jobs_per_tenant=4)),
+                                     ("C5", dict(scale=64, jobs_per_tenant=4))])
+def test_measured_mode_invariants_and_outputs(name, kw):
+    wl = W.CONFIGS[name](**kw)
+    r = run_workload(wl, timing_mode=S.MEASURED)
+    assert r.status == S.OK
+    assert invariants.check(r.trace, wl) == []
+    check_outputs(wl, r)
+    # the KL phases really ran on SM partitions of the persistent kernel
+    parts = {i.kl_partition for i in r.infos}
+    assert min(parts) >= 0
+    assert all(i.kl_gpu_end_ns >= i.kl_gpu_start_ns > 0 for i in r.infos)
+
+
+def test_pageable_buffers_are_staged():
+    wl = W.config_c1(reps=2)
+    r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)
+    assert r.status == S.OK
+    check_outputs(wl, r)
+
+
+def test_full_size_c2_measured_sampled_parity():
+    # BASELINE configs[1] at full size, in the launch configuration bench.py
+    # times (MEASURED, persistent dispatcher): every GEMM output in full, XFER
+    # outputs on a 64 Ki-element sample per job (the oracle one element at a time).
+    wl = W.config_c2(jobs_per_tenant=2)
+    r = run_workload(wl, timing_mode=S.MEASURED, keep_inputs=True)
+    assert r.status == S.OK
+    assert invariants.check(r.trace, wl) == []
+    rng = np.random.default_rng(0)
+    for i, spec in enumerate(wl.jobs):
+        ins = r.inputs[i]
+        if spec.kclass == W.GEMM:
+            ref = K.gemm(ins[0], ins[1])
+            err = np.max(np.abs(r.outputs[i][0].astype(np.float64) - ref)) / np.max(np.abs(ref))
+            assert err <= 1e-5
+        else:
+            idx = np.concatenate([np.arange(64), spec.n - 1 - np.arange(64), rng.integers(0, spec.n, 65536)])
+            assert np.array_equal(r.outputs[i][0][idx], K.xfer(ins[0][idx], spec.seed))

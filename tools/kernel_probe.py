@@ -1,0 +1,47 @@
+"""Launch each tenant kernel stand-alone at its ncu size (for ncu captures).
+
+    ncu --set full --clock-control none --import-source on -k regex:oneshot -c 6 \
+        -o gpurun_out/prof python tools/kernel_probe.py
+
+Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2).
+The persistent dispatcher runs exactly these device bodies on its SM partitions.
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+from paper_conf_sc_senguptagsp14_b200 import strings as S  # noqa: E402
+
+
+def main():
+    which = sys.argv[1:] or ["vscale", "xfer", "gemm"]
+    st = torch.cuda.current_stream().cuda_stream
+    n = 1 << 28
+    if "vscale" in which or "xfer" in which:
+        x = torch.empty(n, dtype=torch.float32, device="cuda").uniform_(-1, 1)
+        y = torch.empty_like(x)
+        for cls, name in ((S.VSCALE, "vscale"), (S.XFER, "xfer")):
+            if name in which:
+                for _ in range(2):
+                    S.kernel_launch(0, S.make_desc(cls, n=n, alpha=1.001, seed=7), [x.data_ptr()], [y.data_ptr()],
+                                    stream=st)
+        torch.cuda.synchronize()
+        del x, y
+    if "gemm" in which:
+        m, nn, k, reps = 128 * 148, 256, 256, 64
+        a = torch.randint(-2, 3, (m, k), device="cuda").to(torch.bfloat16)
+        b = torch.randint(-2, 3, (k, nn), device="cuda").to(torch.bfloat16)
+        c = torch.empty((m, nn), dtype=torch.float32, device="cuda")
+        for _ in range(2):
+            S.kernel_launch(0, S.make_desc(S.GEMM, m=m, n=nn, k=k, reps=reps), [a.data_ptr(), b.data_ptr()],
+                            [c.data_ptr()], stream=st)
+        torch.cuda.synchronize()
+        assert torch.equal(c, a.float() @ b.float())
+    print("probe done")
+
+
+if __name__ == "__main__":
+    main()
