@@ -116,6 +116,71 @@ struct Phys {
   std::vector<cudaEvent_t> ev_pool;
 };
 
+// Parallel host memcpy for PMT staging (one host thread copies ~6-10 GB/s;
+// a 64 MiB pageable buffer is split over a small worker pool).
+class CopyPool {
+ public:
+  explicit CopyPool(int n) {
+    for (int i = 0; i < n; ++i) th_.emplace_back([this] { run(); });
+  }
+  ~CopyPool() {
+    {
+      std::lock_guard<std::mutex> g(mu_);
+      stop_ = true;
+    }
+    cv_.notify_all();
+    for (auto& t : th_) t.join();
+  }
+  void copy(void* dst, const void* src, uint64_t bytes) {
+    constexpr uint64_t kChunk = 4ull << 20;
+    if (bytes <= kChunk || th_.empty()) {
+      memcpy(dst, src, bytes);
+      return;
+    }
+    uint64_t parts = std::min<uint64_t>((bytes + kChunk - 1) / kChunk, th_.size() + 1);
+    uint64_t per = ((bytes / parts) + 63) & ~63ull;
+    std::atomic<int> left{0};
+    std::vector<Task> tasks;
+    for (uint64_t off = per; off < bytes; off += per)
+      tasks.push_back({static_cast<char*>(dst) + off, static_cast<const char*>(src) + off,
+                       std::min(per, bytes - off), &left});
+    left.store((int)tasks.size());
+    {
+      std::lock_guard<std::mutex> g(mu_);
+      for (auto& t : tasks) q_.push_back(t);
+    }
+    cv_.notify_all();
+    memcpy(dst, src, std::min(per, bytes));        // the caller copies the first part
+    while (left.load(std::memory_order_acquire) > 0) std::this_thread::yield();
+  }
+
+ private:
+  struct Task {
+    char* dst;
+    const char* src;
+    uint64_t n;
+    std::atomic<int>* left;
+  };
+  void run() {
+    std::unique_lock<std::mutex> lk(mu_);
+    for (;;) {
+      cv_.wait(lk, [this] { return stop_ || !q_.empty(); });
+      if (stop_ && q_.empty()) return;
+      Task t = q_.front();
+      q_.pop_front();
+      lk.unlock();
+      memcpy(t.dst, t.src, t.n);
+      t.left->fetch_sub(1, std::memory_order_release);
+      lk.lock();
+    }
+  }
+  std::mutex mu_;
+  std::condition_variable cv_;
+  std::deque<Task> q_;
+  std::vector<std::thread> th_;
+  bool stop_ = false;
+};
+
 // Pinned staging buffers for pageable caller memory (the paper's PMT).
 // Buffers are recycled by power-of-two size class and released only at
 // shutdown: cudaFreeHost may synchronise the device, which would wait forever
@@ -200,6 +265,11 @@ class Runtime : public strings::Hooks {
   };
   std::priority_queue<VEv, std::vector<VEv>, std::greater<VEv>> vheap;
   StagingPool staging;
+  CopyPool copier{6};
+  std::deque<std::pair<JobCtx*, uint64_t>> finalize_q;
+  std::condition_variable cv_final;
+  std::vector<std::thread> finalizers;
+  bool stop_final = false;
   std::vector<void*> deferred_host_free;   // strings_host_free while the dispatcher runs
 
   bool virtual_clock() const { return cfg.timing_mode != STRINGS_TIMING_MEASURED; }
@@ -249,6 +319,7 @@ class Runtime : public strings::Hooks {
     }
     t0 = mono_ns();
     engine = std::thread([this] { engine_main(); });
+    for (int i = 0; i < 4; ++i) finalizers.emplace_back([this] { finalizer_main(); });
     return STRINGS_OK;
   }
 
@@ -458,31 +529,60 @@ class Runtime : public strings::Hooks {
 
   void on_job_done(strings::Job& j, uint64_t t) override {
     JobCtx* jc = static_cast<JobCtx*>(j.user);
+    bool staged_out = false;
     if (has_gpu()) {
       Logical& lg = logical[j.gid];
-      for (auto& o : jc->out)
-        if (o.staged && o.bytes) memcpy(o.user, o.dma, o.bytes);
-      for (auto* v : {&jc->in, &jc->out})
-        for (auto& b : *v)
-          if (b.staged && b.dma) {
-            staging.put(b.dma, b.bytes);
-            b.dma = nullptr;
-          }
-      if (jc->slot >= 0) {
+      if (jc->slot >= 0) {              // the D2H finished: the device slot is free now
         lg.free_slots.push_back(jc->slot);
         jc->slot = -1;
       }
+      for (auto& b : jc->in)
+        if (b.staged && b.dma) {
+          staging.put(b.dma, b.bytes);
+          b.dma = nullptr;
+        }
+      for (auto& o : jc->out) staged_out |= o.staged && o.bytes;
     }
+    if (staged_out) {
+      // PMT copy-back to the caller's pageable buffer off the engine thread
+      finalize_q.push_back({jc, t});
+      cv_final.notify_one();
+    } else {
+      finish_job(jc, t);
+    }
+  }
+
+  // Tenant-visible completion (sync returns once every job of the tenant got here).
+  void finish_job(JobCtx* jc, uint64_t t) {
     if (jc->status == STRINGS_EAGAIN) jc->status = STRINGS_OK;
-    Tenant& tn = tenants[j.tenant];
+    Tenant& tn = tenants[jc->job.tenant];
     tn.outstanding -= 1;
     if (jc->status != STRINGS_OK) {
       tn.failed += 1;
       failed_count += 1;
     }
     done_count += 1;
-    last_done = t;
+    last_done = std::max(last_done, t);
     cv_done.notify_all();
+  }
+
+  void finalizer_main() {
+    std::unique_lock<std::mutex> lk(mu);
+    for (;;) {
+      cv_final.wait(lk, [this] { return stop_final || !finalize_q.empty(); });
+      if (finalize_q.empty() && stop_final) return;
+      auto item = finalize_q.front();
+      finalize_q.pop_front();
+      lk.unlock();
+      for (auto& o : item.first->out)
+        if (o.staged && o.bytes) {
+          copier.copy(o.user, o.dma, o.bytes);
+          staging.put(o.dma, o.bytes);
+          o.dma = nullptr;
+        }
+      lk.lock();
+      finish_job(item.first, item.second);
+    }
   }
 
   cudaEvent_t take_event(Phys* ph) {
@@ -687,7 +787,7 @@ class Runtime : public strings::Hooks {
       if (pinned) return STRINGS_OK;
       void* p = staging.get(b.bytes);
       if (!p) return STRINGS_ENOMEM;
-      if (is_in) memcpy(p, b.host, b.bytes);
+      if (is_in) copier.copy(p, b.host, b.bytes);
       hb.dma = p;
       hb.staged = true;
       return STRINGS_OK;
@@ -763,6 +863,12 @@ class Runtime : public strings::Hooks {
       cv_engine.notify_all();
     }
     if (engine.joinable()) engine.join();
+    {
+      std::lock_guard<std::mutex> g(mu);
+      stop_final = true;
+      cv_final.notify_all();
+    }
+    for (auto& f : finalizers) f.join();
     flush_trace();
     if (has_gpu()) {
       teardown_gpus();
@@ -968,9 +1074,12 @@ strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kerne
   }
   if (!cuda_ok(cudaSetDevice(physical_gpu))) return STRINGS_ECUDA;
   if (ctas <= 0) {
-    cudaDeviceProp prop;
-    if (!cuda_ok(cudaGetDeviceProperties(&prop, physical_gpu))) return STRINGS_ECUDA;
-    ctas = prop.multiProcessorCount;
+    static int sm_count[64] = {0};
+    if (physical_gpu < 0 || physical_gpu >= 64) return STRINGS_EINVAL;
+    if (sm_count[physical_gpu] == 0 &&
+        !cuda_ok(cudaDeviceGetAttribute(&sm_count[physical_gpu], cudaDevAttrMultiProcessorCount, physical_gpu)))
+      return STRINGS_ECUDA;
+    ctas = sm_count[physical_gpu];
   }
   KlItem it;
   memset(&it, 0, sizeof it);

@@ -95,11 +95,15 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
 
 // --------------------------------------------------------------------- GEMM
 // Tile 128 x 256 (M x N) per CTA, whole K (<= 256) resident in shared memory
-// in the UMMA canonical K-major SWIZZLE_NONE layout: a core matrix is 8 rows x
-// 16 B (8 bf16 along K) stored contiguously (128 B).
-//   A tile: core (row-group g in 0..15, k-chunk c) at (c*16 + g)*128   -> SBO = 128, LBO = 2048
-//   B tile: core (n-group g in 0..31, k-chunk c)   at (c*32 + g)*128   -> SBO = 128, LBO = 4096
-// (B is transposed while loading: smem holds B^T, K-major.)
+// in UMMA canonical SWIZZLE_NONE layouts built from 128-B "core matrices"
+// (8 rows of 16 B):
+//   A (K-major, A is M x K row-major): core (row-group g in 0..15, k-chunk c)
+//     holds rows 8g..8g+7, k 8c..8c+7; stored at (c*16 + g)*128  -> SBO = 128, LBO = 2048
+//   B (MN-major, B is K x N row-major): core (n-group q in 0..31, k-chunk c)
+//     holds k 8c..8c+7 (one per 16-B row), n 8q..8q+7; at (c*32 + q)*128
+//                                                              -> SBO = 128, LBO = 4096
+// Both are filled with plain 16-B copies (no transposition); 8 consecutive
+// threads write one 128-B core matrix, so the stores are bank-conflict free.
 constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
 constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
 constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
@@ -122,9 +126,10 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
 }
 
 // Instruction descriptor kind::f16: D=f32 [4,6)=1, A=bf16 [7,10)=1, B=bf16 [10,13)=1,
-// A,B K-major (bits 15,16 = 0), N>>3 at [17,23), M>>4 at [24,29).
+// A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29).
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+  return (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(N >> 3) << 17) |
+         ((uint32_t)(M >> 4) << 24);
 }
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -189,29 +194,26 @@ struct GemmSmem {
   uint32_t* tmem_slot; // TMEM base written by tcgen05.alloc
 };
 
-// Load the A tile (rows m0..m0+127, all K) and B^T (cols n0..n0+255, all K)
-// into the canonical layouts above.  All 256 threads participate.
+// Load the A tile (rows m0..m0+127, all K) and the B tile (all K, cols
+// n0..n0+255) into the canonical layouts above.  All 256 threads participate;
+// thread t writes row (t & 7) of a core matrix.
 __device__ inline void gemm_load_tile(const GemmSmem& sm, const uint16_t* __restrict__ A,
-                               const uint16_t* __restrict__ B, uint64_t N, uint64_t K, uint64_t m0,
-                               uint64_t n0) {
+                                      const uint16_t* __restrict__ B, uint64_t N, uint64_t K,
+                                      uint64_t m0, uint64_t n0) {
   const int kchunks = (int)(K / 8);
-  // A: 16-B chunks (row r, k-chunk c) -> core (c, r/8), row r%8
+  // A: 16 x kchunks cores; idx -> (rr = row in core, c = k-chunk, g = row group)
   for (int idx = threadIdx.x; idx < kTileM * kchunks; idx += kThreads) {
-    int r = idx / kchunks, c = idx % kchunks;
+    const int rr = idx & 7, c = (idx >> 3) % kchunks, g = (idx >> 3) / kchunks;
+    const int r = g * 8 + rr;
     uint4 v = *reinterpret_cast<const uint4*>(A + (m0 + r) * K + (uint64_t)c * 8);
-    *reinterpret_cast<uint4*>(sm.a + ((c * 16 + (r >> 3)) * 128 + (r & 7) * 16)) = v;
+    *reinterpret_cast<uint4*>(sm.a + ((c * 16 + g) * 128 + rr * 16)) = v;
   }
-  // B^T: read B[k][n0 + 8q .. +7] (16 B along N), scatter to rows n of the K-major tile
+  // B: 32 x kchunks cores; idx -> (kk = k in core, q = n-group, c = k-chunk)
   for (int idx = threadIdx.x; idx < (int)K * (kTileN / 8); idx += kThreads) {
-    int k = idx / (kTileN / 8), q = idx % (kTileN / 8);
+    const int kk = idx & 7, q = (idx >> 3) & 31, c = idx >> 8;
+    const int k = c * 8 + kk;
     uint4 v = *reinterpret_cast<const uint4*>(B + (uint64_t)k * N + n0 + (uint64_t)q * 8);
-    const uint16_t* e = reinterpret_cast<const uint16_t*>(&v);
-    int c = k >> 3, kk = k & 7;
-#pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      int n = q * 8 + t;
-      *reinterpret_cast<uint16_t*>(sm.b + ((c * 32 + (n >> 3)) * 128 + (n & 7) * 16 + kk * 2)) = e[t];
-    }
+    *reinterpret_cast<uint4*>(sm.b + ((c * 32 + q) * 128 + kk * 16)) = v;
   }
   // make generic-proxy smem writes visible to the tensor core (async proxy)
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
