@@ -370,19 +370,13 @@ def run_strings(args, rank, world, torch, gloo):
 
 
 def max_over(gloo, x: float) -> float:
-    if gloo is None:
-        return x
-    import torch
-    import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
-    return float(t.item())
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    return par.max_over_ranks(gloo, x)
 
 
 def gloo_barrier(gloo):
-    if gloo is not None:
-        import torch.distributed as dist
-        dist.barrier(group=gloo)
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    par.barrier(gloo)
 
 
 # --------------------------------------------------------------- baselines
@@ -439,21 +433,16 @@ def run_reference(args):
 
 def main():
     args = parse_args()
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    info = par.rank_info()
+    world, rank = info.world, info.rank
     if args.impl == "reference":
         if rank == 0:
             run_reference(args)
         return
-    if world > 1:
-        os.environ["CUDA_VISIBLE_DEVICES"] = os.environ.get("LOCAL_RANK", str(rank))
+    par.isolate_gpu(info)                 # one process per GPU (before CUDA init)
     import torch
-    gloo = None
-    if world > 1:
-        import torch.distributed as dist
-        torch.cuda.set_device(0)
-        dist.init_process_group("nccl", device_id=torch.device("cuda:0"))
-        gloo = dist.new_group(backend="gloo")
+    gloo = par.init_groups(info, device_backend="nccl")
     res, wl = run_strings(args, rank, world, torch, gloo)
     if rank == 0:
         if world == 1 and not args.no_static:

@@ -1,0 +1,87 @@
+"""Multi-GPU plumbing: one process per GPU, placement-only sharding.
+
+Tenants are independent, so scaling across the GPUs of a box is placement
+only: there is no data-path collective and no NCCL on the
+hot path.  Two deployment shapes are supported:
+
+* node mode -- one process owns G GPUs and the library's level-1 balancer
+  places every job on one of them (``strings_init(num_gpus=G)``); this is the
+  paper's design (one GPU affinity mapper per node);
+* rank mode -- ``torchrun`` starts one process per GPU; each rank runs its own
+  library instance on its own GPU over its shard of the tenants (weak scaling).
+
+While the persistent dispatcher kernel is resident it owns every SM, so rank
+coordination (barriers, max-over-ranks timing) must not launch device work or
+synchronise the device: it goes through a CPU (gloo) group.
+"""
+from __future__ import annotations
+
+import os
+from dataclasses import dataclass
+from typing import List, Optional
+
+
+@dataclass
+class RankInfo:
+    rank: int
+    world: int
+    local_rank: int
+
+
+def rank_info() -> RankInfo:
+    return RankInfo(int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
+                    int(os.environ.get("LOCAL_RANK", os.environ.get("RANK", "0"))))
+
+
+def isolate_gpu(info: RankInfo) -> None:
+    """Make this rank's GPU the only visible one (must run before CUDA init)."""
+    if info.world > 1:
+        os.environ["CUDA_VISIBLE_DEVICES"] = str(info.local_rank)
+
+
+def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl"):
+    """Default process group (NCCL when a GPU is present) plus a gloo group for
+    host-side coordination.  Returns the gloo group (None for world == 1)."""
+    if info.world == 1:
+        return None
+    import torch
+    import torch.distributed as dist
+    if device_backend == "nccl" and torch.cuda.is_available():
+        torch.cuda.set_device(0)
+        dist.init_process_group("nccl", device_id=torch.device("cuda:0"))
+        return dist.new_group(backend="gloo")
+    dist.init_process_group("gloo")
+    return dist.group.WORLD
+
+
+def barrier(group) -> None:
+    if group is not None:
+        import torch.distributed as dist
+        dist.barrier(group=group)
+
+
+def max_over_ranks(group, x: float) -> float:
+    """Max over ranks of a host-side float (device timings are taken on each
+    rank with CUDA events, then reduced here)."""
+    if group is None:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())
+
+
+def sum_over_ranks(group, x: float) -> float:
+    if group is None:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return float(t.item())
+
+
+def shard_tenants(num_tenants: int, world: int, rank: int) -> List[int]:
+    """Tenants of this rank under strong scaling (round robin, like GRR)."""
+    return [t for t in range(num_tenants) if t % world == rank]
