@@ -50,6 +50,12 @@ def parse_args():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--kl-mode", type=int, default=0, help="0 persistent dispatcher, 1 per-job launches (ncu)")
     p.add_argument("--trace-out", default=None)
+    p.add_argument("--static-repeats", type=int, default=3)
+    p.add_argument("--awake-budget", type=int, default=0, help="A (0 = config default)")
+    p.add_argument("--admit-cap", type=int, default=0, help="M (0 = config default)")
+    p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
+    p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
+    p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
     return p.parse_args()
 
 
@@ -227,6 +233,13 @@ def run_strings(args, rank, world, torch, gloo):
     torch.cuda.synchronize()
 
     wl = W.config_c2(jobs_per_tenant=args.jobs_per_tenant)
+    for name in ("awake_budget", "admit_cap", "partitions"):
+        if getattr(args, name) > 0:
+            setattr(wl.config, name, getattr(args, name))
+    if args.device_policy >= 0:
+        wl.config.device_policy = args.device_policy
+    if args.balancer >= 0:
+        wl.config.balancer = args.balancer
     cfg = wl.config.resolved()
     # inputs resident in pinned host memory before timing (the H2D phase is part of the job, S4)
     ins, outs = [], []
@@ -329,6 +342,13 @@ def run_strings(args, rank, world, torch, gloo):
         lastd[inf.tenant] = max(lastd.get(inf.tenant, 0), inf.t_done[2])
     xs = [busy[t] / max(1, lastd[t] - first[t]) / wl.tenants[t].weight for t in busy]
     jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+    # mean completion latency per tenant in the last timed step (all jobs
+    # submitted at the start of the step), for the weighted speedup
+    step_t0 = min(inf.t_arrival for inf in last)
+    mlat = {}
+    for inf in last:
+        mlat.setdefault(inf.tenant, []).append((inf.t_done[2] - step_t0) / 1e9)
+    mlat = {t: sum(v) / len(v) for t, v in mlat.items()}
     kl_items = jobs_step * args.steps
     res = {
         "metric": METRIC, "value": round(value, 3), "unit": "jobs/s", "n_gpus": world,
@@ -351,6 +371,7 @@ def run_strings(args, rank, world, torch, gloo):
                                 "terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()}},
         "host_link": {k: round(v, 2) for k, v in link.items()},
         "kernel_rooflines": krl,
+        "_mean_latency_s_by_tenant": mlat,
         "jain": round(jain, 4),
         "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step)",
         "gpu_launches": kl_items,
@@ -447,9 +468,16 @@ def main():
     if rank == 0:
         if world == 1 and not args.no_static:
             from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
-            sb = run_static(wl, num_gpus=1)
+            sb = run_static(wl, num_gpus=1, repeats=args.static_repeats)
             res["static_baseline"] = sb
             res["speedup_vs_static"] = round(res["value"] / sb["value"], 3)
+            # weighted speedup, Eq. (2) (reading R-1): mean over tenants of
+            # mean latency under static provisioning / under Strings
+            mine = res.pop("_mean_latency_s_by_tenant")
+            st = sb["mean_latency_s_by_tenant"]
+            ws = sum(st[t] / mine[t] for t in mine) / len(mine)
+            res["weighted_speedup_vs_static"] = round(ws, 3)
+        res.pop("_mean_latency_s_by_tenant", None)
         if world == 1:
             res["cpu_baseline"] = cpu_baseline(wl)
         print(json.dumps(res), flush=True)

@@ -9,6 +9,7 @@
 //     KL   KlItem into the logical device's ring (host-mapped), the persistent
 //          dispatcher kernel claims it (dispatcher.cu)
 //     D2H  cudaMemcpyAsync on the D2H stream + event
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <time.h>
 #include <unistd.h>
@@ -52,11 +53,33 @@ inline bool cuda_ok(cudaError_t e) {
   return false;
 }
 
+// cudaSetDevice only when the calling thread's current device changes.
+inline void set_dev(int d) {
+  static thread_local int cur = -1;
+  if (cur != d) {
+    cudaSetDevice(d);
+    cur = d;
+  }
+}
+
 uint64_t mono_ns() {
   timespec ts;
   clock_gettime(CLOCK_MONOTONIC, &ts);
   return (uint64_t)ts.tv_sec * 1000000000ull + ts.tv_nsec;
 }
+
+// cuStreamWriteValue32 (driver API, fetched through the runtime: no libcuda link).
+typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+WriteValue32Fn g_write_value32 = nullptr;
+
+// Host-mapped completion counters of one logical device's copy streams: after
+// every H2D / D2H op the stream itself writes the op's sequence number here
+// (stream memory operation, ordered after the copy), so the engine thread
+// detects completion with a plain memory read instead of a driver call.
+struct __align__(64) CopyCounters {
+  volatile uint32_t done[3];          // indexed by engine (H2D = 0, D2H = 2)
+  uint32_t pad[13];
+};
 
 constexpr uint64_t kAlign = 256;
 inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
@@ -80,6 +103,7 @@ struct JobCtx {
   bool issued[3] = {false, false, false};
   bool phys_done[3] = {false, false, false};
   uint32_t kl_seq = 0;
+  uint32_t copy_seq[3] = {0, 0, 0};
   int kl_idx = -1;
   int kl_partition = -1;
   uint64_t kl_t0 = 0, kl_t1 = 0;
@@ -100,6 +124,9 @@ struct Logical {
   KlDone* done = nullptr;              // host pointer, kRing entries
   uint32_t tail = 0;                   // items published
   uint32_t completed = 0;              // items whose completion was consumed
+  CopyCounters* ctr = nullptr;         // host view
+  CUdeviceptr ctr_dev = 0;             // device view
+  uint32_t issued[3] = {0, 0, 0};      // copy ops issued per engine
 };
 
 struct Phys {
@@ -108,6 +135,8 @@ struct Phys {
   int L = 0;
   HostCtrl* ctrl = nullptr;            // host-mapped block
   void* ctrl_dev = nullptr;
+  CopyCounters* ctrs = nullptr;        // host-mapped, one per hosted logical device
+  void* ctrs_dev = nullptr;
   uint8_t* dev_state = nullptr;        // heads + parts
   uint8_t* arena = nullptr;
   bool arena_owned = false;
@@ -350,6 +379,20 @@ class Runtime : public strings::Hooks {
       memset(hp, 0, cb);
       ph->ctrl = static_cast<HostCtrl*>(hp);
       if (!cuda_ok(cudaHostGetDevicePointer(&ph->ctrl_dev, hp, 0))) return STRINGS_ECUDA;
+      void* cp = nullptr;
+      if (!cuda_ok(cudaHostAlloc(&cp, sizeof(CopyCounters) * ph->L, cudaHostAllocMapped | cudaHostAllocPortable)))
+        return STRINGS_ENOMEM;
+      memset(cp, 0, sizeof(CopyCounters) * ph->L);
+      ph->ctrs = static_cast<CopyCounters*>(cp);
+      if (!cuda_ok(cudaHostGetDevicePointer(&ph->ctrs_dev, cp, 0))) return STRINGS_ECUDA;
+      if (!g_write_value32) {
+        cudaDriverEntryPointQueryResult q;
+        void* fn = nullptr;
+        if (!cuda_ok(cudaGetDriverEntryPoint("cuStreamWriteValue32", &fn, cudaEnableDefault, &q)) ||
+            q != cudaDriverEntryPointSuccess || !fn)
+          return STRINGS_ECUDA;
+        g_write_value32 = reinterpret_cast<WriteValue32Fn>(fn);
+      }
       // device state: heads[L] (padded) + parts[L*P]
       size_t heads_bytes = 128 * (size_t)ph->L;
       size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
@@ -377,6 +420,8 @@ class Runtime : public strings::Hooks {
         for (int s = cfg.admit_cap - 1; s >= 0; --s) lg.free_slots.push_back(s);
         lg.ring = rings + lg.local;
         lg.done = dones + (size_t)lg.local * kRing;
+        lg.ctr = ph->ctrs + lg.local;
+        lg.ctr_dev = reinterpret_cast<CUdeviceptr>(static_cast<CopyCounters*>(ph->ctrs_dev) + lg.local);
       }
       for (int i = 0; i < 8 * cfg.awake_budget * ph->L + 16; ++i) {
         cudaEvent_t e;
@@ -424,6 +469,8 @@ class Runtime : public strings::Hooks {
       if (ph->arena && ph->arena_owned) cudaFree(ph->arena);
       if (ph->dev_state) cudaFree(ph->dev_state);
       if (ph->ctrl) cudaFreeHost(ph->ctrl);
+      if (ph->ctrs) cudaFreeHost(ph->ctrs);
+      ph->ctrs = nullptr;
       ph->kstream = nullptr;
       ph->arena = nullptr;
       ph->dev_state = nullptr;
@@ -444,7 +491,7 @@ class Runtime : public strings::Hooks {
     }
     Logical& lg = logical[j.gid];
     Phys* ph = lg.phys;
-    cudaSetDevice(ph->dev);
+    set_dev(ph->dev);
     bool ok = true;
     if (engine == strings::ENG_H2D) {
       if (jc->slot < 0) {
@@ -462,8 +509,7 @@ class Runtime : public strings::Hooks {
         if (jc->in[i].bytes)
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma,
                                        jc->in[i].bytes, cudaMemcpyHostToDevice, lg.h2d));
-      jc->ev[engine] = take_event(ph);
-      ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], lg.h2d));
+      ok = ok && signal_copy(lg, jc, engine, lg.h2d);
     } else if (engine == strings::ENG_D2H) {
       uint64_t off = 0;
       for (size_t i = 0; i < jc->out.size() && ok; ++i) {
@@ -472,8 +518,7 @@ class Runtime : public strings::Hooks {
                                        jc->out[i].bytes, cudaMemcpyDeviceToHost, lg.d2h));
         off = align_up(off + jc->out[i].bytes);
       }
-      jc->ev[engine] = take_event(ph);
-      ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], lg.d2h));
+      ok = ok && signal_copy(lg, jc, engine, lg.d2h);
     } else {
       KlItem it;
       memset(&it, 0, sizeof it);
@@ -585,6 +630,18 @@ class Runtime : public strings::Hooks {
     }
   }
 
+  // Append "done[engine] = seq" to the copy stream (ordered after the copies).
+  bool signal_copy(Logical& lg, JobCtx* jc, int engine, cudaStream_t s) {
+    const uint32_t seq = ++lg.issued[engine];
+    jc->copy_seq[engine] = seq;
+    CUresult r = g_write_value32(reinterpret_cast<CUstream>(s), lg.ctr_dev + engine * sizeof(uint32_t), seq, 0);
+    if (r != CUDA_SUCCESS) {
+      g_last_cuda_error.store(10000 + (int32_t)r);
+      return false;
+    }
+    return true;
+  }
+
   cudaEvent_t take_event(Phys* ph) {
     if (ph->ev_pool.empty()) {
       cudaEvent_t e;
@@ -618,7 +675,14 @@ class Runtime : public strings::Hooks {
       jc->phys_done[engine] = true;
       return true;
     }
-    cudaSetDevice(lg.phys->dev);
+    if (engine != strings::ENG_KL) {
+      const uint32_t d = lg.ctr->done[engine];
+      if ((int32_t)(d - jc->copy_seq[engine]) < 0) return false;
+      std::atomic_thread_fence(std::memory_order_acquire);
+      jc->phys_done[engine] = true;
+      return true;
+    }
+    set_dev(lg.phys->dev);
     cudaError_t e = cudaEventQuery(jc->ev[engine]);
     if (e == cudaErrorNotReady) return false;
     if (e != cudaSuccess) {

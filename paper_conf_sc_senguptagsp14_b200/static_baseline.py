@@ -36,6 +36,7 @@ def _tenant_proc(t: int, dev: int, specs, barrier, out_q, visible: str):
     torch.cuda.synchronize()
     barrier.wait()
     t0 = time.monotonic_ns()
+    ends = []
     for spec, ins, dins, outs, douts in jobs:
         for h, d in zip(ins, dins):
             d.copy_(h)                       # synchronous H2D (pinned)
@@ -47,8 +48,9 @@ def _tenant_proc(t: int, dev: int, specs, barrier, out_q, visible: str):
         torch.cuda.synchronize()             # cudaDeviceSynchronize per job
         for h, d in zip(outs, douts):
             h.copy_(d)                       # synchronous D2H
+        ends.append(time.monotonic_ns())
     t1 = time.monotonic_ns()
-    out_q.put((t, t0, t1, len(jobs)))
+    out_q.put((t, t0, t1, len(jobs), ends))
 
 
 def run_static(wl, num_gpus: int = 1, policy: str = "mod", repeats: int = 1) -> dict:
@@ -61,7 +63,7 @@ def run_static(wl, num_gpus: int = 1, policy: str = "mod", repeats: int = 1) -> 
     by_tenant: List[list] = [[] for _ in wl.tenants]
     for s in wl.jobs:
         by_tenant[s.tenant].append(s)
-    spans = []
+    spans, lats = [], []
     for _ in range(repeats):
         barrier = ctx.Barrier(len(by_tenant))
         q = ctx.Queue()
@@ -77,7 +79,14 @@ def run_static(wl, num_gpus: int = 1, policy: str = "mod", repeats: int = 1) -> 
         t0 = min(r[1] for r in res)
         t1 = max(r[2] for r in res)
         spans.append((t1 - t0) / 1e9)
-    span = sorted(spans)[len(spans) // 2]
+        # mean completion latency per tenant (all jobs arrive at the common start t0)
+        lat = {r[0]: sum(e - t0 for e in r[4]) / max(1, len(r[4])) / 1e9 for r in res}
+        lats.append(lat)
+    order = sorted(range(len(spans)), key=lambda i: spans[i])
+    mid = order[len(order) // 2]
+    span = spans[mid]
     return {"value": len(wl.jobs) / span, "unit": "jobs/s", "span_s": span, "processes": len(by_tenant),
+            "spans_s": [round(x, 4) for x in spans],
+            "mean_latency_s_by_tenant": {int(k): round(v, 6) for k, v in sorted(lats[mid].items())},
             "policy": f"tenant mod {num_gpus}" if policy == "mod" else "device 0",
             "copies": "synchronous cudaMemcpy from pinned host memory", "repeats": repeats}
