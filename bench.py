@@ -41,7 +41,7 @@ METRIC = "tenant jobs/sec (8xB200) vs static CUDA provisioning; Jain fairness"
 def parse_args():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--steps", type=int, default=8)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="strings", choices=["strings", "reference"])
     p.add_argument("--jobs-per-tenant", type=int, default=8)

@@ -169,8 +169,7 @@ cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  const uint32_t smem = it.kclass == 1 ? strings_dev::kSmemGemm : 0;
-  strings_dev::oneshot_kernel<<<ctas, strings_dev::kThreads, smem, s>>>(it);
+  strings_dev::oneshot_kernel<<<ctas, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(it);
   return cudaGetLastError();
 }
 

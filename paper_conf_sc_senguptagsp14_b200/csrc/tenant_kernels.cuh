@@ -29,6 +29,24 @@ struct __align__(16) KlItem {
 };
 static_assert(sizeof(KlItem) == 80, "KlItem layout");
 
+// ---------------------------------------------------------- smem / mbarrier
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t a = smem_u32(bar);
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}"
+      :: "r"(a), "r"(parity) : "memory");
+}
+
 // ---------------------------------------------------------------- streaming
 __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
   h ^= h >> 16;
@@ -58,16 +76,18 @@ __device__ __forceinline__ uint32_t elem_op(uint32_t x, float alpha, uint32_t se
 
 // Vectorised grid-stride stream over the group's CTAs: 8 independent 16-B
 // loads in flight per thread (32 KB per CTA) to cover HBM latency.
+// LDG/STG fallback: vectorised grid-stride over elements [e0, e1) of the group
+// (used for unaligned buffers and for the tail after the bulk-copy chunks).
 template <int KCLASS>
-__device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
-                            float alpha, uint32_t seed, int rank, int S) {
+__device__ void stream_ldg(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t e0, uint64_t e1,
+                           float alpha, uint32_t seed, int rank, int S) {
   constexpr int U = 8;
   const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x;
   const uint64_t nthreads = (uint64_t)S * kThreads;
-  const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
-  uint64_t nvec = aligned ? n / 4 : 0;
-  const uint4* xv = reinterpret_cast<const uint4*>(x);
-  uint4* yv = reinterpret_cast<uint4*>(y);
+  const bool aligned = ((reinterpret_cast<uintptr_t>(x + e0) | reinterpret_cast<uintptr_t>(y + e0)) & 15) == 0;
+  const uint64_t nvec = aligned ? (e1 - e0) / 4 : 0;
+  const uint4* xv = reinterpret_cast<const uint4*>(x + e0);
+  uint4* yv = reinterpret_cast<uint4*>(y + e0);
   uint64_t i = tid;
   for (; i + (U - 1) * nthreads < nvec; i += U * nthreads) {
     uint4 v[U];
@@ -90,7 +110,83 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
     v.w = elem_op<KCLASS>(v.w, alpha, seed);
     st_stream(yv + i, v);
   }
-  for (uint64_t e = nvec * 4 + tid; e < n; e += nthreads) y[e] = elem_op<KCLASS>(x[e], alpha, seed);
+  for (uint64_t e = e0 + nvec * 4 + tid; e < e1; e += nthreads) y[e] = elem_op<KCLASS>(x[e], alpha, seed);
+}
+
+constexpr int kStreamStages = 4;
+constexpr uint32_t kStreamChunk = 48 * 1024;             // bytes per stage (4 x 48 KB = 192 KB)
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(
+                   static_cast<uint32_t>(__cvta_generic_to_shared(bar))), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))), "l"(src), "r"(bytes),
+                  "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+               :: "l"(dst), "r"(static_cast<uint32_t>(__cvta_generic_to_shared(src))), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+// Streaming body: the buffer is cut into 48 KB chunks; chunk c belongs to CTA
+// (c mod S).  Each CTA runs a 4-stage TMA bulk-copy pipeline through shared
+// memory (cp.async.bulk global->smem with mbarrier completion, the element op
+// in smem, cp.async.bulk smem->global), keeping ~192 KB of loads in flight per
+// SM: one half-GPU partition saturates HBM.  Unaligned buffers and the tail
+// use the LDG path.
+template <int KCLASS>
+__device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
+                            float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar) {
+  const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
+  const uint64_t bytes = n * 4;
+  const uint64_t nchunks = aligned ? bytes / kStreamChunk : 0;
+  if (nchunks) {
+    const uint64_t my = (uint64_t)rank < nchunks ? (nchunks - 1 - rank) / S + 1 : 0;
+    if (threadIdx.x == 0) {
+      for (int s = 0; s < kStreamStages; ++s) mbar_init(&sbar[s], 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const uint8_t* xb = reinterpret_cast<const uint8_t*>(x);
+    uint8_t* yb = reinterpret_cast<uint8_t*>(y);
+    if (threadIdx.x == 0)
+      for (int s = 0; s < kStreamStages - 1 && (uint64_t)s < my; ++s) {
+        mbar_expect_tx(&sbar[s], kStreamChunk);
+        bulk_g2s(stage + s * kStreamChunk, xb + (rank + (uint64_t)s * S) * kStreamChunk, kStreamChunk, &sbar[s]);
+      }
+    for (uint64_t i = 0; i < my; ++i) {
+      const int s = (int)(i % kStreamStages);
+      const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
+      if (threadIdx.x == 0 && i + kStreamStages - 1 < my) {
+        const int s2 = (int)((i + kStreamStages - 1) % kStreamStages);
+        // the bulk store that last used stage s2 (issued at iteration i-1) must have read smem
+        asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStages - 2) : "memory");
+        mbar_expect_tx(&sbar[s2], kStreamChunk);
+        bulk_g2s(stage + s2 * kStreamChunk, xb + (rank + (i + kStreamStages - 1) * S) * kStreamChunk,
+                 kStreamChunk, &sbar[s2]);
+      }
+      mbar_wait(&sbar[s], ph);
+      uint4* buf = reinterpret_cast<uint4*>(stage + s * kStreamChunk);
+#pragma unroll 4
+      for (int j = threadIdx.x; j < (int)(kStreamChunk / 16); j += kThreads) {
+        uint4 v = buf[j];
+        v.x = elem_op<KCLASS>(v.x, alpha, seed);
+        v.y = elem_op<KCLASS>(v.y, alpha, seed);
+        v.z = elem_op<KCLASS>(v.z, alpha, seed);
+        v.w = elem_op<KCLASS>(v.w, alpha, seed);
+        buf[j] = v;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // smem writes -> async proxy
+      __syncthreads();
+      if (threadIdx.x == 0) bulk_s2g(yb + (rank + i * S) * kStreamChunk, stage + s * kStreamChunk, kStreamChunk);
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // writes done
+    __syncthreads();
+  }
+  stream_ldg<KCLASS>(x, y, nchunks * (kStreamChunk / 4), n, alpha, seed, rank, S);
 }
 
 // --------------------------------------------------------------------- GEMM
@@ -107,12 +203,8 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
 constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
 constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
 constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
-constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 64;     // + mbarrier / tmem slot
+constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 64;     // + mbarriers / tmem slot (tail, see carve_smem)
 constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
-
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
 
 // Shared-memory matrix descriptor (sm_100 UMMA): start>>4 [0,14), LBO>>4 [16,30),
 // SBO>>4 [32,46), version=1 [46,48), base offset 0, layout SWIZZLE_NONE (0) [61,64).
@@ -130,19 +222,6 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
   return (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(N >> 3) << 17) |
          ((uint32_t)(M >> 4) << 24);
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  uint32_t a = smem_u32(bar);
-  asm volatile(
-      "{\n\t.reg .pred P1;\n"
-      "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-      "@!P1 bra WAIT_%=;\n\t}"
-      :: "r"(a), "r"(parity) : "memory");
 }
 
 __device__ __forceinline__ void tmem_alloc(uint32_t* slot_smem, uint32_t cols) {
@@ -192,6 +271,8 @@ struct GemmSmem {
   uint8_t* b;          // kSmemB bytes
   uint64_t* bar;       // MMA-completion mbarrier
   uint32_t* tmem_slot; // TMEM base written by tcgen05.alloc
+  uint8_t* stage;      // streaming stages (aliases a/b: a CTA runs one item at a time)
+  uint64_t* sbar;      // streaming stage mbarriers [kStreamStages]
 };
 
 // Load the A tile (rows m0..m0+127, all K) and the B tile (all K, cols
@@ -282,11 +363,11 @@ __device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, cons
   switch (it.kclass) {
     case 0:
       stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
       break;
     case 2:
       stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
       break;
     case 1:
       gemm_body(reinterpret_cast<const uint16_t*>(it.in0), reinterpret_cast<const uint16_t*>(it.in1),
@@ -296,12 +377,16 @@ __device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, cons
   }
 }
 
+// smem: [A 64 KB][B 128 KB][tail 64 B: GEMM mbarrier @0, TMEM slot @8, 4 stream mbarriers @16..48]
 __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   GemmSmem s;
   s.a = base;
   s.b = base + kSmemA;
-  s.bar = reinterpret_cast<uint64_t*>(base + kSmemA + kSmemB);
-  s.tmem_slot = reinterpret_cast<uint32_t*>(base + kSmemA + kSmemB + 16);
+  uint8_t* tail = base + kSmemA + kSmemB;
+  s.bar = reinterpret_cast<uint64_t*>(tail);
+  s.tmem_slot = reinterpret_cast<uint32_t*>(tail + 8);
+  s.stage = base;
+  s.sbar = reinterpret_cast<uint64_t*>(tail + 16);
   return s;
 }
 
