@@ -349,6 +349,19 @@ def run_strings(args, rank, world, torch, gloo):
     for inf in last:
         mlat.setdefault(inf.tenant, []).append((inf.t_done[2] - step_t0) / 1e9)
     mlat = {t: sum(v) / len(v) for t, v in mlat.items()}
+    # KL phase: device execution (%globaltimer claim -> last CTA done) vs the
+    # host-observed START -> DONE (adds ring pickup + completion notification)
+    timed = infos[-jobs_step * args.steps:]
+    kl_lat = {}
+    for cls, name in ((W.GEMM, "GEMM"), (W.XFER, "XFER")):
+        rows = [inf for inf, spec in zip(timed, wl.jobs * args.steps) if spec.kclass == cls]
+        dev = sorted((r.kl_gpu_end_ns - r.kl_gpu_start_ns) / 1e3 for r in rows)
+        host = sorted((r.t_done[1] - r.t_start[1]) / 1e3 for r in rows)
+        h2d = sorted((r.t_done[0] - r.t_start[0]) / 1e3 for r in rows)
+        if dev:
+            kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
+                            "kl_host_us_p50": round(host[len(host) // 2], 1),
+                            "h2d_host_us_p50": round(h2d[len(h2d) // 2], 1)}
     kl_items = jobs_step * args.steps
     res = {
         "metric": METRIC, "value": round(value, 3), "unit": "jobs/s", "n_gpus": world,
@@ -374,6 +387,7 @@ def run_strings(args, rank, world, torch, gloo):
         "_mean_latency_s_by_tenant": mlat,
         "jain": round(jain, 4),
         "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step)",
+        "phase_latency": kl_lat,
         "gpu_launches": kl_items,
         "gpu_launches_note": "KL work items executed by the persistent dispatcher kernel (launched once at init)"
                              if args.kl_mode == 0 else "per-job tenant kernel launches",

@@ -116,7 +116,11 @@ typedef struct {
     uint64_t t_start[3], t_done[3];          /* per phase H2D, KL, D2H (library clock)       */
     int32_t  kl_slot;                        /* logical KL slot                               */
     int32_t  kl_partition;                   /* physical SM partition that ran the KL        */
-    uint64_t kl_gpu_start_ns, kl_gpu_end_ns; /* %globaltimer stamps of the KL phase          */
+    uint64_t kl_gpu_start_ns, kl_gpu_end_ns; /* %globaltimer: partition claimed the item, last
+                                                CTA finished                                  */
+    uint64_t kl_gpu_exec_ns;                 /* %globaltimer: the body started (after broadcast) */
+    uint64_t kl_host_issue_ns;               /* CLOCK_REALTIME: item published in the ring     */
+    uint64_t kl_host_observe_ns;             /* CLOCK_REALTIME: completion seen by the engine  */
 } strings_job_info_t;
 
 typedef struct {

@@ -24,7 +24,8 @@ struct __align__(64) KlRing {
 struct __align__(32) KlDone {
   volatile uint32_t seq;              // = item.seq when the item has finished
   uint32_t partition;
-  uint64_t t_start, t_end;            // %globaltimer ns
+  uint64_t t_start, t_end;            // %globaltimer ns: leader claim, last CTA done
+  uint64_t t_exec;                    // %globaltimer ns: leader CTA starts the body
 };
 
 // Host-mapped part (cudaHostAlloc mapped): rings + completions + shutdown flag.
@@ -41,6 +42,7 @@ struct __align__(128) PartState {
   uint32_t done_cnt;                  // CTAs finished with the current generation
   uint32_t ring_idx;
   uint64_t t_start;
+  uint64_t t_exec;
   KlItem item;
 };
 
@@ -51,6 +53,7 @@ struct DispatchParams {
   uint32_t* heads;                    // [L] device-memory claim counters
   PartState* parts;                   // [L * P]
   int L, P;                           // logical devices hosted, partitions per logical device
+  uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
 };
 
 inline size_t host_ctrl_bytes(int L) {

@@ -19,6 +19,7 @@
 #include <chrono>
 #include <condition_variable>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <memory>
@@ -60,6 +61,12 @@ inline void set_dev(int d) {
     cudaSetDevice(d);
     cur = d;
   }
+}
+
+uint64_t real_ns() {
+  timespec ts;
+  clock_gettime(CLOCK_REALTIME, &ts);
+  return (uint64_t)ts.tv_sec * 1000000000ull + ts.tv_nsec;
 }
 
 uint64_t mono_ns() {
@@ -106,7 +113,8 @@ struct JobCtx {
   uint32_t copy_seq[3] = {0, 0, 0};
   int kl_idx = -1;
   int kl_partition = -1;
-  uint64_t kl_t0 = 0, kl_t1 = 0;
+  uint64_t kl_t0 = 0, kl_t1 = 0, kl_exec = 0;     // device %globaltimer: claim, end, body start
+  uint64_t kl_issue = 0, kl_observe = 0;          // host CLOCK_REALTIME: published, completion seen
 };
 
 struct Phys;
@@ -438,6 +446,8 @@ class Runtime : public strings::Hooks {
         dp.parts = reinterpret_cast<strings_dev::PartState*>(ph->dev_state + heads_bytes);
         dp.L = ph->L;
         dp.P = cfg.partitions;
+        const char* fl = getenv("STRINGS_DISPATCH_FLAGS");
+        dp.flags = fl ? (uint32_t)strtoul(fl, nullptr, 0) : 0u;
         if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
       }
@@ -539,6 +549,7 @@ class Runtime : public strings::Hooks {
         } else {
           const uint32_t idx = lg.tail % kRing;
           it.seq = lg.tail + 1;
+          it.t_issue = jc->kl_issue = real_ns();
           KlItem* dst = &lg.ring->items[idx];
           memcpy(dst, &it, sizeof it);
           jc->kl_seq = it.seq;
@@ -671,6 +682,8 @@ class Runtime : public strings::Hooks {
       jc->kl_partition = (int)d->partition;
       jc->kl_t0 = d->t_start;
       jc->kl_t1 = d->t_end;
+      jc->kl_exec = d->t_exec;
+      jc->kl_observe = real_ns();
       lg.completed += 1;
       jc->phys_done[engine] = true;
       return true;
@@ -1058,6 +1071,9 @@ strings_status_t strings_job_info(strings_job_t job, strings_job_info_t* info) {
   info->kl_partition = jc->kl_partition;
   info->kl_gpu_start_ns = jc->kl_t0;
   info->kl_gpu_end_ns = jc->kl_t1;
+  info->kl_gpu_exec_ns = jc->kl_exec;
+  info->kl_host_issue_ns = jc->kl_issue;
+  info->kl_host_observe_ns = jc->kl_observe;
   return STRINGS_OK;
 }
 

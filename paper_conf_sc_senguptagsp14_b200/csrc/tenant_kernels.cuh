@@ -26,8 +26,10 @@ struct __align__(16) KlItem {
   float alpha;
   uint32_t seed;
   uint32_t pad;
+  uint64_t t_issue;      // host CLOCK_REALTIME ns when the item was published (telemetry)
+  uint64_t pad2;
 };
-static_assert(sizeof(KlItem) == 80, "KlItem layout");
+static_assert(sizeof(KlItem) == 96, "KlItem layout");
 
 // ---------------------------------------------------------- smem / mbarrier
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -183,7 +185,10 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       __syncthreads();
       if (threadIdx.x == 0) bulk_s2g(yb + (rank + i * S) * kStreamChunk, stage + s * kStreamChunk, kStreamChunk);
     }
-    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // writes done
+    if (threadIdx.x == 0) {
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");                   // writes done
+      asm volatile("fence.proxy.async.global;" ::: "memory");                     // async -> generic
+    }
     __syncthreads();
   }
   stream_ldg<KCLASS>(x, y, nchunks * (kStreamChunk / 4), n, alpha, seed, rank, S);

@@ -53,7 +53,8 @@ class JobInfo(C.Structure):
     _fields_ = [("job", C.c_uint64), ("tenant", C.c_uint32), ("seq", C.c_uint32), ("gid", C.c_int32),
                 ("status", C.c_int32), ("t_arrival", C.c_uint64), ("t_place", C.c_uint64),
                 ("t_start", C.c_uint64 * 3), ("t_done", C.c_uint64 * 3), ("kl_slot", C.c_int32),
-                ("kl_partition", C.c_int32), ("kl_gpu_start_ns", C.c_uint64), ("kl_gpu_end_ns", C.c_uint64)]
+                ("kl_partition", C.c_int32), ("kl_gpu_start_ns", C.c_uint64), ("kl_gpu_end_ns", C.c_uint64),
+                ("kl_gpu_exec_ns", C.c_uint64), ("kl_host_issue_ns", C.c_uint64), ("kl_host_observe_ns", C.c_uint64)]
 
 
 class Stats(C.Structure):
