@@ -358,6 +358,14 @@ def run_strings(args, rank, world, torch, gloo):
         dev = sorted((r.kl_gpu_end_ns - r.kl_gpu_start_ns) / 1e3 for r in rows)
         host = sorted((r.t_done[1] - r.t_start[1]) / 1e3 for r in rows)
         h2d = sorted((r.t_done[0] - r.t_start[0]) / 1e3 for r in rows)
+        if dev and name == "XFER":
+            # per-op copy rate of the 64 MiB XFER transfers while both directions run
+            # (>= 90% of the measured pinned peak; here vs half the bidir peak)
+            d2h = sorted((r.t_done[2] - r.t_start[2]) / 1e3 for r in rows)
+            nb = 4 * [j for j in wl.jobs if j.kclass == W.XFER][0].n
+            kl_lat["XFER_copy_GBps_p50"] = {"h2d": round(nb / (h2d[len(h2d) // 2] * 1e3), 2),
+                                            "d2h": round(nb / (d2h[len(d2h) // 2] * 1e3), 2),
+                                            "half_bidir_peak": round(link["bidir_gbs"] / 2, 2)}
         if dev:
             kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
                             "kl_host_us_p50": round(host[len(host) // 2], 1),
@@ -443,6 +451,36 @@ def cpu_baseline(wl, sample_jobs: int = 16) -> dict:
             "des_s_full_workload": round(des, 3)}
 
 
+def _oracle_shard(specs):
+    """One worker: generate its jobs' inputs (untimed), then time the oracle on them."""
+    import numpy as np
+    import strings_workload as W
+    from oracle import kernels as K
+    data = [W.job_inputs(s) for s in specs]
+    t = time.perf_counter()
+    for spec, ins in zip(specs, data):
+        outs = K.run_job(spec, [np.copy(a) for a in ins])
+        _ = [np.copy(o) for o in outs]
+    return time.perf_counter() - t
+
+
+def cpu_baseline_all_cores(wl, sample_jobs: int = 64) -> dict:
+    """The same oracle sample spread over every host core (one process per core,
+    BLAS single-threaded inside each): jobs / slowest worker's compute time."""
+    import multiprocessing as mp
+    cores = os.cpu_count() or 1
+    sample = wl.jobs[:sample_jobs]
+    shards = [sample[i::cores] for i in range(cores)]
+    shards = [s for s in shards if s]
+    os.environ.setdefault("OMP_NUM_THREADS", "1")
+    os.environ.setdefault("OPENBLAS_NUM_THREADS", "1")
+    with mp.get_context("fork").Pool(len(shards)) as pool:
+        times = pool.map(_oracle_shard, shards)
+    return {"value": round(len(sample) / max(times), 3), "unit": "jobs/s", "cores": len(shards), "kind": "oracle",
+            "sample": f"first {len(sample)} jobs of C2 split over {len(shards)} processes "
+                      "(inputs generated before timing; value = jobs / slowest worker)"}
+
+
 def run_reference(args):
     """--impl reference: the oracle as it stands on the host cores, same config/metric."""
     import strings_workload as W
@@ -494,6 +532,10 @@ def main():
         res.pop("_mean_latency_s_by_tenant", None)
         if world == 1:
             res["cpu_baseline"] = cpu_baseline(wl)
+            try:
+                res["cpu_baseline_all_cores"] = cpu_baseline_all_cores(wl)
+            except Exception as e:  # pragma: no cover - informational only
+                res["cpu_baseline_all_cores"] = {"error": repr(e)}
         print(json.dumps(res), flush=True)
     if world > 1:
         import torch.distributed as dist

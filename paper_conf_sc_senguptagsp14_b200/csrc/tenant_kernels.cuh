@@ -287,20 +287,24 @@ __device__ inline void gemm_load_tile(const GemmSmem& sm, const uint16_t* __rest
                                       const uint16_t* __restrict__ B, uint64_t N, uint64_t K,
                                       uint64_t m0, uint64_t n0) {
   const int kchunks = (int)(K / 8);
+  // cp.async (LDGSTS) 16-B global->smem copies: no register round trip, every
+  // chunk of the thread in flight at once (the fill is latency-bound otherwise)
+  auto cp16 = [](uint8_t* dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(smem_u32(dst)), "l"(src) : "memory");
+  };
   // A: 16 x kchunks cores; idx -> (rr = row in core, c = k-chunk, g = row group)
   for (int idx = threadIdx.x; idx < kTileM * kchunks; idx += kThreads) {
     const int rr = idx & 7, c = (idx >> 3) % kchunks, g = (idx >> 3) / kchunks;
     const int r = g * 8 + rr;
-    uint4 v = *reinterpret_cast<const uint4*>(A + (m0 + r) * K + (uint64_t)c * 8);
-    *reinterpret_cast<uint4*>(sm.a + ((c * 16 + g) * 128 + rr * 16)) = v;
+    cp16(sm.a + ((c * 16 + g) * 128 + rr * 16), A + (m0 + r) * K + (uint64_t)c * 8);
   }
   // B: 32 x kchunks cores; idx -> (kk = k in core, q = n-group, c = k-chunk)
   for (int idx = threadIdx.x; idx < (int)K * (kTileN / 8); idx += kThreads) {
     const int kk = idx & 7, q = (idx >> 3) & 31, c = idx >> 8;
     const int k = c * 8 + kk;
-    uint4 v = *reinterpret_cast<const uint4*>(B + (uint64_t)k * N + n0 + (uint64_t)q * 8);
-    *reinterpret_cast<uint4*>(sm.b + ((c * 32 + q) * 128 + kk * 16)) = v;
+    cp16(sm.b + ((c * 32 + q) * 128 + kk * 16), B + (uint64_t)k * N + n0 + (uint64_t)q * 8);
   }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
   // make generic-proxy smem writes visible to the tensor core (async proxy)
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
