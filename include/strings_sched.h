@@ -129,6 +129,8 @@ typedef struct {
     uint64_t h2d_bytes, d2h_bytes, kernel_bytes, kernel_flop;
     uint64_t trace_records;
     uint64_t decisions;                           /* PLACE + WAKE records                       */
+    uint64_t decision_ns;                         /* engine time inside the decision core,
+                                                     including issuing the woken ops            */
     uint64_t engine_busy_ns[8][3];                /* per logical device (first 8), per engine   */
     int32_t  num_gpus, physical_gpus, partitions, sms_per_partition;
 } strings_stats_t;

@@ -58,6 +58,7 @@ int Core::add_tenant(uint32_t weight, uint32_t max_inflight) {
   t.weight = weight;
   t.c = max_inflight;
   tenants_.push_back(t);
+  sft_.resize(tenants_.size() * 3);
   return static_cast<int>(tenants_.size()) - 1;
 }
 
@@ -72,23 +73,54 @@ void Core::add_job(Job* j) {
 uint64_t Core::next_arrival() const { return arr_.empty() ? UINT64_MAX : (*arr_.begin())->arrival; }
 
 // ---------------------------------------------------------------- trace
+namespace {
+inline char* put_u64(char* p, uint64_t v) {
+  char tmp[24];
+  int n = 0;
+  do {
+    tmp[n++] = char('0' + v % 10);
+    v /= 10;
+  } while (v);
+  while (n) *p++ = tmp[--n];
+  return p;
+}
+inline char* put_opt(char* p, long v) {
+  if (v < 0) {
+    *p++ = '-';
+    return p;
+  }
+  return put_u64(p, (uint64_t)v);
+}
+inline char* put_str(char* p, const char* s) {
+  while (*s) *p++ = *s++;
+  return p;
+}
+}  // namespace
+
 void Core::rec(uint64_t t, const char* kind, int gid, int eng, int slot, long tenant, long seq,
                long job, uint64_t a1, uint64_t a2) {
   char buf[256];
-  char f[5][24];
-  auto put = [&](int i, long v) {
-    if (v < 0) snprintf(f[i], sizeof f[i], "-");
-    else snprintf(f[i], sizeof f[i], "%ld", v);
-  };
-  put(0, gid);
-  put(1, slot);
-  put(2, tenant);
-  put(3, seq);
-  put(4, job);
-  int n = snprintf(buf, sizeof buf, "%llu %s %s %s %s %s %s %s %llu %llu\n",
-                   (unsigned long long)t, kind, f[0], eng < 0 ? "-" : kEngName[eng], f[1], f[2],
-                   f[3], f[4], (unsigned long long)a1, (unsigned long long)a2);
-  trace_.append(buf, n);
+  char* p = put_u64(buf, t);
+  *p++ = ' ';
+  p = put_str(p, kind);
+  *p++ = ' ';
+  p = put_opt(p, gid);
+  *p++ = ' ';
+  p = put_str(p, eng < 0 ? "-" : kEngName[eng]);
+  *p++ = ' ';
+  p = put_opt(p, slot);
+  *p++ = ' ';
+  p = put_opt(p, tenant);
+  *p++ = ' ';
+  p = put_opt(p, seq);
+  *p++ = ' ';
+  p = put_opt(p, job);
+  *p++ = ' ';
+  p = put_u64(p, a1);
+  *p++ = ' ';
+  p = put_u64(p, a2);
+  *p++ = '\n';
+  trace_.append(buf, p - buf);
   ++trace_records_;
 }
 
@@ -114,15 +146,11 @@ bool Core::admission_before(const Job* a, const Job* b) const {
 }
 
 // ---------------------------------------------------------- predictions
-bool Core::has_sample(const Job* j) const {
-  auto it = sft_.find({j->tenant, j->kclass});
-  return it != sft_.end() && it->second.count > 0;
-}
+bool Core::has_sample(const Job* j) const { return sft_[j->tenant * 3 + j->kclass].count > 0; }
 
 Core::Pred Core::pred(const Job* j) const {
-  auto it = sft_.find({j->tenant, j->kclass});
-  if (it != sft_.end() && it->second.count > 0)
-    return {it->second.h2d, it->second.kl, it->second.d2h, it->second.util};
+  const SftRow& r = sft_[j->tenant * 3 + j->kclass];
+  if (r.count > 0) return {r.h2d, r.kl, r.d2h, r.util};
   Pred p;
   p.h2d = cdiv(j->h2d_bytes, kPriorLinkBytesPerNs);
   p.d2h = cdiv(j->d2h_bytes, kPriorLinkBytesPerNs);
@@ -138,60 +166,60 @@ int Core::effective_policy(const Job* j) const {
   return b == B_DYNAMIC ? B_MBF : b;
 }
 
-uint64_t Core::score(int policy, const Job* j, const Device& d) const {
+Core::Agg Core::aggregate(const Device& d) const {
+  Agg a;
+  a.n = d.resident.size();
+  for (const Job* r : d.resident) {
+    Pred q = pred(r);
+    const uint64_t h = r->phase <= ENG_H2D ? q.h2d : 0;
+    const uint64_t k = r->phase <= ENG_KL ? q.kl : 0;
+    const uint64_t dd = r->phase <= ENG_D2H ? q.d2h : 0;
+    a.rem_total += h + k + dd;                   // RTF: predicted remaining runtime
+    a.util += q.util;                            // GUF: summed utilisation
+    a.copy += h + dd;                            // DTF: remaining transfer time
+    a.kl += k;                                   //      and remaining kernel time
+    a.h2d += h;                                  // MBF: per-resource busy time
+    a.d2h += dd;
+    if (r->phase <= ENG_KL) {
+      const uint64_t hb = std::min(q.kl, cdiv(r->hbm_bytes, kPriorHbmBytesPerNs));
+      a.hbm += hb;
+      a.sm += q.kl - hb;
+    }
+  }
+  return a;
+}
+
+// Balancer score of placing j on a device with aggregates a (minimised; R-13).
+uint64_t Core::score_from(int policy, const Agg& a, const Job* j) const {
   switch (policy) {
     case B_GMIN:
     case B_GWTMIN:
-      return d.resident.size();
-    case B_RTF: {                       // predicted remaining runtime
-      uint64_t s = 0;
-      for (const Job* r : d.resident) {
-        Pred p = pred(r);
-        if (r->phase <= ENG_H2D) s += p.h2d;
-        if (r->phase <= ENG_KL) s += p.kl;
-        if (r->phase <= ENG_D2H) s += p.d2h;
-      }
+      return a.n;
+    case B_RTF: {
       Pred p = pred(j);
-      return s + p.h2d + p.kl + p.d2h;
+      return a.rem_total + p.h2d + p.kl + p.d2h;
     }
-    case B_GUF: {                       // summed GPU utilisation (L827)
-      uint64_t s = pred(j).util;
-      for (const Job* r : d.resident) s += pred(r).util;
-      return s;
-    }
-    case B_DTF: {                       // transfer vs compute balance (L829)
+    case B_GUF:                         // L827
+      return a.util + pred(j).util;
+    case B_DTF: {                       // L829
       Pred p = pred(j);
-      uint64_t copy = p.h2d + p.d2h, kern = p.kl;
-      for (const Job* r : d.resident) {
-        Pred q = pred(r);
-        if (r->phase <= ENG_H2D) copy += q.h2d;
-        if (r->phase <= ENG_D2H) copy += q.d2h;
-        if (r->phase <= ENG_KL) kern += q.kl;
-      }
-      return std::max(copy, kern);
+      return std::max(a.copy + p.h2d + p.d2h, a.kl + p.kl);
     }
-    case B_MBF: {                       // bandwidth-bound co-location (L831)
-      uint64_t sh = 0, sd = 0, shbm = 0, ssm = 0;
-      auto add = [&](const Job* r, bool all) {
-        Pred q = pred(r);
-        if (all || r->phase <= ENG_H2D) sh += q.h2d;
-        if (all || r->phase <= ENG_D2H) sd += q.d2h;
-        if (all || r->phase <= ENG_KL) {
-          uint64_t hb = std::min(q.kl, cdiv(r->hbm_bytes, kPriorHbmBytesPerNs));
-          shbm += hb;
-          ssm += q.kl - hb;
-        }
-      };
-      for (const Job* r : d.resident) add(r, false);
-      add(j, true);
-      return std::max(std::max(sh, sd), std::max(shbm, ssm));
+    case B_MBF: {                       // L831
+      Pred p = pred(j);
+      const uint64_t hb = std::min(p.kl, cdiv(j->hbm_bytes, kPriorHbmBytesPerNs));
+      return std::max(std::max(a.h2d + p.h2d, a.d2h + p.d2h), std::max(a.hbm + hb, a.sm + p.kl - hb));
     }
   }
   throw std::logic_error("score: policy");
 }
 
+uint64_t Core::score(int policy, const Job* j, const Device& d) const {
+  return score_from(policy, aggregate(d), j);
+}
+
 int Core::select_device(int policy, const Job* j, const std::vector<int>& adm,
-                        uint64_t* score_out) {
+                        const std::vector<Agg>& aggs, uint64_t* score_out) {
   if (policy == B_GRR) {
     for (int k = 0; k < cfg_.G; ++k) {
       int g = (grr_cursor_ + k) % cfg_.G;
@@ -216,7 +244,7 @@ int Core::select_device(int policy, const Job* j, const std::vector<int>& adm,
   int best = -1;
   uint64_t bs = 0;
   for (int g : adm) {                   // ties -> lowest GID (L687)
-    uint64_t s = score(policy, j, devs_[g]);
+    uint64_t s = score_from(policy, aggs[g], j);
     if (best < 0 || s < bs) {
       best = g;
       bs = s;
@@ -230,17 +258,25 @@ int Core::select_device(int policy, const Job* j, const std::vector<int>& adm,
 void Core::admission(uint64_t t) {
   const bool joint = cfg_.joint &&
                      (cfg_.balancer == B_DTF || cfg_.balancer == B_MBF || cfg_.balancer == B_DYNAMIC);
-  std::vector<Job*> elig;
-  std::vector<int> adm;
+  std::vector<Job*>& elig = scratch_elig_;
+  std::vector<int>& adm = scratch_adm_;
+  std::vector<Agg>& aggs = scratch_aggs_;
+  aggs.resize(devs_.size());
+  const bool need_aggs = cfg_.balancer != B_GRR && cfg_.balancer != B_GMIN && cfg_.balancer != B_GWTMIN;
   for (;;) {
     elig.clear();
     adm.clear();
+    for (auto& d : devs_)
+      if ((int)d.resident.size() < cfg_.M) adm.push_back(d.gid);
+    if (adm.empty()) return;
     for (auto& tn : tenants_)
       if (!tn.pending.empty() && tn.inflight < tn.c && tn.pending.front()->arrived)
         elig.push_back(tn.pending.front());
-    for (auto& d : devs_)
-      if ((int)d.resident.size() < cfg_.M) adm.push_back(d.gid);
-    if (elig.empty() || adm.empty()) return;
+    if (elig.empty()) return;
+    for (int g : adm) {
+      if (need_aggs) aggs[g] = aggregate(devs_[g]);
+      else aggs[g].n = devs_[g].resident.size();
+    }
     std::sort(elig.begin(), elig.end(),
               [this](const Job* a, const Job* b) { return admission_before(a, b); });
     Job* pick = nullptr;
@@ -254,13 +290,13 @@ void Core::admission(uint64_t t) {
         }
       if (pick) {
         pol = B_GMIN;
-        gid = select_device(pol, pick, adm, &sc);
+        gid = select_device(pol, pick, adm, aggs, &sc);
       } else {
         bool have = false;
         for (Job* j : elig) {
           int p = effective_policy(j);
           for (int g : adm) {
-            uint64_t s = score(p, j, devs_[g]);
+            uint64_t s = score_from(p, aggs[g], j);
             if (!have || s < sc) {
               have = true;
               sc = s;
@@ -274,7 +310,7 @@ void Core::admission(uint64_t t) {
     } else {
       pick = elig.front();
       pol = effective_policy(pick);
-      gid = select_device(pol, pick, adm, &sc);
+      gid = select_device(pol, pick, adm, aggs, &sc);
     }
     place(t, pick, gid, pol, sc);
   }
@@ -305,7 +341,8 @@ void Core::wake(uint64_t t, Device& d, Job* j) {
 }
 
 void Core::dispatch(uint64_t t, Device& d) {
-  std::vector<Job*> cand;
+  std::vector<Job*>& cand = scratch_cand_;
+  cand.clear();
   for (Job* j : d.resident)
     if (j->phase < 3 && !j->woken) cand.push_back(j);
   int budget = cfg_.A - d.woken_unfinished;
@@ -317,9 +354,10 @@ void Core::dispatch(uint64_t t, Device& d) {
       std::sort(cand.begin(), cand.end(), by_key);
       for (size_t i = 0; i < cand.size() && budget > 0; ++i, --budget) wake(t, d, cand[i]);
     } else {                                        // Phase Selection, L819 (R-11)
-      std::vector<Job*> ph[3];
+      std::vector<Job*>* ph = scratch_ph_;
+      for (int x = 0; x < 3; ++x) ph[x].clear();
       for (Job* j : cand) ph[j->phase].push_back(j);
-      for (auto& v : ph) std::sort(v.begin(), v.end(), by_key);
+      for (int x = 0; x < 3; ++x) std::sort(ph[x].begin(), ph[x].end(), by_key);
       int active[3];
       for (int x = 0; x < 3; ++x) {
         active[x] = (int)d.fifo[x].size();
@@ -350,7 +388,8 @@ void Core::dispatch(uint64_t t, Device& d) {
         wake(t, d, ph[ENG_KL][head[ENG_KL]++]);
         --budget;
       }
-      std::vector<Job*> copies;
+      std::vector<Job*>& copies = scratch_copies_;
+      copies.clear();
       for (size_t i = head[ENG_H2D]; i < ph[ENG_H2D].size(); ++i) copies.push_back(ph[ENG_H2D][i]);
       for (size_t i = head[ENG_D2H]; i < ph[ENG_D2H].size(); ++i) copies.push_back(ph[ENG_D2H][i]);
       std::sort(copies.begin(), copies.end(), by_key);
@@ -412,7 +451,7 @@ void Core::feedback(uint64_t t, Job* j) {
   for (int x = 0; x < 3; ++x) smp[x] = j->done[x] - j->start[x];
   uint64_t span = t - j->t_place;
   uint64_t util = span ? (smp[ENG_KL] * 65536) / span : 0;
-  SftRow& r = sft_[{j->tenant, j->kclass}];
+  SftRow& r = sft_[j->tenant * 3 + j->kclass];
   if (r.count == 0) {
     r.h2d = smp[0];
     r.kl = smp[1];

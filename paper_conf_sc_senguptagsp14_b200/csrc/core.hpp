@@ -18,6 +18,7 @@
 #include <deque>
 #include <map>
 #include <set>
+#include <unordered_map>
 #include <string>
 #include <vector>
 
@@ -119,6 +120,14 @@ class Core {
     int woken_unfinished = 0;
   };
   struct Pred { uint64_t h2d, kl, d2h, util; };
+  // Per-device sums over resident jobs' remaining predicted work (every balancer
+  // score is such a sum plus the new job's term; integer sums, so computing them
+  // once per admission round gives the same values as summing per candidate).
+  struct Agg {
+    uint64_t n = 0, rem_total = 0, util = 0, copy = 0, kl = 0, h2d = 0, d2h = 0, hbm = 0, sm = 0;
+  };
+  Agg aggregate(const Device& d) const;
+  uint64_t score_from(int policy, const Agg& a, const Job* j) const;
 
   void rec(uint64_t t, const char* kind, int gid, int eng, int slot, long tenant, long seq,
            long job, uint64_t a1, uint64_t a2);
@@ -130,7 +139,8 @@ class Core {
   bool has_sample(const Job* j) const;
   int effective_policy(const Job* j) const;
   uint64_t score(int policy, const Job* j, const Device& d) const;
-  int select_device(int policy, const Job* j, const std::vector<int>& adm, uint64_t* score_out);
+  int select_device(int policy, const Job* j, const std::vector<int>& adm, const std::vector<Agg>& aggs,
+                    uint64_t* score_out);
 
   void admission(uint64_t t);
   void place(uint64_t t, Job* j, int gid, int policy, uint64_t score);
@@ -145,7 +155,7 @@ class Core {
   Hooks* hooks_;
   std::vector<Tenant> tenants_;
   std::vector<Device> devs_;
-  std::map<std::pair<uint32_t, int>, SftRow> sft_;
+  std::vector<SftRow> sft_;           // [tenant * 3 + class]
   struct ArrLess {
     bool operator()(const Job* a, const Job* b) const {
       if (a->arrival != b->arrival) return a->arrival < b->arrival;
@@ -154,7 +164,7 @@ class Core {
     }
   };
   std::set<Job*, ArrLess> arr_;       // submitted, not yet arrived
-  std::map<uint64_t, Job*> jobs_;     // id -> job (unfinished)
+  std::unordered_map<uint64_t, Job*> jobs_;   // id -> job (unfinished)
   uint64_t jobs_total_ = 0, jobs_done_ = 0;
   uint64_t epoch_start_ = 0, next_epoch_;
   int grr_cursor_ = 0;
@@ -163,6 +173,10 @@ class Core {
   std::string trace_;
   uint64_t trace_records_ = 0, decisions_ = 0;
   std::vector<std::vector<uint64_t>> busy_ns_;
+  // scratch buffers reused by the hot paths (no per-call heap allocation)
+  std::vector<Job*> scratch_cand_, scratch_ph_[3], scratch_copies_, scratch_elig_;
+  std::vector<int> scratch_adm_;
+  std::vector<Agg> scratch_aggs_;
 };
 
 // Algorithmic kernel bytes and tensor FLOP of a job.

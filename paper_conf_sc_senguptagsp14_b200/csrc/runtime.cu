@@ -292,6 +292,7 @@ class Runtime : public strings::Hooks {
   uint64_t submitted = 0, done_count = 0, failed_count = 0;
   uint64_t first_submit = 0, last_done = 0;
   uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
+  uint64_t decision_ns = 0;            // time inside Core::step (decisions + op issue)
   // in-flight physical ops (measured mode): (job, engine)
   std::vector<std::pair<JobCtx*, int>> inflight;
   // virtual DONE events (injected / decisions-only)
@@ -766,7 +767,9 @@ class Runtime : public strings::Hooks {
           lk.lock();
         }
       }
+      const uint64_t d0 = mono_ns();
       core->step(t, std::move(batch), first);
+      decision_ns += mono_ns() - d0;
       first = false;
       if (vheap.empty() || vheap.top().t != t) break;
     }
@@ -805,7 +808,9 @@ class Runtime : public strings::Hooks {
       }
       if (batch.empty() && !first) break;
       if (batch.empty() && !progressed && core->next_epoch() != t) break;
+      const uint64_t d0 = mono_ns();
       core->step(t, std::move(batch), first);
+      decision_ns += mono_ns() - d0;
       first = false;
       progressed = false;
     }
@@ -1094,6 +1099,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->kernel_flop = r.kflop_total;
   st->trace_records = r.core->trace_records();
   st->decisions = r.core->decisions();
+  st->decision_ns = r.decision_ns;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

@@ -62,6 +62,7 @@ class Stats(C.Structure):
                 ("t_first_submit_ns", C.c_uint64), ("t_last_done_ns", C.c_uint64),
                 ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64), ("kernel_bytes", C.c_uint64),
                 ("kernel_flop", C.c_uint64), ("trace_records", C.c_uint64), ("decisions", C.c_uint64),
+                ("decision_ns", C.c_uint64),
                 ("engine_busy_ns", (C.c_uint64 * 3) * 8), ("num_gpus", C.c_int32),
                 ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32)]
 
