@@ -57,6 +57,8 @@ typedef uint64_t strings_job_t;
 #define STRINGS_DEV_FIFO 0      /* wake in placement order (baseline)                          */
 #define STRINGS_DEV_LAS  1      /* least attained service, weighted, phase-blind (R-7) */
 #define STRINGS_DEV_PS   2      /* Phase Selection: one per phase, else KL > H2D = D2H */
+#define STRINGS_DEV_TFS  3      /* True Fair-Share: one tenant awake, weight-proportional slices,
+                                   service-history penalty, work conserving    */
 
 /* Tenant kernel classes (the paper's workload classes, Table I). */
 #define STRINGS_VSCALE 0        /* y = alpha * x, fp32, n elements          (memory-bound)      */
@@ -75,7 +77,7 @@ typedef struct {
     int32_t  physical_gpus;  /* physical GPUs to use (first N visible); 0 = all visible         */
     int32_t  balancer;       /* STRINGS_BAL_*                                                   */
     int32_t  las_admission;  /* 1 = admit pending jobs in weighted-LAS order (R-9)              */
-    int32_t  device_policy;  /* STRINGS_DEV_*                                                   */
+    int32_t  device_policy;  /* STRINGS_DEV_* (FIFO, LAS, PS, TFS)                              */
     int32_t  partitions;     /* P KL slots (SM partitions) per device; 0 -> 2                   */
     int32_t  awake_budget;   /* A woken-unfinished ops per device; 0 -> 2 + P (R-11)            */
     int32_t  admit_cap;      /* M resident jobs per device; 0 -> 2 * A (R-12)                   */
@@ -85,7 +87,8 @@ typedef struct {
     uint64_t slot_bytes;     /* device bytes per resident job slot; 0 -> 160 MiB                */
     const char* trace_path;  /* if non-NULL the decision trace is written there at drain/shutdown */
     int32_t  trace_in_memory;/* 1 = keep the trace for strings_trace_copy                       */
-    int32_t  reserved[7];
+    int32_t  reserved[7];    /* reserved[0] = 1: KL phases as per-job launches (profiling)      */
+    uint64_t tfs_slice_ns;   /* TFS base slice S: a tenant of weight w is awake for w*S; 0 -> 500 us */
 } strings_config_t;
 
 /* Kernel descriptor: which tenant kernel the KL phase runs, and its sizes.

@@ -17,6 +17,8 @@ Paper passages (PAPER.md line numbers, section):
   LAS            L693  §IV.B.1      least attained service first (weighted, R-7)
   Eq. (1)        L695               CGS_n = k*GS_n + (1-k)*CGS_{n-1}, k = 0.8 (integer form R-4)
   PS             L819  §IV.B.3      wake threads in different phases, else KL > H2D = D2H > DFL (R-11)
+  TFS            L699, L817 §IV.B.2 at most one tenant awake, weight-proportional slices, penalty
+                                    for overshoot via weighted service history, work-conserving (R-28)
   RTF/GUF/DTF/MBF L823-831 §IV.C    feedback placement policies (scores R-13)
   Policy arbiter L311, L1073        switch on sufficient feedback (R-15)
   RCB / SFT / DST L309-313, L489-515, Fig 6
@@ -104,6 +106,9 @@ class Device:
     busy: List[List[Optional[int]]] = field(default_factory=list)  # per engine, per slot
     woken_unfinished: int = 0
     weight: int = 1        # DST device weight (L309); equal on identical B200s
+    awake: Optional[int] = None          # TFS: the tenant currently awake on this device
+    awake_used: int = 0                  # TFS: its service on this device since it woke
+    svc: Dict[int, int] = field(default_factory=dict)   # TFS: cumulative service per tenant
 
     def __post_init__(self):
         self.busy = [[None], [None] * self.P, [None]]
@@ -126,6 +131,7 @@ class Oracle:
         self.cfg = cfg
         self.G, self.P, self.A, self.M, self.Q = (cfg.num_gpus, cfg.partitions, cfg.awake_budget,
                                                   cfg.admit_cap, cfg.quantum_ns)
+        self.S = cfg.tfs_slice_ns
         assert self.G >= 1 and self.P >= 1 and self.A >= 1 and self.M >= 1 and self.Q >= 1
         self.tenants = [Tenant(weight=t.weight, c=t.max_inflight) for t in wl.tenants]
         self.jobs: List[Job] = []
@@ -362,8 +368,12 @@ class Oracle:
                     if free > 0:
                         self.wake(t, d, j)
                         free -= 1
+            elif pol == W.TFS:                        # L699, L817 (R-28)
+                self.tfs_wake(t, d, cands, free)
             else:
                 raise ValueError(pol)
+        elif pol == W.TFS:
+            self.tfs_wake(t, d, cands, free)         # release bookkeeping even with no budget
         # start pass: free engines / slots take their FIFO heads
         for x in (H2D, KL, D2H):
             for s in range(len(d.busy[x])):
@@ -373,6 +383,34 @@ class Oracle:
                     j.start[x], j.slot[x] = t, s
                     self.rec(t, "START", d.gid, x, s, j.tenant, j.seq, j.id)
                     heapq.heappush(self.done_heap, (t + j.dur[x], d.gid, x, s, j.id))
+
+    def tfs_wake(self, t, d: Device, cands: List[Job], free: int) -> None:
+        """True Fair-Share: only the awake tenant's ops may be woken (at most one
+        backend thread awake, L699).  It stays awake until it has used w_t * S of
+        service on this device since it woke, or has nothing to run (work
+        conserving, L817); it is released only once its woken ops finished.  The
+        next tenant is the one with the least service / weight on this device
+        (cumulative, so an overshoot is paid back in later turns, L817)."""
+        if d.awake is not None:
+            w = self.tenants[d.awake].weight
+            mine = [j for j in cands if j.tenant == d.awake]
+            if d.woken_unfinished == 0 and (d.awake_used >= w * self.S or not mine):
+                d.awake = None
+        if d.awake is None:
+            best = None
+            for tid in sorted({j.tenant for j in cands}):
+                if best is None or d.svc.get(tid, 0) * self.tenants[best].weight < \
+                        d.svc.get(best, 0) * self.tenants[tid].weight:
+                    best = tid
+            if best is not None:
+                d.awake, d.awake_used = best, 0
+        if d.awake is None or d.awake_used >= self.tenants[d.awake].weight * self.S:
+            return
+        for j in sorted((j for j in cands if j.tenant == d.awake), key=lambda j: j.place_order):
+            if free <= 0:
+                break
+            self.wake(t, d, j)
+            free -= 1
 
     # -------------------------------------------------------------- completions
     def complete(self, t, gid, x, s, jid) -> None:
@@ -385,6 +423,9 @@ class Oracle:
         j.phase += 1
         j.woken = False
         tn.gs_acc += t - max(j.start[x], self.epoch_start)
+        d.svc[j.tenant] = d.svc.get(j.tenant, 0) + (t - j.start[x])
+        if d.awake == j.tenant:
+            d.awake_used += t - j.start[x]
         self.rec(t, "DONE", gid, x, s, j.tenant, j.seq, jid, t - j.start[x])
         if x == D2H:
             j.t_jobdone = t

@@ -16,7 +16,10 @@ Checks the invariants of SURVEY.md §8(c) on a canonical trace
       starts after job s's.  Jobs admitted concurrently (c_t > 1, the finite
       server threads of L879) are independent requests (reading R-27).
   I5  work conservation at the end of every timestamp: no engine idles while
-      an op is woken for it; no candidate stays unwoken while budget remains.
+      an op is woken for it; no candidate stays unwoken while budget remains
+      (TFS: no device sits with candidates and nothing woken).
+  I7  TFS: the woken-unfinished ops of a device belong to at
+      most one tenant at any time.
 """
 from __future__ import annotations
 
@@ -132,7 +135,10 @@ def check(lines: List[str], wl: W.Workload) -> List[str]:
                 if fifo[g][x] and any(b is None for b in busy[g][x]):
                     errs.append(f"I5 t={t} gid={g} engine {x} idle with woken op")
             c = candidates(g)
-            if c and woken_unf[g] < A:
+            if cfg.device_policy == W.TFS:
+                if c and woken_unf[g] == 0:
+                    errs.append(f"I5 t={t} gid={g} TFS device idle with {len(c)} candidates")
+            elif c and woken_unf[g] < A:
                 errs.append(f"I5 t={t} gid={g} {len(c)} candidates unwoken with budget {A - woken_unf[g]}")
             if cfg.device_policy == W.LAS:
                 for w in woken_now.get(g, []):
@@ -182,6 +188,10 @@ def check(lines: List[str], wl: W.Workload) -> List[str]:
             j, g, x = r.job, r.gid, r.eng
             if phase[j] != x or woken[j]:
                 errs.append(f"I1 job {j} woken for phase {x} out of order")
+            if cfg.device_policy == W.TFS:
+                others = {ten_of[i] for i in resident[g] if woken[i]} - {ten_of[j]}
+                if others:
+                    errs.append(f"I7 t={r.t} gid={g} TFS woke tenant {ten_of[j]} while {others} awake")
             woken[j] = True
             fifo[g][x].append(j)
             woken_unf[g] += 1

@@ -347,7 +347,9 @@ void Core::dispatch(uint64_t t, Device& d) {
     if (j->phase < 3 && !j->woken) cand.push_back(j);
   int budget = cfg_.A - d.woken_unfinished;
   auto by_key = [this](const Job* a, const Job* b) { return las_before(a, b); };
-  if (!cand.empty() && budget > 0) {
+  if (cfg_.device_policy == P_TFS) {
+    tfs_dispatch(t, d, cand, budget);
+  } else if (!cand.empty() && budget > 0) {
     if (cfg_.device_policy == P_FIFO) {
       for (size_t i = 0; i < cand.size() && budget > 0; ++i, --budget) wake(t, d, cand[i]);
     } else if (cfg_.device_policy == P_LAS) {       // phase-blind
@@ -399,6 +401,45 @@ void Core::dispatch(uint64_t t, Device& d) {
   start_pass(t, d);
 }
 
+// True Fair-Share (R-28).  At most one tenant is awake on
+// a device; it keeps the device for w_t * S of service (ops are not preempted),
+// or until it has nothing left to run (work conserving), and is released only
+// once its woken ops have finished.  The next tenant is the one with the least
+// cumulative service / weight on this device, which pays back any overshoot.
+void Core::tfs_dispatch(uint64_t t, Device& d, const std::vector<Job*>& cand, int budget) {
+  if (d.svc.size() < tenants_.size()) d.svc.resize(tenants_.size(), 0);
+  if (d.awake >= 0) {
+    const uint64_t slice = (uint64_t)tenants_[d.awake].weight * cfg_.tfs_slice;
+    bool has_work = false;
+    for (const Job* j : cand) has_work |= (long)j->tenant == d.awake;
+    if (d.woken_unfinished == 0 && (d.awake_used >= slice || !has_work)) d.awake = -1;
+  }
+  if (d.awake < 0) {
+    long best = -1;
+    for (const Job* j : cand) {
+      const long tid = j->tenant;
+      if (best < 0) {
+        best = tid;
+        continue;
+      }
+      const unsigned __int128 lhs = (unsigned __int128)d.svc[tid] * tenants_[best].weight;
+      const unsigned __int128 rhs = (unsigned __int128)d.svc[best] * tenants_[tid].weight;
+      if (lhs < rhs || (lhs == rhs && tid < best)) best = tid;
+    }
+    if (best >= 0) {
+      d.awake = best;
+      d.awake_used = 0;
+    }
+  }
+  if (d.awake < 0 || d.awake_used >= (uint64_t)tenants_[d.awake].weight * cfg_.tfs_slice) return;
+  for (Job* j : cand) {                         // placement order
+    if (budget <= 0) break;
+    if ((long)j->tenant != d.awake) continue;
+    wake(t, d, j);
+    --budget;
+  }
+}
+
 void Core::start_pass(uint64_t t, Device& d) {
   for (int x = 0; x < 3; ++x) {
     for (size_t s = 0; s < d.busy[x].size(); ++s) {
@@ -429,6 +470,9 @@ void Core::complete(const Completion& c) {
   j->phase += 1;
   j->woken = false;
   busy_ns_[c.gid][c.engine] += t - j->start[c.engine];
+  if (d.svc.size() < tenants_.size()) d.svc.resize(tenants_.size(), 0);
+  d.svc[j->tenant] += t - j->start[c.engine];
+  if (d.awake == (long)j->tenant) d.awake_used += t - j->start[c.engine];
   Tenant& tn = tenants_[j->tenant];
   tn.gs_acc += t - std::max(j->start[c.engine], epoch_start_);
   rec(t, "DONE", c.gid, c.engine, c.slot, j->tenant, j->seq, (long)j->id, t - j->start[c.engine], 0);

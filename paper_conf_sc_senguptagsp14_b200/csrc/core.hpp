@@ -27,12 +27,13 @@ namespace strings {
 enum Engine : int { ENG_H2D = 0, ENG_KL = 1, ENG_D2H = 2 };
 enum KClass : int { K_VSCALE = 0, K_GEMM = 1, K_XFER = 2 };
 enum Balancer : int { B_GRR = 0, B_GMIN, B_GWTMIN, B_RTF, B_GUF, B_DTF, B_MBF, B_DYNAMIC };
-enum DevPolicy : int { P_FIFO = 0, P_LAS = 1, P_PS = 2 };
+enum DevPolicy : int { P_FIFO = 0, P_LAS = 1, P_PS = 2, P_TFS = 3 };
 
 struct CoreConfig {
   int G = 1, P = 2, A = 4, M = 8;
   int balancer = B_GMIN, las_admission = 0, device_policy = P_PS, joint = 0;
   uint64_t Q = 1000000;
+  uint64_t tfs_slice = 500000;        // TFS base slice S (R-28)
 };
 
 // One job's scheduling record (the RCB view of a request).
@@ -118,6 +119,10 @@ class Core {
     std::deque<Job*> fifo[3];
     std::vector<Job*> busy[3];        // H2D: 1 slot, KL: P slots, D2H: 1 slot
     int woken_unfinished = 0;
+    // True Fair-Share (R-28)
+    long awake = -1;                  // tenant awake on this device, -1 = none
+    uint64_t awake_used = 0;          // its service here since it woke
+    std::vector<uint64_t> svc;        // cumulative service per tenant on this device
   };
   struct Pred { uint64_t h2d, kl, d2h, util; };
   // Per-device sums over resident jobs' remaining predicted work (every balancer
@@ -145,6 +150,7 @@ class Core {
   void admission(uint64_t t);
   void place(uint64_t t, Job* j, int gid, int policy, uint64_t score);
   void dispatch(uint64_t t, Device& d);
+  void tfs_dispatch(uint64_t t, Device& d, const std::vector<Job*>& cand, int budget);
   void wake(uint64_t t, Device& d, Job* j);
   void start_pass(uint64_t t, Device& d);
   void complete(const Completion& c);

@@ -322,7 +322,8 @@ class Runtime : public strings::Hooks {
     if (cfg.admit_cap <= 0) cfg.admit_cap = 2 * cfg.awake_budget;
     if (cfg.quantum_ns == 0) cfg.quantum_ns = 1000000;
     if (cfg.slot_bytes == 0) cfg.slot_bytes = 160ull << 20;
-    if (cfg.balancer < 0 || cfg.balancer > 7 || cfg.device_policy < 0 || cfg.device_policy > 2 ||
+    if (cfg.tfs_slice_ns == 0) cfg.tfs_slice_ns = 500000;
+    if (cfg.balancer < 0 || cfg.balancer > 7 || cfg.device_policy < 0 || cfg.device_policy > 3 ||
         cfg.timing_mode < 0 || cfg.timing_mode > 2)
       return STRINGS_EINVAL;
     kl_mode = cfg.reserved[0] == 1 ? 1 : 0;
@@ -344,6 +345,7 @@ class Runtime : public strings::Hooks {
     ccfg.device_policy = cfg.device_policy;
     ccfg.joint = cfg.joint_select;
     ccfg.Q = cfg.quantum_ns;
+    ccfg.tfs_slice = cfg.tfs_slice_ns;
     cfg.physical_gpus = nphys;
     core.reset(new strings::Core(ccfg, this));
     logical.resize(cfg.num_gpus);

@@ -38,8 +38,8 @@ CLASS_NAMES = {VSCALE: "VSCALE", GEMM: "GEMM", XFER: "XFER"}
 
 GRR, GMIN, GWTMIN, RTF, GUF, DTF, MBF, DYNAMIC = range(8)
 BALANCER_NAMES = ["GRR", "GMIN", "GWTMIN", "RTF", "GUF", "DTF", "MBF", "DYNAMIC"]
-FIFO, LAS, PS = 0, 1, 2
-DEVICE_POLICY_NAMES = ["FIFO", "LAS", "PS"]
+FIFO, LAS, PS, TFS = 0, 1, 2, 3
+DEVICE_POLICY_NAMES = ["FIFO", "LAS", "PS", "TFS"]
 
 # Nominal rates used ONLY to make injected durations (inputs).  Integer
 # bytes/ns and FLOP/ns; see DESIGN.md §5 "Injected durations".
@@ -132,6 +132,7 @@ class SystemConfig:
     admit_cap: int = 0         # M (0 -> 2 * A)
     quantum_ns: int = 1_000_000
     joint_select: int = -1     # -1 auto (on for DTF/MBF/DYNAMIC)
+    tfs_slice_ns: int = 500_000  # TFS base slice S (a tenant of weight w is awake for w*S of service)
 
     def resolved(self) -> "SystemConfig":
         c = SystemConfig(**asdict(self))
@@ -344,7 +345,7 @@ def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs
         num_gpus=int(r.integers(1, max_gpus + 1)),
         balancer=int(r.integers(0, 8)),
         las_admission=int(r.integers(0, 2)),
-        device_policy=int(r.integers(0, 3)),
+        device_policy=int(r.integers(0, 4)),
         partitions=int(r.integers(1, 4)),
         quantum_ns=int(r.choice([1_000, 7_919, 100_000, 1_000_000])),
     )
@@ -354,6 +355,8 @@ def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs
         cfg.admit_cap = int(r.integers(1, 8))
     if r.integers(0, 2) == 0:
         cfg.joint_select = int(r.integers(0, 2))
+    if cfg.device_policy == TFS:
+        cfg.tfs_slice_ns = int(r.choice([1, 5_000, 100_000, 500_000]))
     T = int(r.integers(1, max_tenants + 1))
     tenants = [TenantSpec(weight=int(r.integers(1, 9)), max_inflight=int(r.integers(1, 4)))
                for _ in range(T)]

@@ -141,3 +141,23 @@ def test_sync_per_tenant_and_unregister():
         assert st.jobs_done == 12 and st.jobs_failed == 0
     finally:
         S.shutdown()
+
+
+@pytest.mark.parametrize("weights,slice_ns", [((1, 1), 500_000), ((2, 1), 200_000), ((1, 3), 1)])
+def test_tfs_fair_share_trace_matches_oracle(weights, slice_ns):
+    cfg = W.SystemConfig(num_gpus=1, partitions=1, device_policy=W.TFS, admit_cap=1000, tfs_slice_ns=slice_ns)
+    jobs = []
+    for t, size in ((0, 200_000), (1, 50_000)):
+        jobs += [W.JobSpec(tenant=t, kclass=W.VSCALE, n=0, inj_kl_ns=size) for _ in range(60)]
+    wl = W.Workload("tfs", cfg, [W.TenantSpec(weight=w, max_inflight=1000) for w in weights], jobs)
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+    assert r.trace == o.trace
+    assert invariants.check(r.trace, wl) == []
+
+
+@pytest.mark.parametrize("name", ["C1", "C3", "C5"])
+def test_tfs_on_configs_matches_oracle(name):
+    wl = W.CONFIGS[name]()
+    wl.config.device_policy = W.TFS
+    assert run_workload(wl, timing_mode=S.DECISIONS_ONLY).trace == run_oracle(wl).trace

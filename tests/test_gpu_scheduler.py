@@ -88,6 +88,19 @@ def test_measured_mode_invariants_and_outputs(name, kw):
     assert all(i.kl_gpu_end_ns >= i.kl_gpu_start_ns > 0 for i in r.infos)
 
 
+@pytest.mark.parametrize("timing", [S.INJECTED, S.MEASURED])
+def test_tfs_on_hardware(timing):
+    wl = W.config_c1(reps=4)
+    wl.config.device_policy = W.TFS
+    wl.config.tfs_slice_ns = 20_000
+    r = run_workload(wl, timing_mode=timing)
+    assert r.status == S.OK
+    if timing == S.INJECTED:
+        assert r.trace == run_oracle(wl).trace
+    assert invariants.check(r.trace, wl) == []       # incl. I7: one tenant awake per device
+    check_outputs(wl, r)
+
+
 def test_pageable_buffers_are_staged():
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)
