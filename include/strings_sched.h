@@ -87,7 +87,9 @@ typedef struct {
     uint64_t slot_bytes;     /* device bytes per resident job slot; 0 -> 160 MiB                */
     const char* trace_path;  /* if non-NULL the decision trace is written there at drain/shutdown */
     int32_t  trace_in_memory;/* 1 = keep the trace for strings_trace_copy                       */
-    int32_t  reserved[7];    /* reserved[0] = 1: KL phases as per-job launches (profiling)      */
+    int32_t  kl_mode;        /* 0 = persistent dispatcher kernel (product); 1 = per-job launches of
+                                the same bodies on per-slot streams (profilers that replay kernels) */
+    int32_t  reserved[6];
     uint64_t tfs_slice_ns;   /* TFS base slice S: a tenant of weight w is awake for w*S; 0 -> 500 us */
 } strings_config_t;
 

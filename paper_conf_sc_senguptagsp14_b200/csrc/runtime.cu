@@ -326,7 +326,8 @@ class Runtime : public strings::Hooks {
     if (cfg.balancer < 0 || cfg.balancer > 7 || cfg.device_policy < 0 || cfg.device_policy > 3 ||
         cfg.timing_mode < 0 || cfg.timing_mode > 2)
       return STRINGS_EINVAL;
-    kl_mode = cfg.reserved[0] == 1 ? 1 : 0;
+    if (cfg.kl_mode < 0 || cfg.kl_mode > 1) return STRINGS_EINVAL;
+    kl_mode = cfg.kl_mode;
     int nphys = 0;
     if (has_gpu()) {
       if (!cuda_ok(cudaGetDeviceCount(&nphys)) || nphys <= 0) return STRINGS_ECUDA;

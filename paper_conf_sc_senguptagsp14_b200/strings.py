@@ -35,7 +35,7 @@ class Config(C.Structure):
                 ("awake_budget", C.c_int32), ("admit_cap", C.c_int32), ("joint_select", C.c_int32),
                 ("timing_mode", C.c_int32), ("quantum_ns", C.c_uint64), ("slot_bytes", C.c_uint64),
                 ("trace_path", C.c_char_p), ("trace_in_memory", C.c_int32),
-                ("reserved", C.c_int32 * 7), ("tfs_slice_ns", C.c_uint64)]
+                ("kl_mode", C.c_int32), ("reserved", C.c_int32 * 6), ("tfs_slice_ns", C.c_uint64)]
 
 
 class KernelDesc(C.Structure):
@@ -133,8 +133,7 @@ def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy
                admit_cap=admit_cap, joint_select=joint_select, timing_mode=timing_mode,
                quantum_ns=quantum_ns, slot_bytes=slot_bytes,
                trace_path=trace_path.encode() if trace_path else None,
-               trace_in_memory=1 if trace_in_memory else 0, tfs_slice_ns=tfs_slice_ns)
-    c.reserved[0] = kl_mode
+               trace_in_memory=1 if trace_in_memory else 0, kl_mode=kl_mode, tfs_slice_ns=tfs_slice_ns)
     _check(lib.strings_init(C.byref(c)), "strings_init")
 
 

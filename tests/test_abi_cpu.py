@@ -161,3 +161,21 @@ def test_tfs_on_configs_matches_oracle(name):
     wl = W.CONFIGS[name]()
     wl.config.device_policy = W.TFS
     assert run_workload(wl, timing_mode=S.DECISIONS_ONLY).trace == run_oracle(wl).trace
+
+
+def test_slot_size_and_mode_validation():
+    S.init(num_gpus=1, timing_mode=S.DECISIONS_ONLY, slot_bytes=1 << 20)
+    try:
+        t = S.register_tenant()
+        big = S.HostRef(1, 4 << 20)
+        with pytest.raises(S.StringsError) as e:      # 4 MiB in + 4 MiB out > 1 MiB slot
+            S.submit(t, S.make_desc(S.VSCALE, n=1 << 20), [big], [big])
+        assert e.value.status == S.EINVAL
+    finally:
+        S.shutdown()
+    for bad in (dict(kl_mode=2), dict(device_policy=4), dict(balancer=-1)):
+        with pytest.raises(S.StringsError):
+            S.init(timing_mode=S.DECISIONS_ONLY, **bad)
+    with pytest.raises(S.StringsError) as e:
+        S.init(timing_mode=3)
+    assert e.value.status == S.EINVAL
