@@ -56,6 +56,8 @@ def parse_args():
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
+    p.add_argument("--sweep", action="store_true",
+                   help="policy comparison on C2 (device policies x balancers) vs static; not the driver line")
     return p.parse_args()
 
 
@@ -511,8 +513,61 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def policy_sweep(args) -> None:
+    """Paper-style policy comparison (Figs 12-15 analogue) on C2, one B200."""
+    import numpy as np
+    import torch
+
+    import strings_workload as W
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+    from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
+
+    base = W.config_c2(jobs_per_tenant=args.jobs_per_tenant)
+    ins = [[torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory() for a in W.job_inputs(sp)]
+           for sp in base.jobs]
+    outs = [[torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in sp.d2h_sizes()] for sp in base.jobs]
+    st = run_static(base, num_gpus=1, repeats=3)
+    static_lat = st["mean_latency_s_by_tenant"]
+    rows = []
+    combos = [(W.DTF, d) for d in (W.FIFO, W.LAS, W.PS, W.TFS)] + \
+             [(b, W.PS) for b in (W.GRR, W.GMIN, W.RTF, W.GUF, W.MBF, W.DYNAMIC)]
+    for bal, dev in combos:
+        cfg = W.config_c2(jobs_per_tenant=args.jobs_per_tenant).config
+        cfg.balancer, cfg.device_policy = bal, dev
+        cfg = cfg.resolved()
+        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1)
+        tenants = [S.register_tenant(t.weight, t.max_inflight) for t in base.tenants]
+        spans, lat = [], {}
+        for step in range(2 + args.steps):
+            t0 = time.perf_counter()
+            first = None
+            for i, sp in enumerate(base.jobs):
+                jid = S.submit_spec(tenants[sp.tenant], sp, ins[i], outs[i])
+                first = jid if first is None else first
+            assert S.drain() == S.OK
+            if step >= 2:
+                spans.append(time.perf_counter() - t0)
+                infos = [S.job_info(first + i) for i in range(len(base.jobs))]
+                t_arr = min(x.t_arrival for x in infos)
+                for x in infos:
+                    lat.setdefault(x.tenant, []).append((x.t_done[2] - t_arr) / 1e9)
+        S.shutdown()
+        mlat = {t: sum(v) / len(v) for t, v in lat.items()}
+        ws = sum(static_lat[t] / mlat[t] for t in mlat) / len(mlat)
+        xs = [1.0 / mlat[t] for t in mlat]          # progress rate per tenant (equal weights)
+        jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+        rows.append({"balancer": W.BALANCER_NAMES[bal], "device_policy": W.DEVICE_POLICY_NAMES[dev],
+                     "jobs_per_s": round(len(base.jobs) / statistics.median(spans), 1),
+                     "weighted_speedup_vs_static": round(ws, 3), "jain_progress": round(jain, 4)})
+        print(json.dumps(rows[-1]), flush=True)
+    print(json.dumps({"sweep": "C2 on 1 B200", "static_jobs_per_s": round(st["value"], 1), "rows": rows}))
+
+
 def main():
     args = parse_args()
+    if args.sweep:
+        policy_sweep(args)
+        return
     from paper_conf_sc_senguptagsp14_b200 import parallel as par
     info = par.rank_info()
     world, rank = info.world, info.rank
