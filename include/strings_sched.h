@@ -91,6 +91,9 @@ typedef struct {
                                 the same bodies on per-slot streams (profilers that replay kernels) */
     int32_t  reserved[6];
     uint64_t tfs_slice_ns;   /* TFS base slice S: a tenant of weight w is awake for w*S; 0 -> 500 us */
+    const uint32_t* device_weights; /* num_gpus DST weights >= 1 (GWtMin); NULL = all 1.
+                                       Logical devices sharing a physical GPU get SM partitions
+                                       in proportion to their weights (heterogeneous pool).     */
 } strings_config_t;
 
 /* Kernel descriptor: which tenant kernel the KL phase runs, and its sizes.

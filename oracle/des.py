@@ -146,7 +146,7 @@ class Oracle:
                 arrival=s.arrival_ns, h2d_bytes=sum(s.h2d_sizes()), d2h_bytes=sum(s.d2h_sizes()),
                 hbm_bytes=hbm, tflop=fl, dur=(s.inj_h2d_ns, s.inj_kl_ns, s.inj_d2h_ns)))
             self.tenants[s.tenant].pending.append(i)
-        self.devices = [Device(gid=d, P=self.P) for d in range(self.G)]
+        self.devices = [Device(gid=d, P=self.P, weight=cfg.device_weights[d]) for d in range(self.G)]
         self.sft: Dict[Tuple[int, int], SFTEntry] = {}
         self.arrival_order = sorted(range(len(self.jobs)),
                                     key=lambda i: (self.jobs[i].arrival, self.jobs[i].tenant, self.jobs[i].seq))

@@ -47,6 +47,7 @@ Core::Core(const CoreConfig& cfg, Hooks* hooks) : cfg_(cfg), hooks_(hooks), next
   busy_ns_.assign(cfg_.G, std::vector<uint64_t>(3, 0));
   for (int g = 0; g < cfg_.G; ++g) {
     devs_[g].gid = g;
+    devs_[g].weight = g < (int)cfg_.weights.size() ? cfg_.weights[g] : 1;
     devs_[g].busy[ENG_H2D].assign(1, nullptr);
     devs_[g].busy[ENG_KL].assign(cfg_.P, nullptr);
     devs_[g].busy[ENG_D2H].assign(1, nullptr);

@@ -34,6 +34,7 @@ struct CoreConfig {
   int balancer = B_GMIN, las_admission = 0, device_policy = P_PS, joint = 0;
   uint64_t Q = 1000000;
   uint64_t tfs_slice = 500000;        // TFS base slice S (R-28)
+  std::vector<uint32_t> weights;      // DST device weights; empty = all 1
 };
 
 // One job's scheduling record (the RCB view of a request).

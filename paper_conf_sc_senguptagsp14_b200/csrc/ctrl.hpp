@@ -52,6 +52,7 @@ struct DispatchParams {
   KlDone* done;                       // [L * kRing]
   uint32_t* heads;                    // [L] device-memory claim counters
   PartState* parts;                   // [L * P]
+  const int* part_start;              // [L * P + 1] first CTA of each partition (device memory)
   int L, P;                           // logical devices hosted, partitions per logical device
   uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
 };

@@ -42,13 +42,14 @@ __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
 
-__device__ __forceinline__ void partition_of(int b, int G, int NP, int* q, int* start, int* S) {
-  int p = (int)(((long long)b * NP) / G);
-  while (p + 1 < NP && (int)(((long long)(p + 1) * G) / NP) <= b) ++p;
-  while (p > 0 && (int)(((long long)p * G) / NP) > b) --p;
+// Partition q owns CTAs [part_start[q], part_start[q+1]) (sized on the host by
+// logical-device weight, then split evenly into P KL slots).
+__device__ __forceinline__ void partition_of(int b, int NP, const int* part_start, int* q, int* start, int* S) {
+  int p = 0;
+  while (p + 1 < NP && part_start[p + 1] <= b) ++p;
   *q = p;
-  *start = (int)(((long long)p * G) / NP);
-  *S = (int)(((long long)(p + 1) * G) / NP) - *start;
+  *start = part_start[p];
+  *S = part_start[p + 1] - part_start[p];
 }
 
 __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams p) {
@@ -58,7 +59,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   GemmSmem sm = carve_smem(smem);
   const int NP = p.L * p.P;
   int q, start, S;
-  partition_of(blockIdx.x, gridDim.x, NP, &q, &start, &S);
+  partition_of(blockIdx.x, NP, p.part_start, &q, &start, &S);
   const int rank = blockIdx.x - start;
   const int ld = q / p.P;
   PartState* ps = p.parts + q;

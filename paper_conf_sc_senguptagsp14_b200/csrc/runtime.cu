@@ -134,6 +134,7 @@ struct Logical {
   uint32_t completed = 0;              // items whose completion was consumed
   CopyCounters* ctr = nullptr;         // host view
   CUdeviceptr ctr_dev = 0;             // device view
+  int ctas = 0;                        // CTAs (SMs) of this logical device's partitions
   uint32_t issued[3] = {0, 0, 0};      // copy ops issued per engine
 };
 
@@ -150,6 +151,7 @@ struct Phys {
   bool arena_owned = false;
   cudaStream_t kstream = nullptr;
   bool kernel_running = false;
+  std::vector<int> part_start;         // [L*P + 1] partition table (host copy)
   std::vector<cudaEvent_t> ev_pool;
 };
 
@@ -277,6 +279,7 @@ class Runtime : public strings::Hooks {
   strings_config_t cfg{};
   strings::CoreConfig ccfg;
   int kl_mode = 0;                     // 0 persistent, 1 launch (profiling)
+  std::vector<uint32_t> weights;       // DST weight per logical device
   std::unique_ptr<strings::Core> core;
   std::vector<std::unique_ptr<Phys>> phys;
   std::vector<Logical> logical;
@@ -347,6 +350,15 @@ class Runtime : public strings::Hooks {
     ccfg.joint = cfg.joint_select;
     ccfg.Q = cfg.quantum_ns;
     ccfg.tfs_slice = cfg.tfs_slice_ns;
+    weights.assign(cfg.num_gpus, 1);
+    if (cfg.device_weights) {
+      for (int g = 0; g < cfg.num_gpus; ++g) {
+        if (cfg.device_weights[g] == 0) return STRINGS_EINVAL;
+        weights[g] = cfg.device_weights[g];
+      }
+    }
+    cfg.device_weights = nullptr;            // the caller's array need not outlive init
+    ccfg.weights = weights;
     cfg.physical_gpus = nphys;
     core.reset(new strings::Core(ccfg, this));
     logical.resize(cfg.num_gpus);
@@ -383,6 +395,28 @@ class Runtime : public strings::Hooks {
       if (!cuda_ok(cudaGetDeviceProperties(&prop, ph->dev))) return STRINGS_ECUDA;
       ph->sms = prop.multiProcessorCount;
       if (ph->L * cfg.partitions > ph->sms) return STRINGS_EINVAL;
+      // SM shares: logical devices of this GPU get CTAs in proportion to their
+      // weights, each share split evenly into P partitions (one per KL slot)
+      {
+        uint64_t wsum = 0;
+        std::vector<int> lds;
+        for (auto& lg : logical)
+          if (lg.phys == ph.get()) lds.push_back(lg.gid), wsum += weights[lg.gid];
+        ph->part_start.assign(1, 0);
+        uint64_t wacc = 0;
+        for (size_t i = 0; i < lds.size(); ++i) {
+          const int lo = ph->part_start.back();
+          wacc += weights[lds[i]];
+          int hi = (int)((uint64_t)ph->sms * wacc / wsum);
+          hi = std::max(hi, lo + cfg.partitions);
+          const int remaining_ld = (int)(lds.size() - 1 - i);
+          hi = std::min(hi, ph->sms - remaining_ld * cfg.partitions);
+          if (i + 1 == lds.size()) hi = ph->sms;
+          for (int p = 1; p <= cfg.partitions; ++p)
+            ph->part_start.push_back(lo + (int)((int64_t)(hi - lo) * p / cfg.partitions));
+          logical[lds[i]].ctas = hi - lo;
+        }
+      }
       // host-mapped control block
       size_t cb = strings_dev::host_ctrl_bytes(ph->L);
       void* hp = nullptr;
@@ -405,11 +439,15 @@ class Runtime : public strings::Hooks {
           return STRINGS_ECUDA;
         g_write_value32 = reinterpret_cast<WriteValue32Fn>(fn);
       }
-      // device state: heads[L] (padded) + parts[L*P]
+      // device state: heads[L] (padded) + parts[L*P] + partition table
       size_t heads_bytes = 128 * (size_t)ph->L;
       size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
-      if (!cuda_ok(cudaMalloc(&ph->dev_state, heads_bytes + parts_bytes))) return STRINGS_ENOMEM;
+      size_t table_bytes = sizeof(int) * ph->part_start.size();
+      if (!cuda_ok(cudaMalloc(&ph->dev_state, heads_bytes + parts_bytes + table_bytes))) return STRINGS_ENOMEM;
       if (!cuda_ok(cudaMemset(ph->dev_state, 0, heads_bytes + parts_bytes))) return STRINGS_ECUDA;
+      if (!cuda_ok(cudaMemcpy(ph->dev_state + heads_bytes + parts_bytes, ph->part_start.data(), table_bytes,
+                              cudaMemcpyHostToDevice)))
+        return STRINGS_ECUDA;
       if (!cuda_ok(cudaDeviceSynchronize())) return STRINGS_ECUDA;   // zeroed before the dispatcher starts
       // arena: L logical devices x M slots
       size_t arena = (size_t)ph->L * cfg.admit_cap * cfg.slot_bytes;
@@ -448,6 +486,7 @@ class Runtime : public strings::Hooks {
         dp.done = reinterpret_cast<KlDone*>(dbase + sizeof(HostCtrl) + sizeof(KlRing) * ph->L);
         dp.heads = reinterpret_cast<uint32_t*>(ph->dev_state);
         dp.parts = reinterpret_cast<strings_dev::PartState*>(ph->dev_state + heads_bytes);
+        dp.part_start = reinterpret_cast<const int*>(ph->dev_state + heads_bytes + parts_bytes);
         dp.L = ph->L;
         dp.P = cfg.partitions;
         const char* fl = getenv("STRINGS_DISPATCH_FLAGS");
@@ -566,7 +605,7 @@ class Runtime : public strings::Hooks {
       } else {
         cudaStream_t s = lg.kl_streams[lg.next_kl_stream];
         lg.next_kl_stream = (lg.next_kl_stream + 1) % (int)lg.kl_streams.size();
-        int ctas = ph->sms / (ph->L * cfg.partitions);
+        int ctas = std::max(1, lg.ctas / cfg.partitions);
         ok = cuda_ok(strings::launch_oneshot(it, ctas, s));
         jc->ev[engine] = take_event(ph);
         ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], s));
@@ -1108,7 +1147,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->num_gpus = r.cfg.num_gpus;
   st->physical_gpus = r.cfg.physical_gpus;
   st->partitions = r.cfg.partitions;
-  if (!r.phys.empty() && r.phys[0]->L > 0) st->sms_per_partition = r.phys[0]->sms / (r.phys[0]->L * r.cfg.partitions);
+  if (!r.logical.empty() && r.logical[0].ctas > 0) st->sms_per_partition = r.logical[0].ctas / r.cfg.partitions;
   return STRINGS_OK;
 }
 

@@ -35,7 +35,8 @@ class Config(C.Structure):
                 ("awake_budget", C.c_int32), ("admit_cap", C.c_int32), ("joint_select", C.c_int32),
                 ("timing_mode", C.c_int32), ("quantum_ns", C.c_uint64), ("slot_bytes", C.c_uint64),
                 ("trace_path", C.c_char_p), ("trace_in_memory", C.c_int32),
-                ("kl_mode", C.c_int32), ("reserved", C.c_int32 * 6), ("tfs_slice_ns", C.c_uint64)]
+                ("kl_mode", C.c_int32), ("reserved", C.c_int32 * 6), ("tfs_slice_ns", C.c_uint64),
+                ("device_weights", C.POINTER(C.c_uint32))]
 
 
 class KernelDesc(C.Structure):
@@ -127,13 +128,16 @@ def _check(s: int, where: str) -> None:
 def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy=2, partitions=2,
          awake_budget=0, admit_cap=0, joint_select=-1, timing_mode=MEASURED, quantum_ns=1_000_000,
          slot_bytes=0, trace_path: Optional[str] = None, trace_in_memory=True, kl_mode=0,
-         tfs_slice_ns=0) -> None:
+         tfs_slice_ns=0, device_weights: Optional[Sequence[int]] = None) -> None:
     c = Config(num_gpus=num_gpus, physical_gpus=physical_gpus, balancer=balancer, las_admission=las_admission,
                device_policy=device_policy, partitions=partitions, awake_budget=awake_budget,
                admit_cap=admit_cap, joint_select=joint_select, timing_mode=timing_mode,
                quantum_ns=quantum_ns, slot_bytes=slot_bytes,
                trace_path=trace_path.encode() if trace_path else None,
                trace_in_memory=1 if trace_in_memory else 0, kl_mode=kl_mode, tfs_slice_ns=tfs_slice_ns)
+    if device_weights is not None:
+        arr = (C.c_uint32 * len(device_weights))(*device_weights)
+        c.device_weights = C.cast(arr, C.POINTER(C.c_uint32))
     _check(lib.strings_init(C.byref(c)), "strings_init")
 
 
@@ -142,7 +146,7 @@ def init_from_config(cfg, timing_mode=MEASURED, **kw) -> None:
     init(num_gpus=cfg.num_gpus, balancer=cfg.balancer, las_admission=cfg.las_admission,
          device_policy=cfg.device_policy, partitions=cfg.partitions, awake_budget=cfg.awake_budget,
          admit_cap=cfg.admit_cap, joint_select=cfg.joint_select, quantum_ns=cfg.quantum_ns,
-         tfs_slice_ns=cfg.tfs_slice_ns, timing_mode=timing_mode, **kw)
+         tfs_slice_ns=cfg.tfs_slice_ns, device_weights=cfg.device_weights, timing_mode=timing_mode, **kw)
 
 
 def register_tenant(weight: int = 1, max_inflight: int = 1) -> int:

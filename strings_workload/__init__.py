@@ -133,6 +133,7 @@ class SystemConfig:
     quantum_ns: int = 1_000_000
     joint_select: int = -1     # -1 auto (on for DTF/MBF/DYNAMIC)
     tfs_slice_ns: int = 500_000  # TFS base slice S (a tenant of weight w is awake for w*S of service)
+    device_weights: Optional[List[int]] = None   # DST weights per logical device (None = all 1)
 
     def resolved(self) -> "SystemConfig":
         c = SystemConfig(**asdict(self))
@@ -142,6 +143,8 @@ class SystemConfig:
             c.admit_cap = 2 * c.awake_budget
         if c.joint_select < 0:
             c.joint_select = 1 if c.balancer in (DTF, MBF, DYNAMIC) else 0
+        if c.device_weights is None:
+            c.device_weights = [1] * c.num_gpus
         return c
 
 
@@ -357,6 +360,8 @@ def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs
         cfg.joint_select = int(r.integers(0, 2))
     if cfg.device_policy == TFS:
         cfg.tfs_slice_ns = int(r.choice([1, 5_000, 100_000, 500_000]))
+    if r.integers(0, 3) == 0:
+        cfg.device_weights = [int(x) for x in r.integers(1, 4, cfg.num_gpus)]
     T = int(r.integers(1, max_tenants + 1))
     tenants = [TenantSpec(weight=int(r.integers(1, 9)), max_inflight=int(r.integers(1, 4)))
                for _ in range(T)]

@@ -179,3 +179,18 @@ def test_slot_size_and_mode_validation():
     with pytest.raises(S.StringsError) as e:
         S.init(timing_mode=3)
     assert e.value.status == S.EINVAL
+
+
+def test_heterogeneous_gwtmin_parity_and_validation():
+    wl = W.config_c3()
+    wl.config.balancer = W.GWTMIN
+    wl.config.device_weights = [3, 2, 2, 1]
+    o = run_oracle(wl)
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+    assert r.trace == o.trace
+    # the first placements at t=0 follow load/weight: the weight-3 device gets 3 of the first 8
+    first8 = [int(l.split()[2]) for l in r.trace if " PLACE " in l][:8]
+    assert first8.count(0) == 3 and first8.count(3) == 1
+    with pytest.raises(S.StringsError) as e:
+        S.init(num_gpus=2, timing_mode=S.DECISIONS_ONLY, device_weights=[1, 0])
+    assert e.value.status == S.EINVAL

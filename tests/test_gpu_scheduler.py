@@ -101,6 +101,23 @@ def test_tfs_on_hardware(timing):
     check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("timing", [S.INJECTED, S.MEASURED])
+def test_heterogeneous_logical_devices(timing):
+    # NEXT-4: four logical devices with DST weights 3:2:2:1 share the B200; their
+    # SM partitions are sized by weight and GWtMin places by load / weight
+    wl = W.config_c3(scale=4, reps=8)
+    wl.config.balancer = W.GWTMIN
+    wl.config.device_weights = [3, 2, 2, 1]
+    r = run_workload(wl, timing_mode=timing)
+    assert r.status == S.OK
+    if timing == S.INJECTED:
+        assert r.trace == run_oracle(wl).trace
+    assert invariants.check(r.trace, wl) == []
+    check_outputs(wl, r)
+    P = wl.config.partitions
+    assert all(i.kl_partition // P == i.gid for i in r.infos)   # KL ran on its own device's SMs
+
+
 def test_pageable_buffers_are_staged():
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)

@@ -394,3 +394,20 @@ def test_ps_relaxes_tfs_for_throughput():
         o = run_oracle(wl)
         spans[pol] = max(j.t_jobdone for j in o.jobs)
     assert spans[W.PS] < spans[W.TFS]
+
+
+# ------------------------------------------------------- heterogeneous GWtMin
+@pytest.mark.parametrize("weights,jobs", [((2, 1, 1), 12), ((3, 1), 8), ((1, 2, 3), 18)])
+def test_gwtmin_places_in_proportion_to_device_weights(weights, jobs):
+    # weighted minimum load; with identical jobs placed before any
+    # completes, the counts end up proportional to the weights (count/w equalised)
+    cfg = W.SystemConfig(num_gpus=len(weights), balancer=W.GWTMIN, admit_cap=10 ** 6,
+                         device_weights=list(weights))
+    wl = W.Workload("gw", cfg, [W.TenantSpec(max_inflight=10 ** 6)], [kl_only_job(0, 10 ** 6) for _ in range(jobs)])
+    pl = placements(run_oracle(wl))
+    counts = [pl.count(g) for g in range(len(weights))]
+    assert counts == [w * jobs // sum(weights) for w in weights]
+    # GMin ignores the weights: equal counts
+    cfg.balancer = W.GMIN
+    pl = placements(run_oracle(wl))
+    assert max(pl.count(g) for g in range(len(weights))) - min(pl.count(g) for g in range(len(weights))) <= 1
