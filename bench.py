@@ -56,6 +56,8 @@ def parse_args():
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
+    p.add_argument("--fig2", action="store_true",
+                   help="Fig. 2 analogue: N identical requests sequential vs co-resident vs separate contexts")
     p.add_argument("--sweep", action="store_true",
                    help="policy comparison on C2 (device policies x balancers) vs static; not the driver line")
     return p.parse_args()
@@ -563,8 +565,51 @@ def policy_sweep(args) -> None:
     print(json.dumps({"sweep": "C2 on 1 B200", "static_jobs_per_s": round(st["value"], 1), "rows": rows}))
 
 
+def fig2(args) -> None:
+    """PAPER.md L67-73 (Fig. 2): identical MonteCarlo-like requests issued one
+    after another vs co-resident on streams of one context.  Here: 8 identical
+    transfer-heavy XFER jobs (64 MiB each way) (a) from one tenant, strictly
+    sequential; (b) from 8 tenants co-scheduled by Strings (PS); (c) from 8
+    separate processes/contexts (static provisioning)."""
+    import numpy as np
+    import torch
+
+    import strings_workload as W
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+    from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
+
+    n_req = 8
+    specs = [W.with_nominal_durations(W._xfer(t, 100 + t)) for t in range(n_req)]
+    ins = [[torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory() for a in W.job_inputs(sp)] for sp in specs]
+    outs = [[torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in sp.d2h_sizes()] for sp in specs]
+    res = {"requests": n_req, "request": "XFER n=2^24 (64 MiB H2D + 64 MiB D2H)"}
+    for name, tenants_n in (("sequential_one_tenant", 1), ("coresident_strings_ps", n_req)):
+        S.init(num_gpus=1, physical_gpus=1, balancer=W.GMIN, device_policy=W.PS, timing_mode=S.MEASURED)
+        ts = [S.register_tenant(1, 1) for _ in range(tenants_n)]
+        spans = []
+        for rep in range(2 + args.steps):
+            t0 = time.perf_counter()
+            for i, sp in enumerate(specs):
+                S.submit(ts[i % tenants_n], S.make_desc(S.XFER, n=sp.n, seed=sp.seed), ins[i], outs[i])
+            assert S.drain() == S.OK
+            if rep >= 2:
+                spans.append(time.perf_counter() - t0)
+        S.shutdown()
+        res[name + "_ms"] = round(statistics.median(spans) * 1e3, 3)
+    wl = W.Workload("fig2", W.SystemConfig(num_gpus=1), [W.TenantSpec() for _ in range(n_req)],
+                    [W.JobSpec(**vars(sp)) for sp in specs])
+    st = run_static(wl, num_gpus=1, repeats=3)
+    res["separate_contexts_static_ms"] = round(st["span_s"] * 1e3, 3)
+    res["coresident_vs_sequential"] = round(res["sequential_one_tenant_ms"] / res["coresident_strings_ps_ms"], 3)
+    res["coresident_vs_separate_contexts"] = round(res["separate_contexts_static_ms"] / res["coresident_strings_ps_ms"], 3)
+    print(json.dumps(res))
+
+
 def main():
     args = parse_args()
+    if args.fig2:
+        fig2(args)
+        return
     if args.sweep:
         policy_sweep(args)
         return
