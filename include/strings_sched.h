@@ -64,6 +64,9 @@ typedef uint64_t strings_job_t;
 #define STRINGS_VSCALE 0        /* y = alpha * x, fp32, n elements          (memory-bound)      */
 #define STRINGS_GEMM   1        /* C = A.B, bf16 in / fp32 out, R repetitions (compute-bound)   */
 #define STRINGS_XFER   2        /* y = fmix32(x ^ seed), u32, n elements    (transfer-heavy)    */
+#define STRINGS_HIST   3        /* bins[256] u32 = byte histogram of x[n] u8 (Table I: HI)      */
+#define STRINGS_SCAN   4        /* y = inclusive prefix sum of x[n] u32, mod 2^32 (Table I: SC) */
+#define STRINGS_SORT   5        /* each 2048-key segment of x[n] u32 sorted ascending (SN)      */
 
 /* Timing modes. */
 #define STRINGS_TIMING_MEASURED        0  /* real clock, real completions                       */
@@ -101,9 +104,12 @@ typedef struct {
  *   VSCALE: h2d = { x[n] fp32 },                 d2h = { y[n] fp32 }
  *   GEMM:   h2d = { A[m*k] bf16, B[k*n] bf16 },  d2h = { C[m*n] fp32 }  (row-major)
  *           m % 128 == 0, n % 256 == 0, k % 64 == 0, k <= 256, reps >= 1
- *   XFER:   h2d = { x[n] u32 },                  d2h = { y[n] u32 }                           */
+ *   XFER:   h2d = { x[n] u32 },                  d2h = { y[n] u32 }
+ *   HIST:   h2d = { x[n] u8 },                   d2h = { bins[256] u32 }
+ *   SCAN:   h2d = { x[n] u32 },                  d2h = { y[n] u32 }
+ *   SORT:   h2d = { x[n] u32 }, n % 2048 == 0,   d2h = { y[n] u32 }                           */
 typedef struct {
-    uint32_t kclass;         /* STRINGS_VSCALE / STRINGS_GEMM / STRINGS_XFER                  */
+    uint32_t kclass;         /* STRINGS_VSCALE / GEMM / XFER / HIST / SCAN / SORT              */
     uint32_t reps;           /* GEMM repetitions R (R-17); ignored otherwise                  */
     uint64_t n, m, k;        /* sizes (see above)                                             */
     float    alpha;          /* VSCALE scalar                                                 */

@@ -58,6 +58,10 @@ def class_hbm_bytes_and_flop(spec: W.JobSpec) -> Tuple[int, int]:
     if spec.kclass == W.GEMM:
         m, n, k = spec.m, spec.n, spec.k
         return 2 * m * k + 2 * k * n + 4 * m * n, 2 * m * n * k * spec.reps
+    if spec.kclass == W.HIST:
+        return spec.n + 1024, 0                   # read bytes, write 256 u32 bins
+    if spec.kclass in (W.SCAN, W.SORT):
+        return 8 * spec.n, 0                      # read x, write y (u32)
     raise ValueError(spec.kclass)
 
 

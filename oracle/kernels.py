@@ -12,6 +12,13 @@ kernels"; the paper's workload classes, Table I):
   so R does not enter the result.
 * XFER   -- transfer-heavy:          y[i] = fmix32(x[i] ^ seed) in uint32, the
   MurmurHash3 finaliser (reading R-17).  Bit-exact.
+
+NEXT-2 classes shaped like the paper's Table I applications:
+* HIST   -- Histogram (HI):   bins[b] = #{i : x[i] == b}, 256 bins, uint32.
+* SCAN   -- Scan (SC):        y[i] = x[0] + ... + x[i]  mod 2^32 (inclusive).
+* SORT   -- Sorting Networks (SN): every consecutive 2048-key segment sorted
+  ascending (the SDK sample sorts a batch of fixed-length arrays).
+All three are bit-exact.
 """
 from __future__ import annotations
 
@@ -53,6 +60,23 @@ def xfer(x: np.ndarray, seed: int) -> np.ndarray:
     return fmix32(np.asarray(x, dtype=np.uint32) ^ np.uint32(seed & 0xFFFFFFFF))
 
 
+def hist(x: np.ndarray) -> np.ndarray:
+    """256-bin byte histogram (counts fit uint32 for n < 2^32)."""
+    return np.bincount(np.asarray(x, dtype=np.uint8), minlength=256).astype(np.uint32)
+
+
+def scan(x: np.ndarray) -> np.ndarray:
+    """Inclusive prefix sum modulo 2^32 (uint32 wrap-around)."""
+    return np.cumsum(np.asarray(x, dtype=np.uint32), dtype=np.uint32)
+
+
+def sort_segments(x: np.ndarray, seg: int = 2048) -> np.ndarray:
+    """Each consecutive segment of `seg` keys sorted ascending."""
+    x = np.asarray(x, dtype=np.uint32)
+    assert x.size % seg == 0
+    return np.sort(x.reshape(-1, seg), axis=1).reshape(-1)
+
+
 def run_job(spec, inputs):
     """Outputs (list of arrays) of one job given its H2D inputs."""
     import strings_workload as W
@@ -62,4 +86,10 @@ def run_job(spec, inputs):
         return [gemm(inputs[0].reshape(spec.m, spec.k), inputs[1].reshape(spec.k, spec.n))]
     if spec.kclass == W.XFER:
         return [xfer(inputs[0], spec.seed)]
+    if spec.kclass == W.HIST:
+        return [hist(inputs[0])]
+    if spec.kclass == W.SCAN:
+        return [scan(inputs[0])]
+    if spec.kclass == W.SORT:
+        return [sort_segments(inputs[0], W.SORT_SEGMENT)]
     raise ValueError(spec.kclass)

@@ -31,6 +31,15 @@ void class_bytes_flop(int kclass, uint64_t n, uint64_t m, uint64_t k, uint64_t r
       *hbm_bytes = 2 * m * k + 2 * k * n + 4 * m * n;
       *flop = 2 * m * n * k * reps;
       return;
+    case K_HIST:     // read x (u8), write 256 u32 bins
+      *hbm_bytes = n + 1024;
+      *flop = 0;
+      return;
+    case K_SCAN:     // read x, write y (u32)
+    case K_SORT:
+      *hbm_bytes = 8 * n;
+      *flop = 0;
+      return;
   }
   throw std::invalid_argument("kernel class");
 }
@@ -59,7 +68,7 @@ int Core::add_tenant(uint32_t weight, uint32_t max_inflight) {
   t.weight = weight;
   t.c = max_inflight;
   tenants_.push_back(t);
-  sft_.resize(tenants_.size() * 3);
+  sft_.resize(tenants_.size() * K_NCLASS);
   return static_cast<int>(tenants_.size()) - 1;
 }
 
@@ -147,10 +156,10 @@ bool Core::admission_before(const Job* a, const Job* b) const {
 }
 
 // ---------------------------------------------------------- predictions
-bool Core::has_sample(const Job* j) const { return sft_[j->tenant * 3 + j->kclass].count > 0; }
+bool Core::has_sample(const Job* j) const { return sft_[j->tenant * K_NCLASS + j->kclass].count > 0; }
 
 Core::Pred Core::pred(const Job* j) const {
-  const SftRow& r = sft_[j->tenant * 3 + j->kclass];
+  const SftRow& r = sft_[j->tenant * K_NCLASS + j->kclass];
   if (r.count > 0) return {r.h2d, r.kl, r.d2h, r.util};
   Pred p;
   p.h2d = cdiv(j->h2d_bytes, kPriorLinkBytesPerNs);
@@ -496,7 +505,7 @@ void Core::feedback(uint64_t t, Job* j) {
   for (int x = 0; x < 3; ++x) smp[x] = j->done[x] - j->start[x];
   uint64_t span = t - j->t_place;
   uint64_t util = span ? (smp[ENG_KL] * 65536) / span : 0;
-  SftRow& r = sft_[j->tenant * 3 + j->kclass];
+  SftRow& r = sft_[j->tenant * K_NCLASS + j->kclass];
   if (r.count == 0) {
     r.h2d = smp[0];
     r.kl = smp[1];

@@ -25,7 +25,7 @@
 namespace strings {
 
 enum Engine : int { ENG_H2D = 0, ENG_KL = 1, ENG_D2H = 2 };
-enum KClass : int { K_VSCALE = 0, K_GEMM = 1, K_XFER = 2 };
+enum KClass : int { K_VSCALE = 0, K_GEMM = 1, K_XFER = 2, K_HIST = 3, K_SCAN = 4, K_SORT = 5, K_NCLASS = 6 };
 enum Balancer : int { B_GRR = 0, B_GMIN, B_GWTMIN, B_RTF, B_GUF, B_DTF, B_MBF, B_DYNAMIC };
 enum DevPolicy : int { P_FIFO = 0, P_LAS = 1, P_PS = 2, P_TFS = 3 };
 
@@ -162,7 +162,7 @@ class Core {
   Hooks* hooks_;
   std::vector<Tenant> tenants_;
   std::vector<Device> devs_;
-  std::vector<SftRow> sft_;           // [tenant * 3 + class]
+  std::vector<SftRow> sft_;           // [tenant * K_NCLASS + class]
   struct ArrLess {
     bool operator()(const Job* a, const Job* b) const {
       if (a->arrival != b->arrival) return a->arrival < b->arrival;

@@ -44,6 +44,7 @@ struct __align__(128) PartState {
   uint64_t t_start;
   uint64_t t_exec;
   KlItem item;
+  GroupSync sync;                     // barrier + partials for group-wide bodies (SCAN, HIST)
 };
 
 struct DispatchParams {

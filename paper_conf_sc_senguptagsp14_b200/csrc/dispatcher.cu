@@ -117,7 +117,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     seen = g;
     const KlItem it = s_item;
     if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
-    run_item(it, rank, S, sm, tmem, mma_phase);
+    run_item(it, rank, S, sm, tmem, mma_phase, &ps->sync);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -142,6 +142,10 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   cta_teardown(tmem);
 }
 
+// Barrier/partials for stand-alone launches (one group-wide launch at a time
+// per device; the counter returns to zero after every barrier).
+__device__ GroupSync g_oneshot_sync;
+
 // Stand-alone launch of one tenant body on `gridDim.x` CTAs (kernel-level
 // checks outside the scheduler, and KL_MODE_LAUNCH).
 __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(KlItem it) {
@@ -150,7 +154,8 @@ __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(KlItem it) {
   uint32_t tmem = 0, mma_phase = 0;
   const bool gemm = it.kclass == 1;
   if (gemm) tmem = cta_setup(sm);
-  run_item(it, blockIdx.x, gridDim.x, sm, tmem, mma_phase);
+  GroupSync* gs = it.sync ? reinterpret_cast<GroupSync*>(it.sync) : &g_oneshot_sync;
+  run_item(it, blockIdx.x, gridDim.x, sm, tmem, mma_phase, gs);
   if (gemm) cta_teardown(tmem);
 }
 

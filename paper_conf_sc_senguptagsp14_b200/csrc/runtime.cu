@@ -125,6 +125,7 @@ struct Logical {
   int local = 0;                       // index among the logical devices of phys
   cudaStream_t h2d = nullptr, d2h = nullptr;
   std::vector<cudaStream_t> kl_streams;  // KL_MODE_LAUNCH only
+  uint8_t* kl_sync = nullptr;            // KL_MODE_LAUNCH: one GroupSync per KL stream (device)
   int next_kl_stream = 0;
   uint8_t* arena = nullptr;            // M slots of slot_bytes
   std::vector<int> free_slots;
@@ -465,6 +466,9 @@ class Runtime : public strings::Hooks {
           lg.kl_streams.resize(cfg.partitions);
           for (auto& s : lg.kl_streams)
             if (!cuda_ok(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+          const size_t gsb = sizeof(strings_dev::GroupSync) * cfg.partitions;
+          if (!cuda_ok(cudaMalloc(&lg.kl_sync, gsb))) return STRINGS_ENOMEM;
+          if (!cuda_ok(cudaMemset(lg.kl_sync, 0, gsb))) return STRINGS_ECUDA;
         }
         lg.arena = ph->arena + (size_t)lg.local * cfg.admit_cap * cfg.slot_bytes;
         for (int s = cfg.admit_cap - 1; s >= 0; --s) lg.free_slots.push_back(s);
@@ -515,6 +519,8 @@ class Runtime : public strings::Hooks {
         for (auto s : lg.kl_streams) cudaStreamSynchronize(s), cudaStreamDestroy(s);
         lg.h2d = lg.d2h = nullptr;
         lg.kl_streams.clear();
+        if (lg.kl_sync) cudaFree(lg.kl_sync);
+        lg.kl_sync = nullptr;
       }
       for (auto e : ph->ev_pool) cudaEventDestroy(e);
       ph->ev_pool.clear();
@@ -603,8 +609,10 @@ class Runtime : public strings::Hooks {
           std::atomic_thread_fence(std::memory_order_seq_cst);
         }
       } else {
-        cudaStream_t s = lg.kl_streams[lg.next_kl_stream];
+        const int si = lg.next_kl_stream;
+        cudaStream_t s = lg.kl_streams[si];
         lg.next_kl_stream = (lg.next_kl_stream + 1) % (int)lg.kl_streams.size();
+        it.sync = reinterpret_cast<uint64_t>(lg.kl_sync) + si * sizeof(strings_dev::GroupSync);
         int ctas = std::max(1, lg.ctas / cfg.partitions);
         ok = cuda_ok(strings::launch_oneshot(it, ctas, s));
         jc->ev[engine] = take_event(ph);
@@ -881,6 +889,19 @@ class Runtime : public strings::Hooks {
           return STRINGS_EINVAL;
         need_in = {2 * d->m * d->k, 2 * d->k * d->n};
         need_out = {4 * d->m * d->n};
+        break;
+      case STRINGS_HIST:
+        need_in = {d->n};
+        need_out = {1024};
+        break;
+      case STRINGS_SCAN:
+        need_in = {4 * d->n};
+        need_out = {4 * d->n};
+        break;
+      case STRINGS_SORT:
+        if (d->n % 2048) return STRINGS_EINVAL;
+        need_in = {4 * d->n};
+        need_out = {4 * d->n};
         break;
       default:
         return STRINGS_EINVAL;
@@ -1195,9 +1216,9 @@ strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kerne
     if (n_in < 2 || desc->m % 128 || desc->n % 256 || desc->k % 64 || desc->k > 256 || desc->k == 0 ||
         desc->reps == 0)
       return STRINGS_EINVAL;
-  } else if (desc->kclass != STRINGS_VSCALE && desc->kclass != STRINGS_XFER) {
+  } else if (desc->kclass > STRINGS_SORT) {
     return STRINGS_EINVAL;
-  } else if (n_in < 1) {
+  } else if (n_in < 1 || (desc->kclass == STRINGS_SORT && desc->n % 2048)) {
     return STRINGS_EINVAL;
   }
   if (!cuda_ok(cudaSetDevice(physical_gpu))) return STRINGS_ECUDA;
@@ -1208,6 +1229,11 @@ strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kerne
         !cuda_ok(cudaDeviceGetAttribute(&sm_count[physical_gpu], cudaDevAttrMultiProcessorCount, physical_gpu)))
       return STRINGS_ECUDA;
     ctas = sm_count[physical_gpu];
+  }
+  if ((desc->kclass == STRINGS_HIST || desc->kclass == STRINGS_SCAN)) {   // group barrier: all CTAs resident
+    int sms = 0;
+    if (!cuda_ok(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, physical_gpu))) return STRINGS_ECUDA;
+    if (ctas > sms) return STRINGS_EINVAL;
   }
   KlItem it;
   memset(&it, 0, sizeof it);

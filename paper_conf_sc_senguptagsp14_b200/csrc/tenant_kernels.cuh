@@ -27,7 +27,7 @@ struct __align__(16) KlItem {
   uint32_t seed;
   uint32_t pad;
   uint64_t t_issue;      // host CLOCK_REALTIME ns when the item was published (telemetry)
-  uint64_t pad2;
+  uint64_t sync;         // stand-alone launches: GroupSync* to use (0 = the default one)
 };
 static_assert(sizeof(KlItem) == 96, "KlItem layout");
 
@@ -366,10 +366,185 @@ __device__ inline void gemm_body(const uint16_t* __restrict__ A, const uint16_t*
   }
 }
 
+// ------------------------------------------------------- group coordination
+// A "group" is the S CTAs running one item (an SM partition of the dispatcher,
+// or a stand-alone grid).  All of them are co-resident (one CTA per SM), so a
+// counter/generation barrier in global memory is safe.
+struct __align__(128) GroupSync {
+  uint32_t bar_cnt;
+  uint32_t bar_gen;
+  uint32_t pad[30];
+  uint32_t partial[256];               // per-CTA partial results (S <= 256)
+};
+
+__device__ __forceinline__ void group_barrier(GroupSync* gs, int S) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t gen = *reinterpret_cast<volatile uint32_t*>(&gs->bar_gen);
+    if (atomicAdd(&gs->bar_cnt, 1u) == (uint32_t)S - 1) {
+      *reinterpret_cast<volatile uint32_t*>(&gs->bar_cnt) = 0;
+      __threadfence();
+      atomicAdd(&gs->bar_gen, 1u);
+    } else {
+      while (*reinterpret_cast<volatile uint32_t*>(&gs->bar_gen) == gen) __nanosleep(20);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// ---------------------------------------------------- HIST (Table I: HI)
+// bins[256] (u32) = byte histogram of x[n].  Per-warp shared-memory
+// sub-histograms (smem atomics), merged per CTA, then one global atomicAdd per
+// non-zero bin; rank 0 zeroes the output before the group barrier.
+__device__ inline void hist_body(const uint8_t* __restrict__ x, uint32_t* __restrict__ bins, uint64_t n,
+                                 int rank, int S, GroupSync* gs, uint8_t* stage) {
+  uint32_t* sh = reinterpret_cast<uint32_t*>(stage);            // [8 warps][256]
+  const int warp = threadIdx.x >> 5;
+  for (int i = threadIdx.x; i < 8 * 256; i += kThreads) sh[i] = 0;
+  if (rank == 0)
+    for (int i = threadIdx.x; i < 256; i += kThreads) bins[i] = 0;
+  __syncthreads();
+  uint32_t* mine = sh + warp * 256;
+  const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x, nt = (uint64_t)S * kThreads;
+  const bool aligned = (reinterpret_cast<uintptr_t>(x) & 15) == 0;
+  const uint64_t nv = aligned ? n / 16 : 0;
+  const uint4* x4 = reinterpret_cast<const uint4*>(x);
+  for (uint64_t v = tid; v < nv; v += nt) {
+    const uint4 q = ld_stream(x4 + v);
+    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+    for (int a = 0; a < 4; ++a)
+#pragma unroll
+      for (int b = 0; b < 4; ++b) atomicAdd(&mine[(w[a] >> (8 * b)) & 0xFF], 1u);
+  }
+  for (uint64_t e = nv * 16 + tid; e < n; e += nt) atomicAdd(&mine[x[e]], 1u);
+  __syncthreads();
+  uint32_t total = 0;                                              // thread t owns bin t
+  for (int w = 0; w < 8; ++w) total += sh[w * 256 + threadIdx.x];
+  group_barrier(gs, S);                                            // output zeroed by rank 0
+  if (total) atomicAdd(&bins[threadIdx.x], total);
+}
+
+// ---------------------------------------------------- SCAN (Table I: SC)
+// y = inclusive prefix sum of x (u32, mod 2^32) over the whole group:
+// per-CTA chunk sums -> group barrier -> chunk offset -> tiled block scan.
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t u = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += u;
+  }
+  return v;
+}
+
+__device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
+                                 int S, GroupSync* gs, uint8_t* stage) {
+  uint32_t* wsum = reinterpret_cast<uint32_t*>(stage);           // [8] warp totals + [1] broadcast
+  const uint64_t chunk = ((n + S - 1) / S + 7) & ~7ull;
+  const uint64_t b0 = min(n, (uint64_t)rank * chunk), b1 = min(n, b0 + chunk);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  // 1. chunk sum
+  uint32_t s = 0;
+  for (uint64_t e = b0 + threadIdx.x; e < b1; e += kThreads) s += x[e];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) wsum[warp] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < 8; ++w) t += wsum[w];
+    gs->partial[rank] = t;
+  }
+  group_barrier(gs, S);
+  // 2. offset of this chunk
+  if (threadIdx.x == 0) {
+    uint32_t off = 0;
+    for (int r = 0; r < rank; ++r) off += *reinterpret_cast<volatile uint32_t*>(&gs->partial[r]);
+    wsum[8] = off;
+  }
+  __syncthreads();
+  uint32_t carry = wsum[8];
+  __syncthreads();
+  // 3. tiles of 256 threads x 8 consecutive elements
+  for (uint64_t base = b0; base < b1; base += kThreads * 8) {
+    const uint64_t e0 = base + (uint64_t)threadIdx.x * 8;
+    uint32_t v[8];
+    uint32_t run = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      v[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
+      run += v[i];
+      v[i] = run;                                                   // thread-local inclusive
+    }
+    const uint32_t incl = warp_incl_scan(run);
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    uint32_t wpre = 0, tile = 0;
+    for (int w = 0; w < 8; ++w) {
+      const uint32_t t = wsum[w];
+      if (w < warp) wpre += t;
+      tile += t;
+    }
+    const uint32_t excl = carry + wpre + incl - run;               // sum before this thread's 8
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      if (e0 + i < b1) y[e0 + i] = excl + v[i];
+    carry += tile;
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------- SORT (Table I: SN, batch sort)
+// Each consecutive segment of 2048 u32 keys is sorted ascending by a bitonic
+// sorting network in shared memory (CUDA SDK "sortingNetworks" shape).
+constexpr int kSortSeg = 2048;
+__device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
+                                 int S, uint8_t* stage) {
+  uint32_t* key = reinterpret_cast<uint32_t*>(stage);
+  const uint64_t nseg = n / kSortSeg;
+  for (uint64_t seg = rank; seg < nseg; seg += S) {
+    const uint32_t* src = x + seg * kSortSeg;
+    for (int i = threadIdx.x; i < kSortSeg; i += kThreads) key[i] = src[i];
+    __syncthreads();
+    for (int k = 2; k <= kSortSeg; k <<= 1) {
+      for (int j = k >> 1; j > 0; j >>= 1) {
+        for (int i = threadIdx.x; i < kSortSeg / 2; i += kThreads) {
+          const int a = ((i / j) * 2 * j) + (i % j), b = a + j;
+          const bool up = (a & k) == 0;
+          const uint32_t ka = key[a], kb = key[b];
+          if ((ka > kb) == up) {
+            key[a] = kb;
+            key[b] = ka;
+          }
+        }
+        __syncthreads();
+      }
+    }
+    uint32_t* dst = y + seg * kSortSeg;
+    for (int i = threadIdx.x; i < kSortSeg; i += kThreads) dst[i] = key[i];
+    __syncthreads();
+  }
+}
+
 // Run one work item on this CTA (rank of S).
 __device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, const GemmSmem& sm,
-                                         uint32_t tmem_base, uint32_t& mma_phase) {
+                                         uint32_t tmem_base, uint32_t& mma_phase, GroupSync* gs) {
   switch (it.kclass) {
+    case 3:
+      hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
+                sm.stage);
+      break;
+    case 4:
+      scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
+                gs, sm.stage);
+      break;
+    case 5:
+      sort_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
+                sm.stage);
+      break;
     case 0:
       stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
                      it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);

@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(_HERE, "lib", "libstrings_sched.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "strings_sched.h")
 
 OK, EINVAL, ENOMEM, EAGAIN, ECUDA, ESTATE, EFAULT = 0, -1, -2, -3, -4, -5, -6
-VSCALE, GEMM, XFER = 0, 1, 2
+VSCALE, GEMM, XFER, HIST, SCAN, SORT = 0, 1, 2, 3, 4, 5
 MEASURED, INJECTED, DECISIONS_ONLY = 0, 1, 2
 
 

@@ -33,8 +33,9 @@ import numpy as np
 # ----------------------------------------------------------------------------
 # Enumerations (numeric values are part of the C ABI, include/strings_sched.h)
 # ----------------------------------------------------------------------------
-VSCALE, GEMM, XFER = 0, 1, 2
-CLASS_NAMES = {VSCALE: "VSCALE", GEMM: "GEMM", XFER: "XFER"}
+VSCALE, GEMM, XFER, HIST, SCAN, SORT = 0, 1, 2, 3, 4, 5
+CLASS_NAMES = {VSCALE: "VSCALE", GEMM: "GEMM", XFER: "XFER", HIST: "HIST", SCAN: "SCAN", SORT: "SORT"}
+SORT_SEGMENT = 2048
 
 GRR, GMIN, GWTMIN, RTF, GUF, DTF, MBF, DYNAMIC = range(8)
 BALANCER_NAMES = ["GRR", "GMIN", "GWTMIN", "RTF", "GUF", "DTF", "MBF", "DYNAMIC"]
@@ -108,16 +109,21 @@ class JobSpec:
     inj_d2h_ns: int = 0
 
     # Buffer sizes (bytes).  The H2D buffers of a job are, in order:
-    #   VSCALE: x[n] fp32;  GEMM: A[m*k] bf16, B[k*n] bf16;  XFER: x[n] u32
-    # and its D2H buffer is y[n] fp32 / C[m*n] fp32 / y[n] u32.
+    #   VSCALE: x[n] fp32;  GEMM: A[m*k] bf16, B[k*n] bf16;  XFER/SCAN/SORT: x[n] u32;
+    #   HIST: x[n] u8
+    # and its D2H buffer is y[n] fp32 / C[m*n] fp32 / y[n] u32 / bins[256] u32.
     def h2d_sizes(self) -> List[int]:
         if self.kclass == GEMM:
             return [2 * self.m * self.k, 2 * self.k * self.n]
+        if self.kclass == HIST:
+            return [self.n]
         return [4 * self.n]
 
     def d2h_sizes(self) -> List[int]:
         if self.kclass == GEMM:
             return [4 * self.m * self.n]
+        if self.kclass == HIST:
+            return [1024]
         return [4 * self.n]
 
 
@@ -169,12 +175,14 @@ class Workload:
 def nominal_durations(j: JobSpec) -> tuple:
     h2d = sum(j.h2d_sizes())
     d2h = sum(j.d2h_sizes())
+    kl_flop = 0
     if j.kclass == GEMM:
         kl_bytes = 2 * j.m * j.k + 2 * j.k * j.n + 4 * j.m * j.n
         kl_flop = 2 * j.m * j.n * j.k * j.reps
+    elif j.kclass == HIST:
+        kl_bytes = j.n + 1024
     else:
         kl_bytes = 8 * j.n
-        kl_flop = 0
     kl = max(_ceil_div(kl_bytes, INJ_HBM_BYTES_PER_NS), _ceil_div(kl_flop, INJ_KL_FLOP_PER_NS))
     return (_ceil_div(h2d, INJ_LINK_BYTES_PER_NS), kl, _ceil_div(d2h, INJ_LINK_BYTES_PER_NS))
 
@@ -199,8 +207,14 @@ def job_inputs(j: JobSpec) -> List[np.ndarray]:
     rng = np.random.Generator(np.random.PCG64(j.data_seed))
     if j.kclass == VSCALE:
         return [rng.uniform(-1.0, 1.0, size=j.n).astype(np.float32)]
-    if j.kclass == XFER:
+    if j.kclass in (XFER, SCAN, SORT):
         return [rng.integers(0, 1 << 32, size=j.n, dtype=np.uint64).astype(np.uint32)]
+    if j.kclass == HIST:
+        # image-like bytes: a skewed mixture (a few hot bins + uniform background)
+        hot = rng.integers(0, 256, size=8)
+        pick = rng.integers(0, 4, size=j.n)
+        vals = np.where(pick == 0, hot[rng.integers(0, 8, size=j.n)], rng.integers(0, 256, size=j.n))
+        return [vals.astype(np.uint8)]
     if j.kclass == GEMM:
         if j.int_valued:
             a = rng.integers(-2, 3, size=(j.m, j.k)).astype(np.float32)
@@ -217,6 +231,8 @@ def job_output_shapes(j: JobSpec) -> List[tuple]:
         return [((j.m, j.n), np.float32)]
     if j.kclass == VSCALE:
         return [((j.n,), np.float32)]
+    if j.kclass == HIST:
+        return [((256,), np.uint32)]
     return [((j.n,), np.uint32)]
 
 
@@ -370,7 +386,7 @@ def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs
     jobs = []
     for i in range(njobs):
         t = int(r.integers(0, T))
-        c = int(r.integers(0, 3))
+        c = int(r.integers(0, 6))
         ds = seed * 7919 + i
         if c == VSCALE:
             j = JobSpec(tenant=t, kclass=VSCALE, n=int(r.choice([0, 1, 5, 1024, 4099])) if tiny else VSCALE_N,
@@ -378,9 +394,15 @@ def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs
         elif c == GEMM:
             j = JobSpec(tenant=t, kclass=GEMM, m=128, n=256, k=int(r.choice([64, 128, 256])),
                         reps=int(r.integers(1, 5)), data_seed=ds, int_valued=bool(r.integers(0, 2)))
-        else:
+        elif c == XFER:
             j = JobSpec(tenant=t, kclass=XFER, n=int(r.choice([0, 3, 4096, 65537])) if tiny else XFER_N,
                         seed=int(r.integers(0, 1 << 32)), data_seed=ds)
+        elif c == HIST:
+            j = JobSpec(tenant=t, kclass=HIST, n=int(r.choice([0, 1, 17, 4096, 100_003])), data_seed=ds)
+        elif c == SCAN:
+            j = JobSpec(tenant=t, kclass=SCAN, n=int(r.choice([0, 1, 9, 2047, 70_001])), data_seed=ds)
+        else:
+            j = JobSpec(tenant=t, kclass=SORT, n=SORT_SEGMENT * int(r.choice([0, 1, 3, 40])), data_seed=ds)
         if r.integers(0, 2):
             arrivals[t] += int(r.choice([0, 0, 1, 500, 20_000, 2_000_000]))
         j.arrival_ns = arrivals[t]

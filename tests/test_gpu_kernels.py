@@ -103,3 +103,39 @@ def test_gemm_structured_operands_catch_layout_errors():
     ab, bb = W.f32_to_bf16_bits(a), W.f32_to_bf16_bits(b)
     (c,) = _launch(S.make_desc(S.GEMM, m=m, n=n, k=k, reps=1), [ab, bb], [np.zeros((m, n), np.float32)])
     assert np.array_equal(c, K.gemm(ab, bb))
+
+
+# ------------------------------------------------ NEXT-2: HIST / SCAN / SORT
+@pytest.mark.parametrize("n", [0, 1, 15, 16, 4097, 1_000_003, 1 << 24])
+@pytest.mark.parametrize("ctas", [0, 1, 37])
+def test_hist_bit_exact(n, ctas):
+    spec = W.JobSpec(tenant=0, kclass=W.HIST, n=n, data_seed=n + ctas)
+    (x,) = W.job_inputs(spec)
+    (h,) = _launch(S.make_desc(S.HIST, n=n), [x], [np.zeros(256, np.uint32)], ctas)
+    assert np.array_equal(h, K.hist(x))
+
+
+def test_hist_single_bin_contention():
+    x = np.full(1 << 20, 7, np.uint8)
+    (h,) = _launch(S.make_desc(S.HIST, n=x.size), [x], [np.zeros(256, np.uint32)])
+    assert h[7] == x.size and h.sum() == x.size
+
+
+@pytest.mark.parametrize("n", [0, 1, 7, 8, 2047, 2049, 100_003, (1 << 22) + 5])
+@pytest.mark.parametrize("ctas", [0, 1, 5, 148])
+def test_scan_bit_exact(n, ctas):
+    x = np.random.default_rng(n).integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    (y,) = _launch(S.make_desc(S.SCAN, n=n), [x], [np.zeros(n, np.uint32)], ctas)
+    assert np.array_equal(y, K.scan(x))
+
+
+@pytest.mark.parametrize("segs", [0, 1, 3, 150, 2048])
+@pytest.mark.parametrize("ctas", [0, 7])
+def test_sort_bit_exact(segs, ctas):
+    n = 2048 * segs
+    rng = np.random.default_rng(segs)
+    x = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    if n:
+        x[:2048] = rng.integers(0, 4, 2048)            # many duplicates in the first segment
+    (y,) = _launch(S.make_desc(S.SORT, n=n), [x], [np.zeros(n, np.uint32)], ctas)
+    assert np.array_equal(y, K.sort_segments(x))

@@ -65,7 +65,7 @@ def test_configs_injected_on_logical_devices(name, kw):
     check_outputs(wl, r)
 
 
-@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("seed", range(24))
 def test_random_workloads_injected(seed):
     wl = W.random_workload(seed, max_gpus=3)
     o = run_oracle(wl)

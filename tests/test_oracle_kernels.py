@@ -121,3 +121,39 @@ def test_run_job_shapes(cls):
     assert [a.nbytes for a in ins] == j.h2d_sizes()
     outs = K.run_job(j, ins)
     assert [a.nbytes for a in outs] == j.d2h_sizes()
+
+
+# ------------------------------------------------- NEXT-2 (Table I shapes)
+def test_hist_brute_force_and_total():
+    rng = np.random.default_rng(5)
+    x = rng.integers(0, 256, 3000).astype(np.uint8)
+    h = K.hist(x)
+    want = [0] * 256
+    for v in x.tolist():
+        want[v] += 1
+    assert h.tolist() == want and h.dtype == np.uint32 and int(h.sum()) == x.size
+    assert K.hist(np.zeros(0, np.uint8)).tolist() == [0] * 256
+
+
+def test_scan_definition_wraps_mod_2_32():
+    x = np.array([0xFFFFFFFF, 2, 3, 0x80000000, 0x80000000], dtype=np.uint32)
+    acc, want = 0, []
+    for v in x.tolist():
+        acc = (acc + v) % (1 << 32)
+        want.append(acc)
+    assert K.scan(x).tolist() == want
+    rng = np.random.default_rng(1)
+    y = rng.integers(0, 1 << 32, 10000, dtype=np.uint64).astype(np.uint32)
+    s = K.scan(y)
+    assert s[0] == y[0] and np.array_equal((s[1:] - s[:-1]).astype(np.uint32), y[1:])   # difference invariant
+
+
+def test_sort_segments_sorted_permutation():
+    rng = np.random.default_rng(2)
+    x = rng.integers(0, 1 << 32, 3 * 2048, dtype=np.uint64).astype(np.uint32)
+    y = K.sort_segments(x)
+    for sgm in range(3):
+        a, b = x[sgm * 2048:(sgm + 1) * 2048], y[sgm * 2048:(sgm + 1) * 2048]
+        assert np.all(b[1:] >= b[:-1])                        # ascending
+        assert sorted(a.tolist()) == b.tolist()               # a permutation of its own segment
+    assert K.sort_segments(np.array([3, 1, 2, 0], np.uint32), seg=4).tolist() == [0, 1, 2, 3]
