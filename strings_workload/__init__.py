@@ -355,6 +355,56 @@ def config_c5(seed: int = 1, reps: int = 64, scale: int = 1, jobs_per_tenant: in
 
 CONFIGS = {"C1": config_c1, "C2": config_c2, "C3": config_c3, "C4": config_c4, "C5": config_c5}
 
+# ----------------------------------------------------------------------------
+# NEXT-2: the paper's pairwise mix (6 long x 4 short apps -> 24
+# pairs A..X in Table I order).  Here: long = {GEMM (MM), HIST (HI), SCAN (SC)},
+# short = {VSCALE (BS-like streaming), XFER (MC-like transfer-heavy), SORT (SN)}
+# -> 9 pairs A..I.  Each pair runs `instances` tenants of each app, requests
+# arriving by Eq. (4) with lambda proportional to the app's runtime (L885-889).
+# ----------------------------------------------------------------------------
+PAIR_LONG = ("GEMM", "HIST", "SCAN")
+PAIR_SHORT = ("VSCALE", "XFER", "SORT")
+PAIRS = [(a, b) for a in PAIR_LONG for b in PAIR_SHORT]          # A..I
+
+
+def _pair_job(cls: str, t: int, ds: int, scale: int) -> JobSpec:
+    if cls == "GEMM":
+        return _gemm(t, ds, reps=256)
+    if cls == "HIST":
+        return JobSpec(tenant=t, kclass=HIST, n=(1 << 26) // scale, data_seed=ds)
+    if cls == "SCAN":
+        return JobSpec(tenant=t, kclass=SCAN, n=(1 << 24) // scale, data_seed=ds)
+    if cls == "VSCALE":
+        return _vscale(t, ds, n=VSCALE_N // scale)
+    if cls == "XFER":
+        return _xfer(t, ds, n=(1 << 22) // scale)
+    if cls == "SORT":
+        return JobSpec(tenant=t, kclass=SORT, n=max(SORT_SEGMENT, (1 << 20) // scale), data_seed=ds)
+    raise ValueError(cls)
+
+
+def config_pair(index: int, seed: int = 1, num_gpus: int = 2, balancer: int = GMIN, instances: int = 4,
+                jobs_per_tenant: int = 8, load: float = 0.8, scale: int = 1) -> Workload:
+    """Pair `index` (0 = 'A' ...) of the pairwise mix."""
+    a, b = PAIRS[index]
+    cfg = SystemConfig(num_gpus=num_gpus, balancer=balancer, device_policy=PS)
+    tenants = [TenantSpec() for _ in range(2 * instances)]
+    rng = SplitMix64(0xA11CE + 97 * index + seed)
+    jobs = []
+    for t in range(2 * instances):
+        cls = a if t % 2 == 0 else b
+        now = 0
+        for s in range(jobs_per_tenant):
+            j = with_nominal_durations(_pair_job(cls, t, seed * 1_000_003 + t * 1009 + s, scale))
+            t_solo = max(j.inj_h2d_ns, j.inj_kl_ns, j.inj_d2h_ns)
+            # per-tenant rate: the pair's 2*instances tenants share num_gpus devices at `load`
+            lam = t_solo * (2 * instances) / (num_gpus * load)
+            now += exp_interarrival_ns(rng, lam)
+            j.arrival_ns = now
+            jobs.append(j)
+    jobs.sort(key=lambda j: (j.arrival_ns, j.tenant))
+    return Workload(f"pair-{chr(65 + index)}:{a}-{b}", cfg, tenants, jobs)
+
 
 def random_workload(seed: int, max_gpus: int = 3, max_tenants: int = 6, max_jobs: int = 24,
                     tiny: bool = True) -> Workload:

@@ -194,3 +194,10 @@ def test_heterogeneous_gwtmin_parity_and_validation():
     with pytest.raises(S.StringsError) as e:
         S.init(num_gpus=2, timing_mode=S.DECISIONS_ONLY, device_weights=[1, 0])
     assert e.value.status == S.EINVAL
+
+
+@pytest.mark.parametrize("pair", range(9))
+def test_pairwise_mix_trace_matches_oracle(pair):
+    for bal in (W.GMIN, W.DTF, W.MBF):
+        wl = W.config_pair(pair, balancer=bal)
+        assert run_workload(wl, timing_mode=S.DECISIONS_ONLY).trace == run_oracle(wl).trace

@@ -118,6 +118,20 @@ def test_heterogeneous_logical_devices(timing):
     assert all(i.kl_partition // P == i.gid for i in r.infos)   # KL ran on its own device's SMs
 
 
+@pytest.mark.parametrize("pair", [1, 5, 7])
+def test_pairwise_mix_on_hardware(pair):
+    # NEXT-2 pairs (GEMM-XFER, HIST-SORT, SCAN-XFER), 2 logical devices, MBF placement:
+    # injected decisions identical to the oracle, measured-mode invariants, exact outputs
+    for timing in (S.INJECTED, S.MEASURED):
+        wl = W.config_pair(pair, balancer=W.MBF, instances=2, jobs_per_tenant=3, scale=16)
+        r = run_workload(wl, timing_mode=timing)
+        assert r.status == S.OK
+        if timing == S.INJECTED:
+            assert r.trace == run_oracle(wl).trace
+        assert invariants.check(r.trace, wl) == []
+        check_outputs(wl, r)
+
+
 def test_pageable_buffers_are_staged():
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)
