@@ -57,6 +57,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   __shared__ KlItem s_item;
   __shared__ uint32_t s_gen;
   GemmSmem sm = carve_smem(smem);
+  if ((smem_u32(smem) & 1023u) != 0) __trap();   // SWIZZLE_128B tiles need a 1 KB-aligned base
   const int NP = p.L * p.P;
   int q, start, S;
   partition_of(blockIdx.x, NP, p.part_start, &q, &start, &S);
@@ -117,7 +118,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     seen = g;
     const KlItem it = s_item;
     if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
-    run_item(it, rank, S, sm, tmem, mma_phase, &ps->sync);
+    run_item(it, &ps->item, true, rank, S, sm, tmem, mma_phase, &ps->sync);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -148,14 +149,14 @@ __device__ GroupSync g_oneshot_sync;
 
 // Stand-alone launch of one tenant body on `gridDim.x` CTAs (kernel-level
 // checks outside the scheduler, and KL_MODE_LAUNCH).
-__global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(KlItem it) {
+__global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_constant__ KlItem it) {
   extern __shared__ __align__(1024) uint8_t smem[];
   GemmSmem sm = carve_smem(smem);
   uint32_t tmem = 0, mma_phase = 0;
   const bool gemm = it.kclass == 1;
   if (gemm) tmem = cta_setup(sm);
   GroupSync* gs = it.sync ? reinterpret_cast<GroupSync*>(it.sync) : &g_oneshot_sync;
-  run_item(it, blockIdx.x, gridDim.x, sm, tmem, mma_phase, gs);
+  run_item(it, &it, false, blockIdx.x, gridDim.x, sm, tmem, mma_phase, gs);
   if (gemm) cta_teardown(tmem);
 }
 

@@ -75,9 +75,53 @@ uint64_t mono_ns() {
   return (uint64_t)ts.tv_sec * 1000000000ull + ts.tv_nsec;
 }
 
-// cuStreamWriteValue32 (driver API, fetched through the runtime: no libcuda link).
+// Driver API entry points, fetched through the runtime (no libcuda link).
 typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 WriteValue32Fn g_write_value32 = nullptr;
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn g_encode_tiled = nullptr;
+
+template <typename Fn>
+bool driver_entry(const char* name, Fn* out) {
+  if (*out) return true;
+  cudaDriverEntryPointQueryResult q;
+  void* fn = nullptr;
+  if (!cuda_ok(cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q)) || q != cudaDriverEntryPointSuccess ||
+      !fn)
+    return false;
+  *out = reinterpret_cast<Fn>(fn);
+  return true;
+}
+
+// TMA tensor maps of a GEMM job (A: M x K bf16 K-major, box 64 x 128; B: K x N
+// bf16 N-major, box 64 x 64; both SWIZZLE_128B) written into the work item.
+bool encode_gemm_maps(KlItem& it) {
+  if (!driver_entry("cuTensorMapEncodeTiled", &g_encode_tiled)) return false;
+  const cuuint32_t estr[2] = {1, 1};
+  {
+    const cuuint64_t dim[2] = {it.k, it.m};
+    const cuuint64_t stride[1] = {it.k * 2};
+    const cuuint32_t box[2] = {64, 128};
+    if (g_encode_tiled(reinterpret_cast<CUtensorMap*>(it.tmap_a), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                       reinterpret_cast<void*>(it.in0), dim, stride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                       CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return false;
+  }
+  {
+    const cuuint64_t dim[2] = {it.n, it.k};
+    const cuuint64_t stride[1] = {it.n * 2};
+    const cuuint32_t box[2] = {64, 64};
+    if (g_encode_tiled(reinterpret_cast<CUtensorMap*>(it.tmap_b), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                       reinterpret_cast<void*>(it.in1), dim, stride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                       CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return false;
+  }
+  return true;
+}
 
 // Host-mapped completion counters of one logical device's copy streams: after
 // every H2D / D2H op the stream itself writes the op's sequence number here
@@ -592,7 +636,10 @@ class Runtime : public strings::Hooks {
       it.reps = jc->desc.reps ? jc->desc.reps : 1;
       it.alpha = jc->desc.alpha;
       it.seed = jc->desc.seed;
-      if (kl_mode == 0) {
+      if (it.kclass == STRINGS_GEMM && !encode_gemm_maps(it)) ok = false;
+      if (!ok) {
+        // leave the op failed (fault localised to this job)
+      } else if (kl_mode == 0) {
         if (lg.tail - lg.completed >= (uint32_t)kRing) {
           ok = false;  // cannot happen with A <= kRing; treat as a job fault
         } else {
@@ -1247,6 +1294,7 @@ strings_status_t strings_kernel_launch(int32_t physical_gpu, const strings_kerne
   it.reps = desc->reps ? desc->reps : 1;
   it.alpha = desc->alpha;
   it.seed = desc->seed;
+  if (it.kclass == STRINGS_GEMM && !encode_gemm_maps(it)) return STRINGS_ECUDA;
   return cuda_ok(strings::launch_oneshot(it, ctas, static_cast<cudaStream_t>(stream))) ? STRINGS_OK
                                                                                       : STRINGS_ECUDA;
 }

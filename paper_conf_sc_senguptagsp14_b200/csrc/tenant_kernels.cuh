@@ -8,6 +8,7 @@
 //   XFER    y = fmix32(x ^ seed)     u32 (MurmurHash3 finaliser)
 //   GEMM    C = A . B, R repetitions bf16 -> fp32, tcgen05 + TMEM (R-17, R-22)
 #pragma once
+#include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -16,7 +17,8 @@ namespace strings_dev {
 constexpr int kThreads = 256;
 
 // One KL work item (also the layout of the host-mapped KL ring entries).
-struct __align__(16) KlItem {
+// GEMM items carry the TMA tensor maps of A and B (encoded on the host per job).
+struct __align__(64) KlItem {
   uint32_t seq;          // claim number (1-based, monotone per ring); written last by the host
   uint32_t kclass;
   uint64_t job;
@@ -28,8 +30,12 @@ struct __align__(16) KlItem {
   uint32_t pad;
   uint64_t t_issue;      // host CLOCK_REALTIME ns when the item was published (telemetry)
   uint64_t sync;         // stand-alone launches: GroupSync* to use (0 = the default one)
+  uint64_t pad3[4];
+  uint8_t tmap_a[128];   // CUtensorMap of A (bf16 M x K, K-major, box 64 x 128, SWIZZLE_128B)
+  uint8_t tmap_b[128];   // CUtensorMap of B (bf16 K x N, N-major, box 64 x 64,  SWIZZLE_128B)
 };
-static_assert(sizeof(KlItem) == 96, "KlItem layout");
+static_assert(sizeof(KlItem) == 384, "KlItem layout");
+static_assert(offsetof(KlItem, tmap_a) % 64 == 0, "tensor maps must be 64-B aligned");
 
 // ---------------------------------------------------------- smem / mbarrier
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -195,30 +201,36 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
 }
 
 // --------------------------------------------------------------------- GEMM
-// Tile 128 x 256 (M x N) per CTA, whole K (<= 256) resident in shared memory
-// in UMMA canonical SWIZZLE_NONE layouts built from 128-B "core matrices"
-// (8 rows of 16 B):
-//   A (K-major, A is M x K row-major): core (row-group g in 0..15, k-chunk c)
-//     holds rows 8g..8g+7, k 8c..8c+7; stored at (c*16 + g)*128  -> SBO = 128, LBO = 2048
-//   B (MN-major, B is K x N row-major): core (n-group q in 0..31, k-chunk c)
-//     holds k 8c..8c+7 (one per 16-B row), n 8q..8q+7; at (c*32 + q)*128
-//                                                              -> SBO = 128, LBO = 4096
-// Both are filled with plain 16-B copies (no transposition); 8 consecutive
-// threads write one 128-B core matrix, so the stores are bank-conflict free.
+// Tile 128 x 256 (M x N) per CTA, whole K (<= 256) resident in shared memory in
+// the UMMA canonical SWIZZLE_128B layouts that TMA tensor loads produce:
+//   A (K-major, M x K row-major): 4 K-slabs of 64 elements; slab c = 128 rows x
+//     128 B (16 KB) at c*16 KB, 16-B chunks XOR-swizzled by row%8 inside each
+//     1 KB atom of 8 rows.  UMMA desc: SBO = 1024 (8-row atom), LBO unused (16);
+//     a K=16 step inside a slab advances the start address by 32 B.
+//   B (MN-major, K x N row-major): 4 N-slabs of 64 elements; slab j = 256 k-rows x
+//     128 B (32 KB) at 64 KB + j*32 KB.  UMMA desc: LBO = 32 KB (next N-slab),
+//     SBO = 1024 (8 k-rows); a K=16 step advances the start by 16 rows = 2 KB.
+// The fill is split into four K-chunks (A slab c + the 64 k-rows c of every B
+// slab, 48 KB), each completing its own mbarrier, so the first repetition's MMAs
+// start as soon as their chunk has landed.
 constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
 constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
 constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
 constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 64;     // + mbarriers / tmem slot (tail, see carve_smem)
 constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
+constexpr uint32_t kSlabA = 128 * 128;                   // 16 KB
+constexpr uint32_t kSlabB = 256 * 128;                   // 32 KB
+constexpr uint32_t kChunkB = 64 * 128;                   // 64 k-rows of one B slab: 8 KB
 
 // Shared-memory matrix descriptor (sm_100 UMMA): start>>4 [0,14), LBO>>4 [16,30),
-// SBO>>4 [32,46), version=1 [46,48), base offset 0, layout SWIZZLE_NONE (0) [61,64).
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+// SBO>>4 [32,46), version=1 [46,48), base offset 0, layout [61,64) (2 = SWIZZLE_128B).
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
   uint64_t d = 0;
   d |= (uint64_t)((saddr >> 4) & 0x3FFF);
   d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
   d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
   d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
   return d;
 }
 
@@ -271,71 +283,70 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+// TMA 2D tile load (tensor map in global or param space) completing on `bar`.
+__device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int c0, int c1, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+      :: "r"(smem_u32(dst)), "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(bar)) : "memory");
+}
+
 struct GemmSmem {
-  uint8_t* a;          // kSmemA bytes, 128-B aligned
+  uint8_t* a;          // kSmemA bytes, 1024-B aligned
   uint8_t* b;          // kSmemB bytes
   uint64_t* bar;       // MMA-completion mbarrier
   uint32_t* tmem_slot; // TMEM base written by tcgen05.alloc
   uint8_t* stage;      // streaming stages (aliases a/b: a CTA runs one item at a time)
-  uint64_t* sbar;      // streaming stage mbarriers [kStreamStages]
+  uint64_t* sbar;      // streaming stage mbarriers / GEMM fill mbarriers [4]
 };
-
-// Load the A tile (rows m0..m0+127, all K) and the B tile (all K, cols
-// n0..n0+255) into the canonical layouts above.  All 256 threads participate;
-// thread t writes row (t & 7) of a core matrix.
-__device__ inline void gemm_load_tile(const GemmSmem& sm, const uint16_t* __restrict__ A,
-                                      const uint16_t* __restrict__ B, uint64_t N, uint64_t K,
-                                      uint64_t m0, uint64_t n0) {
-  const int kchunks = (int)(K / 8);
-  // cp.async (LDGSTS) 16-B global->smem copies: no register round trip, every
-  // chunk of the thread in flight at once (the fill is latency-bound otherwise)
-  auto cp16 = [](uint8_t* dst, const void* src) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(smem_u32(dst)), "l"(src) : "memory");
-  };
-  // A: 16 x kchunks cores; idx -> (rr = row in core, c = k-chunk, g = row group)
-  for (int idx = threadIdx.x; idx < kTileM * kchunks; idx += kThreads) {
-    const int rr = idx & 7, c = (idx >> 3) % kchunks, g = (idx >> 3) / kchunks;
-    const int r = g * 8 + rr;
-    cp16(sm.a + ((c * 16 + g) * 128 + rr * 16), A + (m0 + r) * K + (uint64_t)c * 8);
-  }
-  // B: 32 x kchunks cores; idx -> (kk = k in core, q = n-group, c = k-chunk)
-  for (int idx = threadIdx.x; idx < (int)K * (kTileN / 8); idx += kThreads) {
-    const int kk = idx & 7, q = (idx >> 3) & 31, c = idx >> 8;
-    const int k = c * 8 + kk;
-    cp16(sm.b + ((c * 32 + q) * 128 + kk * 16), B + (uint64_t)k * N + n0 + (uint64_t)q * 8);
-  }
-  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-  // make generic-proxy smem writes visible to the tensor core (async proxy)
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  __syncthreads();
-}
 
 // Units u = tile * R + rep, tile = (mt, nt); this CTA takes the contiguous
 // chunk [rank*U/S, (rank+1)*U/S).  Each repetition is a full 16-MMA chain into
-// the TMEM accumulator; C is written from repetition R-1 (R-17).
-__device__ inline void gemm_body(const uint16_t* __restrict__ A, const uint16_t* __restrict__ B,
-                          float* __restrict__ C, uint64_t M, uint64_t N, uint64_t K, uint32_t R,
-                          int rank, int S, const GemmSmem& sm, uint32_t tmem_base,
-                          uint32_t& mma_phase) {
+// the TMEM accumulator; C is written from repetition R-1 (R-17).  tmap_a/tmap_b
+// point to the job's tensor maps (global memory: tmap_global = true, each
+// consumer fences the tensormap proxy; kernel-parameter space otherwise).
+__device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, bool tmap_global,
+                                 float* __restrict__ C, uint64_t M, uint64_t N, uint64_t K, uint32_t R,
+                                 int rank, int S, const GemmSmem& sm, uint32_t tmem_base, uint32_t& mma_phase) {
   const uint64_t tiles_n = N / kTileN, tiles = (M / kTileM) * tiles_n;
   const uint64_t U = tiles * R;
   const uint64_t u0 = (U * rank) / S, u1 = (U * (rank + 1)) / S;
   const uint32_t idesc = umma_idesc_bf16(kTileM, kTileN);
   const uint32_t a_base = smem_u32(sm.a), b_base = smem_u32(sm.b);
+  const int kchunks = (int)(K / 64);
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (threadIdx.x == 0 && tmap_global && u0 < u1) {
+    asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_a) : "memory");
+    asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_b) : "memory");
+  }
   uint64_t u = u0;
   while (u < u1) {
     const uint64_t tile = u / R;
     const uint64_t last = min(u1, (tile + 1) * R);        // exclusive end of this tile's run
     const uint64_t mt = tile / tiles_n, nt = tile % tiles_n;
-    gemm_load_tile(sm, A, B, N, K, mt * kTileM, nt * kTileN);
     if (threadIdx.x == 0) {
-      tc_fence_after();
+      for (int c = 0; c < kchunks; ++c) mbar_init(&sm.sbar[c], 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      for (int c = 0; c < kchunks; ++c) {
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+                     :: "r"(smem_u32(&sm.sbar[c])), "r"(kSlabA + 4 * kChunkB) : "memory");
+        tma_load_2d(sm.a + c * kSlabA, tmap_a, 64 * c, (int)(mt * kTileM), &sm.sbar[c]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          tma_load_2d(sm.b + j * kSlabB + c * kChunkB, tmap_b, (int)(nt * kTileN) + 64 * j, 64 * c, &sm.sbar[c]);
+      }
       for (uint64_t v = u; v < last; ++v) {
-        for (uint32_t ks = 0; ks < K / 16; ++ks) {
-          uint64_t da = umma_desc(a_base + ks * 2 * 2048, 2048, 128);
-          uint64_t db = umma_desc(b_base + ks * 2 * 4096, 4096, 128);
-          umma_bf16(tmem_base, da, db, idesc, ks > 0 ? 1u : 0u);
+        for (int c = 0; c < kchunks; ++c) {
+          if (v == u) {
+            mbar_wait(&sm.sbar[c], 0);
+            tc_fence_after();
+          }
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const int ks = 4 * c + kk;
+            const uint64_t da = umma_desc_sw128(a_base + c * kSlabA + kk * 32, 16, 1024);
+            const uint64_t db = umma_desc_sw128(b_base + ks * 2048, kSlabB, 1024);
+            umma_bf16(tmem_base, da, db, idesc, ks > 0 ? 1u : 0u);
+          }
         }
       }
       umma_commit(sm.bar);            // arrives when every MMA above has completed
@@ -530,8 +541,10 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
 }
 
 // Run one work item on this CTA (rank of S).
-__device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, const GemmSmem& sm,
-                                         uint32_t tmem_base, uint32_t& mma_phase, GroupSync* gs) {
+// `tmaps` is the item as it sits in global memory (dispatcher mailbox,
+// tmap_global = true) or in kernel-parameter space (stand-alone launches).
+__device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, bool tmap_global, int rank, int S,
+                                         const GemmSmem& sm, uint32_t tmem_base, uint32_t& mma_phase, GroupSync* gs) {
   switch (it.kclass) {
     case 3:
       hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
@@ -554,9 +567,8 @@ __device__ __forceinline__ void run_item(const KlItem& it, int rank, int S, cons
                      it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
       break;
     case 1:
-      gemm_body(reinterpret_cast<const uint16_t*>(it.in0), reinterpret_cast<const uint16_t*>(it.in1),
-                reinterpret_cast<float*>(it.out0), it.m, it.n, it.k, it.reps, rank, S, sm, tmem_base,
-                mma_phase);
+      gemm_body(tmaps->tmap_a, tmaps->tmap_b, tmap_global, reinterpret_cast<float*>(it.out0), it.m, it.n, it.k,
+                it.reps, rank, S, sm, tmem_base, mma_phase);
       break;
   }
 }
