@@ -96,7 +96,8 @@ bool driver_entry(const char* name, Fn* out) {
 }
 
 // TMA tensor maps of a GEMM job (A: M x K bf16 K-major, box 64 x 128; B: K x N
-// bf16 N-major, box 64 x 64; both SWIZZLE_128B) written into the work item.
+// bf16 N-major, box 64 x 64; C: M x N fp32, box 32 x 128; all SWIZZLE_128B)
+// written into the work item.
 bool encode_gemm_maps(KlItem& it) {
   if (!driver_entry("cuTensorMapEncodeTiled", &g_encode_tiled)) return false;
   const cuuint32_t estr[2] = {1, 1};
@@ -116,6 +117,16 @@ bool encode_gemm_maps(KlItem& it) {
     const cuuint32_t box[2] = {64, 64};
     if (g_encode_tiled(reinterpret_cast<CUtensorMap*>(it.tmap_b), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
                        reinterpret_cast<void*>(it.in1), dim, stride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                       CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return false;
+  }
+  {
+    const cuuint64_t dim[2] = {it.n, it.m};
+    const cuuint64_t stride[1] = {it.n * 4};
+    const cuuint32_t box[2] = {32, 128};
+    if (g_encode_tiled(reinterpret_cast<CUtensorMap*>(it.tmap_c), CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                       reinterpret_cast<void*>(it.out0), dim, stride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                        CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return false;

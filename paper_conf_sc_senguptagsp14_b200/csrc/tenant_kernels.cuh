@@ -33,8 +33,9 @@ struct __align__(64) KlItem {
   uint64_t pad3[4];
   uint8_t tmap_a[128];   // CUtensorMap of A (bf16 M x K, K-major, box 64 x 128, SWIZZLE_128B)
   uint8_t tmap_b[128];   // CUtensorMap of B (bf16 K x N, N-major, box 64 x 64,  SWIZZLE_128B)
+  uint8_t tmap_c[128];   // CUtensorMap of C (fp32 M x N, N-major, box 32 x 128, SWIZZLE_128B)
 };
-static_assert(sizeof(KlItem) == 384, "KlItem layout");
+static_assert(sizeof(KlItem) == 512, "KlItem layout");
 static_assert(offsetof(KlItem, tmap_a) % 64 == 0, "tensor maps must be 64-B aligned");
 
 // ---------------------------------------------------------- smem / mbarrier
@@ -283,6 +284,12 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+// TMA 2D tile store from shared memory (bulk async-group completion).
+__device__ __forceinline__ void tma_store_2d(const void* tmap, const void* src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+               :: "l"(tmap), "r"(smem_u32(src)), "r"(c0), "r"(c1) : "memory");
+}
+
 // TMA 2D tile load (tensor map in global or param space) completing on `bar`.
 __device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int c0, int c1, uint64_t* bar) {
   asm volatile(
@@ -304,7 +311,7 @@ struct GemmSmem {
 // the TMEM accumulator; C is written from repetition R-1 (R-17).  tmap_a/tmap_b
 // point to the job's tensor maps (global memory: tmap_global = true, each
 // consumer fences the tensormap proxy; kernel-parameter space otherwise).
-__device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, bool tmap_global,
+__device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, const void* tmap_c, bool tmap_global,
                                  float* __restrict__ C, uint64_t M, uint64_t N, uint64_t K, uint32_t R,
                                  int rank, int S, const GemmSmem& sm, uint32_t tmem_base, uint32_t& mma_phase) {
   const uint64_t tiles_n = N / kTileN, tiles = (M / kTileM) * tiles_n;
@@ -317,6 +324,7 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, bool tm
   if (threadIdx.x == 0 && tmap_global && u0 < u1) {
     asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_a) : "memory");
     asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_b) : "memory");
+    asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_c) : "memory");
   }
   uint64_t u = u0;
   while (u < u1) {
@@ -356,19 +364,34 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, bool tm
     mma_phase ^= 1;
     tc_fence_after();
     if ((last - 1) % R == R - 1) {    // this run contains the final repetition: epilogue
+      // TMEM -> registers -> smem staging in the TMA SWIZZLE_128B layout of a
+      // 32-column x 128-row fp32 box (row r at r*128 B, 16-B chunk q at q ^ (r%8):
+      // the 8 lanes of a store phase hit 8 different chunks, no bank conflicts)
+      // -> eight TMA tensor stores of the 128 x 256 tile.  A/B smem is free: every
+      // MMA has completed (sm.bar).
       const int lane_base = (warp & 3) * 32;
       const int col0 = (warp >> 2) * 128;
-      const uint64_t row = mt * kTileM + lane_base + lane;
-      float* crow = C + row * N + nt * kTileN;
+      const int r = lane_base + lane;
 #pragma unroll 1
       for (int cc = 0; cc < 128; cc += 32) {
-        uint32_t r[32];
-        tmem_ld32(tmem_base + ((uint32_t)lane_base << 16) + (uint32_t)(col0 + cc), r);
-        float4* dst = reinterpret_cast<float4*>(crow + col0 + cc);
+        uint32_t v[32];
+        tmem_ld32(tmem_base + ((uint32_t)lane_base << 16) + (uint32_t)(col0 + cc), v);
+        uint8_t* box = sm.a + ((col0 + cc) / 32) * (128 * 128);
 #pragma unroll
-        for (int q = 0; q < 8; ++q)
-          dst[q] = make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]),
-                               __uint_as_float(r[4 * q + 2]), __uint_as_float(r[4 * q + 3]));
+        for (int q = 0; q < 8; ++q) {
+          uint4 w = make_uint4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+          *reinterpret_cast<uint4*>(box + r * 128 + ((q ^ (r & 7)) << 4)) = w;
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // smem writes -> async proxy
+      __syncthreads();
+      if (threadIdx.x == 0) {
+#pragma unroll
+        for (int g = 0; g < 8; ++g)
+          tma_store_2d(tmap_c, sm.a + g * (128 * 128), (int)(nt * kTileN) + 32 * g, (int)(mt * kTileM));
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");    // C written before the item ends
+        asm volatile("fence.proxy.async.global;" ::: "memory");
       }
     }
     tc_fence_before();
@@ -567,8 +590,8 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
                      it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
       break;
     case 1:
-      gemm_body(tmaps->tmap_a, tmaps->tmap_b, tmap_global, reinterpret_cast<float*>(it.out0), it.m, it.n, it.k,
-                it.reps, rank, S, sm, tmem_base, mma_phase);
+      gemm_body(tmaps->tmap_a, tmaps->tmap_b, tmaps->tmap_c, tmap_global, reinterpret_cast<float*>(it.out0), it.m,
+                it.n, it.k, it.reps, rank, S, sm, tmem_base, mma_phase);
       break;
   }
 }
