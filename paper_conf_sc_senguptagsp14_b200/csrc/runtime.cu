@@ -5,10 +5,13 @@
 //   API calls (any thread) --> inbox under mu_ --> engine thread
 //   engine thread: drives strings::Core (core.cpp) in one of three timing
 //   modes and implements its Hooks by issuing physical ops at WAKE:
-//     H2D  cudaMemcpyAsync on the logical device's H2D stream + event
+//     H2D  cudaMemcpyAsync on the logical device's H2D stream, then a stream
+//          memory op writes the op's sequence number to a host-mapped counter
 //     KL   KlItem into the logical device's ring (host-mapped), the persistent
-//          dispatcher kernel claims it (dispatcher.cu)
-//     D2H  cudaMemcpyAsync on the D2H stream + event
+//          dispatcher kernel claims it (dispatcher.cu) and writes a completion word
+//     D2H  cudaMemcpyAsync on the D2H stream + counter write
+//   A watchdog polls the dispatcher stream: a sticky CUDA error (device fault)
+//   poisons that GPU's tenants (STRINGS_ECUDA at sync) instead of hanging.
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <time.h>
@@ -816,6 +819,30 @@ class Runtime : public strings::Hooks {
     return true;
   }
 
+  // Watchdog (rate-limited): the persistent dispatcher must still be running.
+  // A device fault ends it with a sticky error; every tenant of the process
+  // then fails (merged context: P:L183 shortcoming 1) rather than hang.
+  uint64_t last_health = 0;
+  bool healthy() {
+    if (fatal != STRINGS_OK) return false;
+    if (!has_gpu() || kl_mode != 0) return true;
+    const uint64_t t = mono_ns();
+    if (t - last_health < 10000000ull) return true;
+    last_health = t;
+    for (auto& ph : phys) {
+      if (!ph->kernel_running) continue;
+      set_dev(ph->dev);
+      const cudaError_t e = cudaStreamQuery(ph->kstream);
+      if (e == cudaErrorNotReady) continue;
+      cuda_ok(e == cudaSuccess ? cudaErrorLaunchFailure : e);
+      ph->kernel_running = false;
+      fatal = STRINGS_ECUDA;
+      cv_done.notify_all();
+      return false;
+    }
+    return true;
+  }
+
   // ------------------------------------------------------------- engine
   void take_inbox(std::vector<JobCtx*>& out) {
     out.swap(inbox);
@@ -870,6 +897,10 @@ class Runtime : public strings::Hooks {
       for (auto& c : batch) {
         JobCtx* jc = jobs[c.job].get();
         while (!phys_complete(jc, c.engine)) {
+          if (!healthy()) {
+            stop = true;
+            return;
+          }
           lk.unlock();
           std::this_thread::yield();
           lk.lock();
@@ -923,6 +954,10 @@ class Runtime : public strings::Hooks {
       progressed = false;
     }
     if (!progressed) {
+      if (!healthy()) {
+        stop = true;
+        return;
+      }
       lk.unlock();
       std::this_thread::yield();
       lk.lock();
