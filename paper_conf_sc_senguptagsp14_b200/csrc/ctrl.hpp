@@ -56,6 +56,7 @@ struct DispatchParams {
   const int* part_start;              // [L * P + 1] first CTA of each partition (device memory)
   int L, P;                           // logical devices hosted, partitions per logical device
   uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
+  uint64_t fault_job;                 // fault injection (STRINGS_FAULT_JOB): trap on this job id
 };
 
 inline size_t host_ctrl_bytes(int L) {

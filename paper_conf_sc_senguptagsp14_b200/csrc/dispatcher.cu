@@ -117,6 +117,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     if (g == kStop) break;
     seen = g;
     const KlItem it = s_item;
+    if (it.job == p.fault_job) __trap();          // fault injection (tests the watchdog)
     if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
     run_item(it, &ps->item, true, rank, S, sm, tmem, mma_phase, &ps->sync);
     __syncthreads();

@@ -553,6 +553,8 @@ class Runtime : public strings::Hooks {
         dp.P = cfg.partitions;
         const char* fl = getenv("STRINGS_DISPATCH_FLAGS");
         dp.flags = fl ? (uint32_t)strtoul(fl, nullptr, 0) : 0u;
+        const char* fj = getenv("STRINGS_FAULT_JOB");
+        dp.fault_job = fj ? (uint64_t)strtoull(fj, nullptr, 0) : ~0ull;
         if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
       }
@@ -969,6 +971,10 @@ class Runtime : public strings::Hooks {
                           int32_t n_h2d, const strings_buf_t* d2h, int32_t n_d2h, uint32_t prio,
                           strings_job_t* out) {
     if (!d) return STRINGS_EINVAL;
+    {
+      std::lock_guard<std::mutex> g(mu);
+      if (fatal != STRINGS_OK) return fatal;       // device fault: the GPU's tenants are poisoned
+    }
     std::vector<uint64_t> need_in, need_out;
     switch (d->kclass) {
       case STRINGS_VSCALE:

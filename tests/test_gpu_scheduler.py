@@ -157,3 +157,46 @@ def test_full_size_c2_measured_sampled_parity():
         else:
             idx = np.concatenate([np.arange(64), spec.n - 1 - np.arange(64), rng.integers(0, spec.n, 65536)])
             assert np.array_equal(r.outputs[i][0][idx], K.xfer(ins[0][idx], spec.seed))
+
+
+_FAULT_SCRIPT = r"""
+import os, sys, time
+sys.path.insert(0, os.getcwd())
+import strings_workload as W
+from paper_conf_sc_senguptagsp14_b200 import strings as S
+wl = W.config_c1(reps=2)
+S.init_from_config(wl.config.resolved(), timing_mode=S.MEASURED, physical_gpus=1)
+ts = [S.register_tenant() for _ in wl.tenants]
+import numpy as np
+bufs = []
+for spec in wl.jobs:
+    ins = W.job_inputs(spec)
+    outs = [np.zeros(shape, dt) for shape, dt in W.job_output_shapes(spec)]
+    bufs.append((ins, outs))
+    try:
+        S.submit_spec(ts[spec.tenant], spec, ins, outs)
+    except S.StringsError as e:          # the fault may already have been detected
+        assert e.status == S.ECUDA
+t0 = time.time()
+st = S.drain()
+print("STATUS", st, "CUDAERR", S.last_cuda_error(), "SECONDS", round(time.time() - t0, 2), flush=True)
+S.shutdown()
+"""
+
+
+def test_device_fault_fails_tenants_instead_of_hanging(tmp_path):
+    # fault injection: the dispatcher traps while running job 3; the watchdog must
+    # turn the sticky error into STRINGS_ECUDA for the waiting tenants (no hang)
+    import os
+    import subprocess
+    import sys
+    script = tmp_path / "fault.py"
+    script.write_text(_FAULT_SCRIPT)
+    env = dict(os.environ, STRINGS_FAULT_JOB="3")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    p = subprocess.run([sys.executable, str(script)], cwd=root, env=env, capture_output=True, text=True,
+                       timeout=180)
+    line = [l for l in p.stdout.splitlines() if l.startswith("STATUS")]
+    assert line, p.stdout + p.stderr
+    f = line[0].split()
+    assert int(f[1]) == S.ECUDA and int(f[3]) != 0 and float(f[5]) < 30
