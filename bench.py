@@ -256,7 +256,7 @@ def run_strings(args, rank, world, torch, gloo):
         ins.append(pins)
         outs.append([torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
     S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1, kl_mode=args.kl_mode,
-                       trace_in_memory=True)
+                       trace_in_memory=bool(args.trace_out))
     # the persistent dispatcher now owns every SM: no torch kernels, no device-wide sync until shutdown
     tenants = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
     stream = torch.cuda.Stream()
@@ -270,7 +270,7 @@ def run_strings(args, rank, world, torch, gloo):
 
     for _ in range(args.warmup):
         one_step()
-    trace_start = len(S.trace())
+    trace_start = len(S.trace()) if args.trace_out else 0
     gloo_barrier(gloo)
     stream.synchronize()
     with ClockSampler(int(os.environ.get("LOCAL_RANK", 0)) if world > 1 else 0) as clk:
@@ -283,7 +283,7 @@ def run_strings(args, rank, world, torch, gloo):
         t_wall = time.perf_counter() - t_wall
     gloo_barrier(gloo)
     dt = ev0.elapsed_time(ev1) / 1e3
-    trace = S.trace()[trace_start:]
+    trace = S.trace()[trace_start:] if args.trace_out else []
     # steady state: the same K batches submitted back to back, one drain at the end
     # (no per-step pipeline fill/drain; each tenant's jobs still run in order)
     stream.synchronize()

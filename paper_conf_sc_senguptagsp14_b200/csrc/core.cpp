@@ -109,6 +109,8 @@ inline char* put_str(char* p, const char* s) {
 
 void Core::rec(uint64_t t, const char* kind, int gid, int eng, int slot, long tenant, long seq,
                long job, uint64_t a1, uint64_t a2) {
+  ++trace_records_;
+  if (!cfg_.record_trace) return;
   char buf[256];
   char* p = put_u64(buf, t);
   *p++ = ' ';
@@ -131,7 +133,6 @@ void Core::rec(uint64_t t, const char* kind, int gid, int eng, int slot, long te
   p = put_u64(p, a2);
   *p++ = '\n';
   trace_.append(buf, p - buf);
-  ++trace_records_;
 }
 
 // ---------------------------------------------------------------- orders

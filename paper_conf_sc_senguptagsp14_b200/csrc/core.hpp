@@ -35,6 +35,7 @@ struct CoreConfig {
   uint64_t Q = 1000000;
   uint64_t tfs_slice = 500000;        // TFS base slice S (R-28)
   std::vector<uint32_t> weights;      // DST device weights; empty = all 1
+  bool record_trace = true;           // keep the decision trace
 };
 
 // One job's scheduling record (the RCB view of a request).

@@ -409,6 +409,7 @@ class Runtime : public strings::Hooks {
     ccfg.joint = cfg.joint_select;
     ccfg.Q = cfg.quantum_ns;
     ccfg.tfs_slice = cfg.tfs_slice_ns;
+    ccfg.record_trace = cfg.trace_in_memory || cfg.trace_path;
     weights.assign(cfg.num_gpus, 1);
     if (cfg.device_weights) {
       for (int g = 0; g < cfg.num_gpus; ++g) {
