@@ -56,6 +56,8 @@ def parse_args():
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
+    p.add_argument("--configs", action="store_true",
+                   help="run BASELINE configs C1-C5 at full size (node mode, logical devices if G > GPUs)")
     p.add_argument("--fig2", action="store_true",
                    help="Fig. 2 analogue: N identical requests sequential vs co-resident vs separate contexts")
     p.add_argument("--sweep", action="store_true",
@@ -620,8 +622,71 @@ def fig2(args) -> None:
     print(json.dumps(res))
 
 
+def run_configs(args) -> None:
+    """All five BASELINE.json configurations at full size, MEASURED timing, node
+    mode (one process, G logical devices mapped round-robin onto the visible
+    GPUs).  Host buffers are allocated per tenant and reused by its jobs (every
+    tenant has c_t = 1, so its jobs never overlap).  Reports jobs/s, span,
+    Jain (service/elapsed), and the invariant check of the measured trace."""
+    import numpy as np
+    import torch
+
+    import strings_workload as W
+    from oracle import invariants
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+
+    ngpu = torch.cuda.device_count()
+    names = os.environ.get("BENCH_CONFIGS", "C1,C2,C3,C4,C5").split(",")
+    for name in names:
+        wl = W.CONFIGS[name]()
+        cfg = wl.config.resolved()
+        # per-tenant buffers sized for the tenant's largest job
+        need_in, need_out = {}, {}
+        for sp in wl.jobs:
+            need_in[sp.tenant] = [max(a, b) for a, b in zip(need_in.get(sp.tenant, [0, 0]),
+                                                          (sp.h2d_sizes() + [0])[:2])]
+            need_out[sp.tenant] = max(need_out.get(sp.tenant, 0), sum(sp.d2h_sizes()))
+        hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
+        hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
+        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=True)
+        ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+        t0 = time.perf_counter()
+        for sp in wl.jobs:
+            ins = [S.HostRef(hin[sp.tenant][i].data_ptr(), b) for i, b in enumerate(sp.h2d_sizes())]
+            outs = [S.HostRef(hout[sp.tenant].data_ptr(), b) for b in sp.d2h_sizes()]
+            S.submit_spec(ts[sp.tenant], sp, ins, outs)
+        st = S.drain()
+        wall = time.perf_counter() - t0
+        tr = S.trace()
+        infos = [S.job_info(i) for i in range(len(wl.jobs))]
+        S.shutdown()
+        errs = invariants.check(tr, wl)
+        busy, first, last = {}, {}, {}
+        for inf in infos:
+            busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
+            first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
+            last[inf.tenant] = max(last.get(inf.tenant, 0), inf.t_done[2])
+        xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
+        jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+        span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
+        print(json.dumps({"config": name, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
+                          "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
+                          "balancer": W.BALANCER_NAMES[cfg.balancer],
+                          "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
+                          "status": st, "jobs_per_s": round(len(wl.jobs) / span, 1),
+                          "span_ms": round(span * 1e3, 2), "wall_ms": round(wall * 1e3, 2),
+                          "jain": round(jain, 4), "invariant_violations": len(errs),
+                          "violations_sample": errs[:3],
+                          "note": "logical devices share the physical GPUs' host links and SMs"
+                          if cfg.num_gpus > ngpu else "one logical device per GPU"}), flush=True)
+        del hin, hout
+
+
 def main():
     args = parse_args()
+    if args.configs:
+        run_configs(args)
+        return
     if args.fig2:
         fig2(args)
         return

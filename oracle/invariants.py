@@ -7,8 +7,8 @@ Checks the invariants of SURVEY.md §8(c) on a canonical trace
       WAKE/START/DONE per phase, in the order H2D < KL < D2H, on one GID.
   I2  LAS ordering: every LAS admission (when LAS admission is on and joint
       selection is off) places a job of minimal weighted key among the
-      eligible ones; every LAS-policy wake pass wakes keys no larger than any
-      candidate it leaves unwoken (reading R-7).
+      eligible ones; every LAS-policy wake takes a minimal-key candidate of its
+      device at that moment (reading R-7).
   I3  resource exclusivity: <= 1 op per copy engine, <= P KL ops per device,
       <= A woken-unfinished ops, <= M resident jobs, <= c_t in-flight per tenant.
   I4  per-tenant order: a tenant's jobs are admitted in
@@ -140,11 +140,7 @@ def check(lines: List[str], wl: W.Workload) -> List[str]:
                     errs.append(f"I5 t={t} gid={g} TFS device idle with {len(c)} candidates")
             elif c and woken_unf[g] < A:
                 errs.append(f"I5 t={t} gid={g} {len(c)} candidates unwoken with budget {A - woken_unf[g]}")
-            if cfg.device_policy == W.LAS:
-                for w in woken_now.get(g, []):
-                    for u in c:
-                        if las_cmp(u, w) < 0:
-                            errs.append(f"I2 t={t} gid={g} LAS woke job {w} before lower-key job {u}")
+
 
     cur_t = None
     woken_now: Dict[int, List[int]] = {}
@@ -188,6 +184,13 @@ def check(lines: List[str], wl: W.Workload) -> List[str]:
             j, g, x = r.job, r.gid, r.eng
             if phase[j] != x or woken[j]:
                 errs.append(f"I1 job {j} woken for phase {x} out of order")
+            if cfg.device_policy == W.LAS:
+                # a LAS pass wakes candidates in key order: each woken job has the
+                # minimal key among the device's candidates at that moment (exact
+                # per pass, even when one timestamp holds several passes)
+                for u in candidates(g):
+                    if u != j and las_cmp(u, j) < 0:
+                        errs.append(f"I2 t={r.t} gid={g} LAS woke job {j} before lower-key job {u}")
             if cfg.device_policy == W.TFS:
                 others = {ten_of[i] for i in resident[g] if woken[i]} - {ten_of[j]}
                 if others:

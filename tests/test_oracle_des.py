@@ -411,3 +411,18 @@ def test_gwtmin_places_in_proportion_to_device_weights(weights, jobs):
     cfg.balancer = W.GMIN
     pl = placements(run_oracle(wl))
     assert max(pl.count(g) for g in range(len(weights))) - min(pl.count(g) for g in range(len(weights))) <= 1
+
+
+def test_invariant_checker_catches_las_wake_order():
+    # a LAS device trace with two WAKEs of one pass swapped must be flagged (I2)
+    wl = W.config_c3()
+    wl.config.device_policy = W.LAS
+    tr = run_oracle(wl).trace
+    assert invariants.check(tr, wl) == []
+    for i in range(len(tr) - 1):
+        a, b = tr[i].split(), tr[i + 1].split()
+        if a[1] == b[1] == "WAKE" and a[0] == b[0] and a[2] == b[2] and a[5] != b[5]:
+            m = tr[:i] + [tr[i + 1], tr[i]] + tr[i + 2:]
+            if any(e.startswith("I2") for e in invariants.check(m, wl)):
+                return
+    pytest.fail("no LAS wake-order mutation detected")
