@@ -74,6 +74,17 @@ def test_random_workloads_injected(seed):
     check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("seed", range(100, 124))
+def test_random_workloads_measured(seed):
+    # fuzz the real-time path: random classes/policies/budgets/caps/weights; the
+    # measured trace must satisfy I1-I5/I7 and every output must be exact
+    wl = W.random_workload(seed, max_gpus=3)
+    r = run_workload(wl, timing_mode=S.MEASURED)
+    assert r.status == S.OK
+    assert invariants.check(r.trace, wl) == []
+    check_outputs(wl, r)
+
+
 @pytest.mark.parametrize("name,kw", [("C1", {}), ("C2", dict(scale=16, jobs_per_tenant=4)),
                                      ("C5", dict(scale=64, jobs_per_tenant=4))])
 def test_measured_mode_invariants_and_outputs(name, kw):
