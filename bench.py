@@ -413,6 +413,7 @@ def run_strings(args, rank, world, torch, gloo):
                      "unit": "GB/s", "frac": round(link_gbs / link["bidir_gbs"], 4), "traffic": None,
                      "resource": "copy engines H2D+D2H (the step's dominant resource)",
                      "peak_source": "measured in this run: concurrent pinned H2D+D2H cudaMemcpyAsync 256 MiB"},
+        "roofline_kernel": _kernel_roofline(kl_lat, wl, peaks),
         "overlapped_roofline": {"tstar_ms": round(tstar * 1e3, 3), "span_ms": round(span_step * 1e3, 3),
                                 "frac": round(tstar / span_step, 4),
                                 "terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()}},
@@ -438,6 +439,25 @@ def run_strings(args, rank, world, torch, gloo):
         with open(args.trace_out, "w") as f:
             f.write("\n".join(trace) + "\n")
     return res, wl
+
+
+def _kernel_roofline(kl_lat, wl, peaks) -> dict:
+    """The dominant kernel work inside the timed step: XFER items run by the
+    persistent dispatcher on one P=2 SM partition (74 SMs), HBM-bound.
+    achieved = algorithmic bytes per item (read + write) / median device time
+    of the item (%globaltimer claim -> last CTA done)."""
+    import strings_workload as W
+    x = kl_lat.get("XFER")
+    n = [j for j in wl.jobs if j.kclass == W.XFER][0].n
+    if not x:
+        return None
+    gbs = 8 * n / (x["kl_device_us_p50"] * 1e3)
+    return {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline)", "bound": "hbm",
+            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+            "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": None,
+            "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (74 of 148 SMs); the other "
+            "partition often runs an item concurrently and shares HBM; device time includes the partition "
+            "broadcast and completion publish (stand-alone full-GPU runs: kernel_rooflines)"}
 
 
 def max_over(gloo, x: float) -> float:
