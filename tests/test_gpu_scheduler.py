@@ -143,6 +143,17 @@ def test_pairwise_mix_on_hardware(pair):
         check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("seed", [3, 8, 21])
+def test_kl_launch_mode(seed):
+    # kl_mode 1 (per-job launches of the same bodies, for profilers): same decisions in
+    # INJECTED mode, exact outputs; HIST/SCAN use a per-stream group barrier
+    wl = W.random_workload(seed, max_gpus=2)
+    r = run_workload(wl, timing_mode=S.INJECTED, kl_mode=1)
+    assert r.status == S.OK
+    assert r.trace == run_oracle(wl).trace
+    check_outputs(wl, r)
+
+
 def test_pageable_buffers_are_staged():
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)
