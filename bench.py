@@ -257,8 +257,9 @@ def run_strings(args, rank, world, torch, gloo):
             pins.append(p)
         ins.append(pins)
         outs.append([torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
+    arenas = S.torch_arenas(cfg.num_gpus, 1, cfg.admit_cap)      # PyTorch provides the device memory
     S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1, kl_mode=args.kl_mode,
-                       trace_in_memory=bool(args.trace_out))
+                       trace_in_memory=bool(args.trace_out), arenas=arenas)
     # the persistent dispatcher now owns every SM: no torch kernels, no device-wide sync until shutdown
     tenants = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
     stream = torch.cuda.Stream()

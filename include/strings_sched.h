@@ -98,6 +98,11 @@ typedef struct {
     const uint32_t* device_weights; /* num_gpus DST weights >= 1 (GWtMin); NULL = all 1.
                                        Logical devices sharing a physical GPU get SM partitions
                                        in proportion to their weights (heterogeneous pool).     */
+    void* const* ext_arenas;        /* optional, per physical GPU used: caller-owned device memory
+                                       (e.g. a torch allocation) for the resident-job slots; must
+                                       hold (logical devices on that GPU) x admit_cap x slot_bytes
+                                       and stay valid until strings_shutdown.  NULL = cudaMalloc.  */
+    const uint64_t* ext_arena_bytes;/* sizes of ext_arenas[i]                                      */
 } strings_config_t;
 
 /* Kernel descriptor: which tenant kernel the KL phase runs, and its sizes.

@@ -425,6 +425,8 @@ class Runtime : public strings::Hooks {
     for (int g = 0; g < cfg.num_gpus; ++g) logical[g].gid = g;
     if (has_gpu()) {
       strings_status_t s = init_gpus(nphys);
+      cfg.ext_arenas = nullptr;            // only read during init
+      cfg.ext_arena_bytes = nullptr;
       if (s != STRINGS_OK) {
         teardown_gpus();
         return s;
@@ -509,10 +511,20 @@ class Runtime : public strings::Hooks {
                               cudaMemcpyHostToDevice)))
         return STRINGS_ECUDA;
       if (!cuda_ok(cudaDeviceSynchronize())) return STRINGS_ECUDA;   // zeroed before the dispatcher starts
-      // arena: L logical devices x M slots
+      // arena: L logical devices x M slots (caller/torch-provided or our own)
       size_t arena = (size_t)ph->L * cfg.admit_cap * cfg.slot_bytes;
-      if (!cuda_ok(cudaMalloc(&ph->arena, arena))) return STRINGS_ENOMEM;
-      ph->arena_owned = true;
+      if (cfg.ext_arenas && cfg.ext_arenas[ph->dev]) {
+        if (!cfg.ext_arena_bytes || cfg.ext_arena_bytes[ph->dev] < arena) return STRINGS_EINVAL;
+        cudaPointerAttributes pa;
+        if (!cuda_ok(cudaPointerGetAttributes(&pa, cfg.ext_arenas[ph->dev])) || pa.type != cudaMemoryTypeDevice ||
+            pa.device != ph->dev)
+          return STRINGS_EINVAL;
+        ph->arena = static_cast<uint8_t*>(cfg.ext_arenas[ph->dev]);
+        ph->arena_owned = false;
+      } else {
+        if (!cuda_ok(cudaMalloc(&ph->arena, arena))) return STRINGS_ENOMEM;
+        ph->arena_owned = true;
+      }
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->kstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
       uint8_t* base = static_cast<uint8_t*>(hp) + sizeof(HostCtrl);
       KlRing* rings = reinterpret_cast<KlRing*>(base);

@@ -32,10 +32,16 @@ class RunResult:
 def run_workload(wl: W.Workload, timing_mode: int = S.INJECTED, pinned: bool = True,
                  inputs: Optional[List[List[np.ndarray]]] = None, keep_inputs: bool = False,
                  trace_path: Optional[str] = None, physical_gpus: int = 0, kl_mode: int = 0,
-                 slot_bytes: int = 0) -> RunResult:
+                 slot_bytes: int = 0, torch_memory: bool = True) -> RunResult:
     cfg = wl.config.resolved()
+    arenas = None
+    if timing_mode != S.DECISIONS_ONLY and torch_memory:
+        import torch                       # PyTorch provides the device memory (slot arenas)
+        nphys = physical_gpus or torch.cuda.device_count()
+        arenas = S.torch_arenas(cfg.num_gpus, min(nphys, cfg.num_gpus), cfg.admit_cap, slot_bytes)
+        physical_gpus = len(arenas)
     S.init_from_config(cfg, timing_mode=timing_mode, trace_path=trace_path, physical_gpus=physical_gpus,
-                       kl_mode=kl_mode, slot_bytes=slot_bytes)
+                       kl_mode=kl_mode, slot_bytes=slot_bytes, arenas=arenas)
     pinned_arrays = []
     try:
         for t in wl.tenants:
@@ -84,4 +90,5 @@ def run_workload(wl: W.Workload, timing_mode: int = S.INJECTED, pinned: bool = T
         S.shutdown()
         for a in pinned_arrays:
             S.free_pinned(a)
+        del arenas
     return RunResult(tr, outputs, infos, st, wall, status, kept)

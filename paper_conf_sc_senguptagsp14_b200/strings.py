@@ -36,7 +36,8 @@ class Config(C.Structure):
                 ("timing_mode", C.c_int32), ("quantum_ns", C.c_uint64), ("slot_bytes", C.c_uint64),
                 ("trace_path", C.c_char_p), ("trace_in_memory", C.c_int32),
                 ("kl_mode", C.c_int32), ("reserved", C.c_int32 * 6), ("tfs_slice_ns", C.c_uint64),
-                ("device_weights", C.POINTER(C.c_uint32))]
+                ("device_weights", C.POINTER(C.c_uint32)),
+                ("ext_arenas", C.POINTER(C.c_void_p)), ("ext_arena_bytes", C.POINTER(C.c_uint64))]
 
 
 class KernelDesc(C.Structure):
@@ -128,7 +129,10 @@ def _check(s: int, where: str) -> None:
 def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy=2, partitions=2,
          awake_budget=0, admit_cap=0, joint_select=-1, timing_mode=MEASURED, quantum_ns=1_000_000,
          slot_bytes=0, trace_path: Optional[str] = None, trace_in_memory=True, kl_mode=0,
-         tfs_slice_ns=0, device_weights: Optional[Sequence[int]] = None) -> None:
+         tfs_slice_ns=0, device_weights: Optional[Sequence[int]] = None,
+         arenas: Optional[Sequence] = None) -> None:
+    """arenas: optional per-physical-GPU device buffers (torch tensors or
+    (pointer, nbytes) pairs) for the resident-job slots; see torch_arenas()."""
     c = Config(num_gpus=num_gpus, physical_gpus=physical_gpus, balancer=balancer, las_admission=las_admission,
                device_policy=device_policy, partitions=partitions, awake_budget=awake_budget,
                admit_cap=admit_cap, joint_select=joint_select, timing_mode=timing_mode,
@@ -138,6 +142,12 @@ def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy
     if device_weights is not None:
         arr = (C.c_uint32 * len(device_weights))(*device_weights)
         c.device_weights = C.cast(arr, C.POINTER(C.c_uint32))
+    if arenas is not None:
+        ptrs = [(a.data_ptr(), a.numel() * a.element_size()) if hasattr(a, "data_ptr") else a for a in arenas]
+        pa = (C.c_void_p * len(ptrs))(*[p for p, _ in ptrs])
+        pb = (C.c_uint64 * len(ptrs))(*[b for _, b in ptrs])
+        c.ext_arenas = C.cast(pa, C.POINTER(C.c_void_p))
+        c.ext_arena_bytes = C.cast(pb, C.POINTER(C.c_uint64))
     _check(lib.strings_init(C.byref(c)), "strings_init")
 
 
@@ -147,6 +157,23 @@ def init_from_config(cfg, timing_mode=MEASURED, **kw) -> None:
          device_policy=cfg.device_policy, partitions=cfg.partitions, awake_budget=cfg.awake_budget,
          admit_cap=cfg.admit_cap, joint_select=cfg.joint_select, quantum_ns=cfg.quantum_ns,
          tfs_slice_ns=cfg.tfs_slice_ns, device_weights=cfg.device_weights, timing_mode=timing_mode, **kw)
+
+
+DEFAULT_SLOT_BYTES = 160 << 20
+
+
+def torch_arenas(num_gpus: int, physical_gpus: int, admit_cap: int, slot_bytes: int = 0):
+    """Device memory for the resident-job slots allocated by PyTorch (the north
+    star's "PyTorch for device memory"): one uint8 tensor per physical GPU sized
+    for the logical devices mapped onto it (logical g -> physical g mod N).
+    Keep the returned tensors alive until strings_shutdown."""
+    import torch
+    slot = slot_bytes or DEFAULT_SLOT_BYTES
+    out = []
+    for p in range(physical_gpus):
+        n_logical = len([g for g in range(num_gpus) if g % physical_gpus == p])
+        out.append(torch.empty(max(1, n_logical * admit_cap * slot), dtype=torch.uint8, device=f"cuda:{p}"))
+    return out
 
 
 def register_tenant(weight: int = 1, max_inflight: int = 1) -> int:

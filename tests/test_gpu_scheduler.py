@@ -154,6 +154,29 @@ def test_kl_launch_mode(seed):
     check_outputs(wl, r)
 
 
+def test_torch_arena_validation():
+    # the slot arena may come from PyTorch; a too-small or host allocation is rejected
+    import torch
+    small = torch.empty(1 << 20, dtype=torch.uint8, device="cuda:0")
+    with pytest.raises(S.StringsError) as e:
+        S.init(num_gpus=1, physical_gpus=1, arenas=[small])
+    assert e.value.status == S.EINVAL
+    host = torch.empty(1 << 20, dtype=torch.uint8).pin_memory()
+    with pytest.raises(S.StringsError):
+        S.init(num_gpus=1, physical_gpus=1, slot_bytes=1 << 10, admit_cap=4, arenas=[host])
+    arenas = S.torch_arenas(1, 1, 8, 1 << 20)
+    S.init(num_gpus=1, physical_gpus=1, admit_cap=8, slot_bytes=1 << 20, arenas=arenas)
+    try:
+        t = S.register_tenant()
+        x = np.arange(1024, dtype=np.uint32)
+        y = np.zeros(1024, np.uint32)
+        S.submit(t, S.make_desc(S.XFER, n=1024, seed=9), [x], [y])
+        assert S.sync(t) == S.OK
+        assert np.array_equal(y, K.xfer(x, 9))
+    finally:
+        S.shutdown()
+
+
 def test_pageable_buffers_are_staged():
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED, pinned=False)
