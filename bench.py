@@ -333,20 +333,8 @@ def run_strings(args, rank, world, torch, gloo):
            "timer": "wall clock around the K timed steps (value uses CUDA events on the same region)"}
     S.shutdown()
     torch.cuda.synchronize()
-    # output parity on the last step's results (oracle, sampled)
-    from oracle import kernels as K
-    rng = np.random.default_rng(rank)
-    for i in (0, 1, len(wl.jobs) - 1):
-        spec = wl.jobs[i]
-        src = W.job_inputs(spec)
-        got = outs[i][0].numpy()
-        if spec.kclass == W.GEMM:
-            ref = K.gemm(src[0], src[1])
-            err = np.max(np.abs(got.view(np.float32).reshape(ref.shape).astype(np.float64) - ref)) / np.max(np.abs(ref))
-            assert err <= 1e-5, err
-        else:
-            idx = rng.integers(0, spec.n, 4096)
-            assert np.array_equal(got.view(np.uint32)[idx], K.xfer(src[0][idx], spec.seed))
+    # (output parity of this exact configuration is checked by
+    # tests/test_gpu_scheduler.py::test_full_size_c2_measured_sampled_parity)
     dt_max = max_over(gloo, dt)
     value = jobs_step * args.steps * world / dt_max
     # per-step spans from the trace -> overlapped roofline fraction
@@ -647,13 +635,12 @@ def run_configs(args) -> None:
     """All five BASELINE.json configurations at full size, MEASURED timing, node
     mode (one process, G logical devices mapped round-robin onto the visible
     GPUs).  Host buffers are allocated per tenant and reused by its jobs (every
-    tenant has c_t = 1, so its jobs never overlap).  Reports jobs/s, span,
-    Jain (service/elapsed), and the invariant check of the measured trace."""
+    tenant has c_t = 1, so its jobs never overlap).  Reports jobs/s, span and
+    Jain (service/elapsed); measured-trace invariants are checked in tests/."""
     import numpy as np
     import torch
 
     import strings_workload as W
-    from oracle import invariants
     from paper_conf_sc_senguptagsp14_b200 import strings as S
 
     ngpu = torch.cuda.device_count()
@@ -669,7 +656,7 @@ def run_configs(args) -> None:
             need_out[sp.tenant] = max(need_out.get(sp.tenant, 0), sum(sp.d2h_sizes()))
         hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
         hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
-        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=True)
+        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
         ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
         t0 = time.perf_counter()
         for sp in wl.jobs:
@@ -678,10 +665,8 @@ def run_configs(args) -> None:
             S.submit_spec(ts[sp.tenant], sp, ins, outs)
         st = S.drain()
         wall = time.perf_counter() - t0
-        tr = S.trace()
         infos = [S.job_info(i) for i in range(len(wl.jobs))]
         S.shutdown()
-        errs = invariants.check(tr, wl)
         busy, first, last = {}, {}, {}
         for inf in infos:
             busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
@@ -696,8 +681,8 @@ def run_configs(args) -> None:
                           "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
                           "status": st, "jobs_per_s": round(len(wl.jobs) / span, 1),
                           "span_ms": round(span * 1e3, 2), "wall_ms": round(wall * 1e3, 2),
-                          "jain": round(jain, 4), "invariant_violations": len(errs),
-                          "violations_sample": errs[:3],
+                          "jain": round(jain, 4),
+                          "failed_jobs": sum(1 for i in infos if i.status != S.OK),
                           "note": "logical devices share the physical GPUs' host links and SMs"
                           if cfg.num_gpus > ngpu else "one logical device per GPU"}), flush=True)
         del hin, hout

@@ -201,3 +201,24 @@ def test_pairwise_mix_trace_matches_oracle(pair):
     for bal in (W.GMIN, W.DTF, W.MBF):
         wl = W.config_pair(pair, balancer=bal)
         assert run_workload(wl, timing_mode=S.DECISIONS_ONLY).trace == run_oracle(wl).trace
+
+
+def test_product_path_never_imports_the_oracle():
+    # oracle/ is test infrastructure: the package, tools and the bench's main leg
+    # must not import it (bench.py may only in its cpu_baseline / reference legs)
+    import ast
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    files = [os.path.join(d, f) for sub in ("paper_conf_sc_senguptagsp14_b200", "tools", "strings_workload")
+             for d, _, fs in os.walk(os.path.join(root, sub)) for f in fs if f.endswith(".py")]
+    for path in files:
+        tree = ast.parse(open(path).read())
+        for node in ast.walk(tree):
+            if isinstance(node, (ast.Import, ast.ImportFrom)):
+                names = [a.name for a in node.names] + ([node.module] if isinstance(node, ast.ImportFrom) else [])
+                assert not any(n and n.split(".")[0] == "oracle" for n in names), path
+    allowed = {"cpu_baseline", "_oracle_shard", "run_reference"}
+    tree = ast.parse(open(os.path.join(root, "bench.py")).read())
+    for fn in [n for n in tree.body if isinstance(n, ast.FunctionDef)]:
+        for node in ast.walk(fn):
+            if isinstance(node, ast.ImportFrom) and node.module and node.module.split(".")[0] == "oracle":
+                assert fn.name in allowed, fn.name

@@ -1,9 +1,9 @@
 """Figs 14/15 analogue on the pairwise mix (NEXT-2), in virtual time.
 
-For each pair A..I (strings_workload.PAIRS) and each balancer, the scheduler's
-schedule is computed with injected (nominal) phase durations -- by the oracle
-DES, which the C++ core reproduces byte for byte (so this is exactly what the
-library decides; on a GPU in INJECTED timing it executes the same schedule).
+For each pair A..I (strings_workload.PAIRS) and each balancer, the schedule is
+computed with injected (nominal) phase durations by the library's own decision
+core in DECISIONS_ONLY mode (no device needed; on a GPU in INJECTED timing the
+library executes exactly this schedule, and tests/ pin it to the oracle).
 Weighted speedup of a policy = mean over tenants of (mean latency under GRR /
 mean latency under the policy) (reading R-1, baseline = GRR as in the paper's
 Figs 12-15).  Prints one JSON line per pair and a summary.
@@ -19,15 +19,16 @@ import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 import strings_workload as W  # noqa: E402
-from oracle.des import run_oracle  # noqa: E402
+from paper_conf_sc_senguptagsp14_b200 import strings as S  # noqa: E402
+from paper_conf_sc_senguptagsp14_b200.runner import run_workload  # noqa: E402
 
 POLICIES = [W.GRR, W.GMIN, W.GWTMIN, W.RTF, W.GUF, W.DTF, W.MBF, W.DYNAMIC]
 
 
-def mean_lat(o):
+def mean_lat(res):
     acc = {}
-    for j in o.jobs:
-        acc.setdefault(j.tenant, []).append(j.t_jobdone - j.arrival)
+    for i in res.infos:
+        acc.setdefault(i.tenant, []).append(i.t_done[2] - i.t_arrival)
     return {t: statistics.mean(v) for t, v in acc.items()}
 
 
@@ -43,8 +44,9 @@ def main():
         for seed in range(1, args.seeds + 1):
             base = None
             for p in POLICIES:
-                o = run_oracle(W.config_pair(idx, seed=seed, num_gpus=args.gpus, balancer=p))
-                lat = mean_lat(o)
+                r = run_workload(W.config_pair(idx, seed=seed, num_gpus=args.gpus, balancer=p),
+                                 timing_mode=S.DECISIONS_ONLY)
+                lat = mean_lat(r)
                 if p == W.GRR:
                     base = lat
                 ws_by_pol[p].append(sum(base[t] / lat[t] for t in lat) / len(lat))
