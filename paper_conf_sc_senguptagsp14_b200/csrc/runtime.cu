@@ -329,6 +329,14 @@ struct Tenant {
   bool active = true;
 };
 
+// PMT staging copy threads: most of the host's cores (the engine thread and the
+// caller keep one each); STRINGS_COPY_THREADS overrides.
+int copy_threads() {
+  if (const char* e = getenv("STRINGS_COPY_THREADS")) return std::max(0, atoi(e));
+  const int hw = (int)std::thread::hardware_concurrency();
+  return std::min(12, std::max(2, hw - 4));
+}
+
 class Runtime;
 Runtime* g_rt = nullptr;
 std::mutex g_init_mu;
@@ -365,7 +373,7 @@ class Runtime : public strings::Hooks {
   };
   std::priority_queue<VEv, std::vector<VEv>, std::greater<VEv>> vheap;
   StagingPool staging;
-  CopyPool copier{6};
+  CopyPool copier{copy_threads()};
   std::deque<std::pair<JobCtx*, uint64_t>> finalize_q;
   std::condition_variable cv_final;
   std::vector<std::thread> finalizers;
