@@ -153,6 +153,9 @@ typedef struct {
                                                      including issuing the woken ops            */
     uint64_t engine_busy_ns[8][3];                /* per logical device (first 8), per engine   */
     int32_t  num_gpus, physical_gpus, partitions, sms_per_partition;
+    uint64_t issue_ns;                            /* part of decision_ns spent issuing woken ops
+                                                     (cudaMemcpyAsync, stream writes, KL ring
+                                                     publish); decision_ns - issue_ns = decisions */
 } strings_stats_t;
 
 /* Initialise the runtime (gPool creation): enumerate the GPUs,

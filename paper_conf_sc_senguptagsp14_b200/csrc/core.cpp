@@ -53,6 +53,7 @@ bool Completion::operator<(const Completion& o) const {
 
 Core::Core(const CoreConfig& cfg, Hooks* hooks) : cfg_(cfg), hooks_(hooks), next_epoch_(cfg.Q) {
   devs_.resize(cfg_.G);
+  dev_dirty_.assign(cfg_.G, 0);
   busy_ns_.assign(cfg_.G, std::vector<uint64_t>(3, 0));
   for (int g = 0; g < cfg_.G; ++g) {
     devs_[g].gid = g;
@@ -274,6 +275,14 @@ void Core::admission(uint64_t t) {
   std::vector<Agg>& aggs = scratch_aggs_;
   aggs.resize(devs_.size());
   const bool need_aggs = cfg_.balancer != B_GRR && cfg_.balancer != B_GMIN && cfg_.balancer != B_GWTMIN;
+  // Aggregates depend only on the resident jobs' phases and the SFT, neither of
+  // which changes during admission: compute them once, then refresh only the
+  // device that received a job.  Every selection below is a linear min scan in
+  // admission order (no sort): O(T + T*G) per placement.
+  for (auto& d : devs_) {
+    if (need_aggs) aggs[d.gid] = aggregate(d);
+    else aggs[d.gid].n = d.resident.size();
+  }
   for (;;) {
     elig.clear();
     adm.clear();
@@ -284,32 +293,23 @@ void Core::admission(uint64_t t) {
       if (!tn.pending.empty() && tn.inflight < tn.c && tn.pending.front()->arrived)
         elig.push_back(tn.pending.front());
     if (elig.empty()) return;
-    for (int g : adm) {
-      if (need_aggs) aggs[g] = aggregate(devs_[g]);
-      else aggs[g].n = devs_[g].resident.size();
-    }
-    std::sort(elig.begin(), elig.end(),
-              [this](const Job* a, const Job* b) { return admission_before(a, b); });
     Job* pick = nullptr;
     int gid = -1, pol = B_GMIN;
     uint64_t sc = 0;
     if (joint) {
+      // first job in admission order still placed by GMin (no sample yet) ...
       for (Job* j : elig)
-        if (effective_policy(j) == B_GMIN) {
-          pick = j;
-          break;
-        }
+        if (effective_policy(j) == B_GMIN && (!pick || admission_before(j, pick))) pick = j;
       if (pick) {
         pol = B_GMIN;
         gid = select_device(pol, pick, adm, aggs, &sc);
       } else {
-        bool have = false;
+        // ... else the lexicographic min of (score, admission order, GID)
         for (Job* j : elig) {
           int p = effective_policy(j);
           for (int g : adm) {
             uint64_t s = score_from(p, aggs[g], j);
-            if (!have || s < sc) {
-              have = true;
+            if (!pick || s < sc || (s == sc && j != pick && admission_before(j, pick))) {
               sc = s;
               pick = j;
               gid = g;
@@ -319,11 +319,14 @@ void Core::admission(uint64_t t) {
         }
       }
     } else {
-      pick = elig.front();
+      for (Job* j : elig)
+        if (!pick || admission_before(j, pick)) pick = j;
       pol = effective_policy(pick);
       gid = select_device(pol, pick, adm, aggs, &sc);
     }
     place(t, pick, gid, pol, sc);
+    if (need_aggs) aggs[gid] = aggregate(devs_[gid]);
+    else aggs[gid].n = devs_[gid].resident.size();
   }
 }
 
@@ -337,6 +340,7 @@ void Core::place(uint64_t t, Job* j, int gid, int policy, uint64_t score) {
   j->t_place = t;
   j->place_order = place_counter_++;
   devs_[gid].resident.push_back(j);
+  dev_dirty_[gid] = 1;
   ++decisions_;
   rec(t, "PLACE", gid, -1, -1, j->tenant, j->seq, (long)j->id, policy, score);
 }
@@ -476,6 +480,7 @@ void Core::complete(const Completion& c) {
   if (d.busy[c.engine].at(c.slot) != j) throw std::logic_error("complete: engine not running job");
   const uint64_t t = c.t;
   d.busy[c.engine][c.slot] = nullptr;
+  dev_dirty_[c.gid] = 1;
   --d.woken_unfinished;
   j->done[c.engine] = t;
   j->phase += 1;
@@ -493,6 +498,7 @@ void Core::complete(const Completion& c) {
     ++jobs_done_;
     rec(t, "JOB_DONE", c.gid, -1, -1, j->tenant, j->seq, (long)j->id, t - j->arrival, 0);
     feedback(t, j);
+    adm_dirty_ = true;
     d.resident.erase(std::find(d.resident.begin(), d.resident.end(), j));
     --tn.inflight;
     jobs_.erase(it);
@@ -552,11 +558,19 @@ void Core::step(uint64_t t, std::vector<Completion> dones, bool first) {
       Job* j = *arr_.begin();
       arr_.erase(arr_.begin());
       j->arrived = true;
+      adm_dirty_ = true;
       rec(t, "ARRIVE", -1, -1, -1, j->tenant, j->seq, (long)j->id, j->prio, 0);
     }
   }
-  admission(t);
-  for (auto& d : devs_) dispatch(t, d);
+  if (adm_dirty_) {
+    adm_dirty_ = false;
+    admission(t);
+  }
+  for (auto& d : devs_)
+    if (dev_dirty_[d.gid]) {
+      dev_dirty_[d.gid] = 0;
+      dispatch(t, d);
+    }
 }
 
 void Core::close_epochs_before(uint64_t t) {

@@ -185,6 +185,11 @@ class Core {
   std::vector<Job*> scratch_cand_, scratch_ph_[3], scratch_copies_, scratch_elig_;
   std::vector<int> scratch_adm_;
   std::vector<Agg> scratch_aggs_;
+  // Work-skipping: a dispatch pass on a device whose state did not change since
+  // its last pass, or an admission pass with no job arrival/completion since the
+  // last one, is a no-op (each pass runs to its fixed point), so it is skipped.
+  bool adm_dirty_ = false;
+  std::vector<char> dev_dirty_;
 };
 
 // Algorithmic kernel bytes and tensor FLOP of a job.

@@ -363,6 +363,7 @@ class Runtime : public strings::Hooks {
   uint64_t first_submit = 0, last_done = 0;
   uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
   uint64_t decision_ns = 0;            // time inside Core::step (decisions + op issue)
+  uint64_t issue_ns = 0;               // of which: issuing woken ops (on_wake)
   // in-flight physical ops (measured mode): (job, engine)
   std::vector<std::pair<JobCtx*, int>> inflight;
   // virtual DONE events (injected / decisions-only)
@@ -629,6 +630,12 @@ class Runtime : public strings::Hooks {
       jc->phys_done[engine] = true;
       return;
     }
+    const uint64_t i0 = mono_ns();
+    issue(j, jc, engine);
+    issue_ns += mono_ns() - i0;
+  }
+
+  void issue(strings::Job& j, JobCtx* jc, int engine) {
     Logical& lg = logical[j.gid];
     Phys* ph = lg.phys;
     set_dev(ph->dev);
@@ -1283,6 +1290,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->trace_records = r.core->trace_records();
   st->decisions = r.core->decisions();
   st->decision_ns = r.decision_ns;
+  st->issue_ns = r.issue_ns;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

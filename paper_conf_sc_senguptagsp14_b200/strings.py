@@ -66,7 +66,8 @@ class Stats(C.Structure):
                 ("kernel_flop", C.c_uint64), ("trace_records", C.c_uint64), ("decisions", C.c_uint64),
                 ("decision_ns", C.c_uint64),
                 ("engine_busy_ns", (C.c_uint64 * 3) * 8), ("num_gpus", C.c_int32),
-                ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32)]
+                ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32),
+                ("issue_ns", C.c_uint64)]
 
 
 def _load() -> C.CDLL:
