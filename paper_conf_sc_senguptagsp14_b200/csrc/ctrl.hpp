@@ -55,8 +55,14 @@ struct DispatchParams {
   PartState* parts;                   // [L * P]
   const int* part_start;              // [L * P + 1] first CTA of each partition (device memory)
   int L, P;                           // logical devices hosted, partitions per logical device
-  uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
+  uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off,
+                                      // bit1 host doorbell
   uint64_t fault_job;                 // fault injection (STRINGS_FAULT_JOB): trap on this job id
+  uint32_t poll_max_ns;               // idle-poll back-off cap (STRINGS_POLL_MAX_NS)
+  // Device-memory doorbells (default): word 32*ld = ring tail of logical device
+  // ld, word 32*L = shutdown; written by the host through cuStreamWriteValue32.
+  // flags bit1 (STRINGS_DOORBELL=host): poll the host-mapped ring tail instead.
+  uint32_t* doorbells;
 };
 
 inline size_t host_ctrl_bytes(int L) {

@@ -10,8 +10,13 @@
 // operands fit), split into NP = L*P partitions of contiguous CTAs.  Partition
 // q serves logical device q / P.  Its leader (CTA rank 0, thread 0):
 //   1. waits until the previous item is finished by every CTA (done_gen),
-//   2. polls the ring tail in host memory (ld.acquire.sys, nanosleep back-off)
-//      and claims the next item with a CAS on the device claim counter,
+//   2. polls its logical device's doorbell word in device memory (ld.acquire.gpu,
+//      nanosleep back-off; the host writes the ring tail there with
+//      cuStreamWriteValue32) and claims the next item with a CAS on the device
+//      claim counter, then reads the item from the host-mapped ring.  Polling
+//      L2 instead of host memory keeps the PCIe link free for the tenants'
+//      DMA: with 16 leaders polling host memory the copy engines lost 4x
+//      throughput (profiles/r01_doorbell.md),
 //   3. copies the item into the partition mailbox and publishes gen+1
 //      (st.release.gpu).
 // Every CTA of the partition waits for the new generation, runs its share of
@@ -73,8 +78,9 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         while (ld_acquire_gpu(&ps->done_gen) != seen) __nanosleep(32);
         uint32_t g;
         uint32_t backoff = 32;
+        const bool host_db = p.flags & 2u;
         for (;;) {
-          const uint32_t tail = ld_acquire_sys(&p.rings[ld].tail);
+          const uint32_t tail = host_db ? ld_acquire_sys(&p.rings[ld].tail) : ld_acquire_gpu(&p.doorbells[32 * ld]);
           const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&p.heads[ld]);
           if (h < tail) {
             if (atomicCAS(&p.heads[ld], h, h + 1) == h) {
@@ -97,13 +103,13 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
             }
             continue;
           }
-          if (ld_acquire_sys(&p.ctrl->shutdown)) {
+          if (host_db ? ld_acquire_sys(&p.ctrl->shutdown) : ld_acquire_gpu(&p.doorbells[32 * p.L])) {
             g = kStop;
             break;
           }
           if (p.flags & 1u) continue;
           __nanosleep(backoff);
-          if (backoff < 1024) backoff <<= 1;
+          if (backoff < p.poll_max_ns) backoff <<= 1;
         }
         st_release_gpu(&ps->gen, g);
       }

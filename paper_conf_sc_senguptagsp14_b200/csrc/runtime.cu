@@ -209,6 +209,13 @@ struct Phys {
   uint8_t* arena = nullptr;
   bool arena_owned = false;
   cudaStream_t kstream = nullptr;
+  // Copy streams shared by the logical devices hosted here (STRINGS_COPY_STREAMS=physical)
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  // KL doorbells: ring tails + shutdown in device memory, written by stream
+  // memory ops on this stream, so the dispatcher polls L2, not host memory
+  cudaStream_t dbstream = nullptr;
+  uint8_t* doorbells = nullptr;
+  bool host_doorbell = false;          // STRINGS_DOORBELL=host: leaders poll the host ring tail
   bool kernel_running = false;
   std::vector<int> part_start;         // [L*P + 1] partition table (host copy)
   std::vector<cudaEvent_t> ev_pool;
@@ -510,12 +517,16 @@ class Runtime : public strings::Hooks {
           return STRINGS_ECUDA;
         g_write_value32 = reinterpret_cast<WriteValue32Fn>(fn);
       }
-      // device state: heads[L] (padded) + parts[L*P] + partition table
+      // device state: heads[L] (padded) + parts[L*P] + partition table + doorbells
+      // (one 128-B line per logical device's ring tail, one for shutdown)
       size_t heads_bytes = 128 * (size_t)ph->L;
       size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
       size_t table_bytes = sizeof(int) * ph->part_start.size();
-      if (!cuda_ok(cudaMalloc(&ph->dev_state, heads_bytes + parts_bytes + table_bytes))) return STRINGS_ENOMEM;
-      if (!cuda_ok(cudaMemset(ph->dev_state, 0, heads_bytes + parts_bytes))) return STRINGS_ECUDA;
+      size_t db_off = align_up(heads_bytes + parts_bytes + table_bytes);
+      size_t db_bytes = 128 * ((size_t)ph->L + 1);
+      if (!cuda_ok(cudaMalloc(&ph->dev_state, db_off + db_bytes))) return STRINGS_ENOMEM;
+      if (!cuda_ok(cudaMemset(ph->dev_state, 0, db_off + db_bytes))) return STRINGS_ECUDA;
+      ph->doorbells = ph->dev_state + db_off;
       if (!cuda_ok(cudaMemcpy(ph->dev_state + heads_bytes + parts_bytes, ph->part_start.data(), table_bytes,
                               cudaMemcpyHostToDevice)))
         return STRINGS_ECUDA;
@@ -535,13 +546,27 @@ class Runtime : public strings::Hooks {
         ph->arena_owned = true;
       }
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->kstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+      if (!cuda_ok(cudaStreamCreateWithFlags(&ph->dbstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+      const char* dbm = getenv("STRINGS_DOORBELL");
+      ph->host_doorbell = dbm && strcmp(dbm, "host") == 0;
       uint8_t* base = static_cast<uint8_t*>(hp) + sizeof(HostCtrl);
       KlRing* rings = reinterpret_cast<KlRing*>(base);
       KlDone* dones = reinterpret_cast<KlDone*>(base + sizeof(KlRing) * ph->L);
+      const char* cs = getenv("STRINGS_COPY_STREAMS");
+      const bool shared_copy = cs && strcmp(cs, "physical") == 0;
+      if (shared_copy) {
+        if (!cuda_ok(cudaStreamCreateWithFlags(&ph->h2d, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        if (!cuda_ok(cudaStreamCreateWithFlags(&ph->d2h, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+      }
       for (auto& lg : logical) {
         if (lg.phys != ph.get()) continue;
-        if (!cuda_ok(cudaStreamCreateWithFlags(&lg.h2d, cudaStreamNonBlocking))) return STRINGS_ECUDA;
-        if (!cuda_ok(cudaStreamCreateWithFlags(&lg.d2h, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        if (shared_copy) {
+          lg.h2d = ph->h2d;
+          lg.d2h = ph->d2h;
+        } else {
+          if (!cuda_ok(cudaStreamCreateWithFlags(&lg.h2d, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+          if (!cuda_ok(cudaStreamCreateWithFlags(&lg.d2h, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+        }
         if (kl_mode == 1) {
           lg.kl_streams.resize(cfg.partitions);
           for (auto& s : lg.kl_streams)
@@ -577,6 +602,10 @@ class Runtime : public strings::Hooks {
         dp.flags = fl ? (uint32_t)strtoul(fl, nullptr, 0) : 0u;
         const char* fj = getenv("STRINGS_FAULT_JOB");
         dp.fault_job = fj ? (uint64_t)strtoull(fj, nullptr, 0) : ~0ull;
+        const char* pm = getenv("STRINGS_POLL_MAX_NS");
+        dp.poll_max_ns = pm ? (uint32_t)strtoul(pm, nullptr, 0) : 1024u;
+        dp.doorbells = reinterpret_cast<uint32_t*>(ph->doorbells);
+        if (ph->host_doorbell) dp.flags |= 2u;
         if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
       }
@@ -591,19 +620,26 @@ class Runtime : public strings::Hooks {
       if (ph->kernel_running) {
         ph->ctrl->shutdown = 1;
         std::atomic_thread_fence(std::memory_order_seq_cst);
+        g_write_value32(reinterpret_cast<CUstream>(ph->dbstream),
+                        reinterpret_cast<CUdeviceptr>(ph->doorbells + 128 * (size_t)ph->L), 1, 0);
         cudaStreamSynchronize(ph->kstream);
         ph->kernel_running = false;
       }
       for (auto& lg : logical) {
         if (lg.phys != ph.get()) continue;
-        if (lg.h2d) cudaStreamSynchronize(lg.h2d), cudaStreamDestroy(lg.h2d);
-        if (lg.d2h) cudaStreamSynchronize(lg.d2h), cudaStreamDestroy(lg.d2h);
+        if (lg.h2d && lg.h2d != ph->h2d) cudaStreamSynchronize(lg.h2d), cudaStreamDestroy(lg.h2d);
+        if (lg.d2h && lg.d2h != ph->d2h) cudaStreamSynchronize(lg.d2h), cudaStreamDestroy(lg.d2h);
         for (auto s : lg.kl_streams) cudaStreamSynchronize(s), cudaStreamDestroy(s);
         lg.h2d = lg.d2h = nullptr;
         lg.kl_streams.clear();
         if (lg.kl_sync) cudaFree(lg.kl_sync);
         lg.kl_sync = nullptr;
       }
+      if (ph->dbstream) cudaStreamSynchronize(ph->dbstream), cudaStreamDestroy(ph->dbstream);
+      ph->dbstream = nullptr;
+      if (ph->h2d) cudaStreamSynchronize(ph->h2d), cudaStreamDestroy(ph->h2d);
+      if (ph->d2h) cudaStreamSynchronize(ph->d2h), cudaStreamDestroy(ph->d2h);
+      ph->h2d = ph->d2h = nullptr;
       for (auto e : ph->ev_pool) cudaEventDestroy(e);
       ph->ev_pool.clear();
       if (ph->kstream) cudaStreamDestroy(ph->kstream);
@@ -698,6 +734,16 @@ class Runtime : public strings::Hooks {
           lg.tail += 1;
           lg.ring->tail = lg.tail;
           std::atomic_thread_fence(std::memory_order_seq_cst);
+          if (!ph->host_doorbell) {
+            // doorbell: the new tail into device memory through a stream memory op
+            CUresult r = g_write_value32(reinterpret_cast<CUstream>(ph->dbstream),
+                                         reinterpret_cast<CUdeviceptr>(ph->doorbells + 128 * (size_t)lg.local),
+                                         lg.tail, 0);
+            if (r != CUDA_SUCCESS) {
+              g_last_cuda_error.store(10000 + (int32_t)r);
+              ok = false;
+            }
+          }
         }
       } else {
         const int si = lg.next_kl_stream;
