@@ -23,6 +23,7 @@ JSON line keys beyond the base contract:
 from __future__ import annotations
 
 import argparse
+import dataclasses
 import json
 import os
 import statistics
@@ -56,6 +57,7 @@ def parse_args():
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
+    p.add_argument("--config-repeats", type=int, default=3, help="timed runs per config in --configs")
     p.add_argument("--configs", action="store_true",
                    help="run BASELINE configs C1-C5 at full size (node mode, logical devices if G > GPUs)")
     p.add_argument("--fig2", action="store_true",
@@ -202,8 +204,14 @@ def kernel_rooflines(torch, S, peaks) -> list:
 
 
 # ------------------------------------------------------- strings arm
-def tstar_device(wl, link, hbm_gbs, tflops) -> float:
-    """Overlapped roofline T*_d (s) for one device running all of wl."""
+def tstar_device(wl, link, hbm_gbs, tflops, kl_slots: int = 2) -> float:
+    """Overlapped roofline T*_d (s) for one physical device running all of wl
+    (SURVEY §8(d)): the busiest of the host-link directions (and their
+    concurrent sum), HBM, the tensor pipe, the longest per-tenant chain
+    (H2D -> KL -> D2H of its jobs back to back, c_t = 1) and, for open-loop
+    arrivals, the latest arrival plus its job's chain.  A KL slot owns 1 /
+    kl_slots of the SMs (tensor time); HBM is credited at the full peak, so T*
+    stays a lower bound."""
     import strings_workload as W
     bh, bd = link["h2d_gbs"] * 1e9, link["d2h_gbs"] * 1e9
     bb = link["bidir_gbs"] * 1e9
@@ -211,19 +219,25 @@ def tstar_device(wl, link, hbm_gbs, tflops) -> float:
     d2h = sum(sum(j.d2h_sizes()) for j in wl.jobs)
     hbm = flop = 0
     chains = {}
+    t0 = min(j.arrival_ns for j in wl.jobs) if wl.jobs else 0
+    arrival_bound = 0.0
     for j in wl.jobs:
         if j.kclass == W.GEMM:
             jb = 2 * j.m * j.k + 2 * j.k * j.n + 4 * j.m * j.n
             jf = 2 * j.m * j.n * j.k * j.reps
+        elif j.kclass == W.HIST:
+            jb, jf = j.n + 1024, 0
         else:
             jb, jf = 8 * j.n, 0
         hbm += jb
         flop += jf
-        kl = max(jb / (hbm_gbs * 1e9), jf / (tflops * 1e12 / 2))   # a KL slot has half the SMs (P=2)
-        chains[j.tenant] = chains.get(j.tenant, 0.0) + sum(j.h2d_sizes()) / bh + kl + sum(j.d2h_sizes()) / bd
+        kl = max(jb / (hbm_gbs * 1e9), jf / (tflops * 1e12 / kl_slots))
+        one = sum(j.h2d_sizes()) / bh + kl + sum(j.d2h_sizes()) / bd
+        chains[j.tenant] = chains.get(j.tenant, 0.0) + one
+        arrival_bound = max(arrival_bound, (j.arrival_ns - t0) / 1e9 + one)
     terms = {"h2d": h2d / bh, "d2h": d2h / bd, "bidir": (h2d + d2h) / bb,
              "hbm": (hbm + h2d + d2h) / (hbm_gbs * 1e9), "tensor": flop / (tflops * 1e12),
-             "chain": max(chains.values())}
+             "chain": max(chains.values()), "arrival": arrival_bound}
     return max(terms.values()), terms
 
 
@@ -638,15 +652,21 @@ def run_configs(args) -> None:
     """All five BASELINE.json configurations at full size, MEASURED timing, node
     mode (one process, G logical devices mapped round-robin onto the visible
     GPUs).  Host buffers are allocated per tenant and reused by its jobs (every
-    tenant has c_t = 1, so its jobs never overlap).  Reports jobs/s, span and
-    Jain (service/elapsed); measured-trace invariants are checked in tests/."""
-    import numpy as np
+    tenant has c_t = 1, so its jobs never overlap).  One untimed warm-up run,
+    then `--config-repeats` timed runs; reports the median jobs/s and span, the
+    overlapped roofline T* of the physical GPU (all jobs of the
+    config share its host link and SMs) and T*/span, and Jain
+    (service/elapsed).  Measured-trace invariants are checked in tests/."""
+    import statistics
+
     import torch
 
     import strings_workload as W
     from paper_conf_sc_senguptagsp14_b200 import strings as S
 
     ngpu = torch.cuda.device_count()
+    peaks = measured_peaks()
+    link = host_link_peaks(torch)
     names = os.environ.get("BENCH_CONFIGS", "C1,C2,C3,C4,C5").split(",")
     for name in names:
         wl = W.CONFIGS[name]()
@@ -659,33 +679,52 @@ def run_configs(args) -> None:
             need_out[sp.tenant] = max(need_out.get(sp.tenant, 0), sum(sp.d2h_sizes()))
         hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
         hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
-        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
-        ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
-        t0 = time.perf_counter()
-        for sp in wl.jobs:
-            ins = [S.HostRef(hin[sp.tenant][i].data_ptr(), b) for i, b in enumerate(sp.h2d_sizes())]
-            outs = [S.HostRef(hout[sp.tenant].data_ptr(), b) for b in sp.d2h_sizes()]
-            S.submit_spec(ts[sp.tenant], sp, ins, outs)
-        st = S.drain()
-        wall = time.perf_counter() - t0
-        infos = [S.job_info(i) for i in range(len(wl.jobs))]
-        S.shutdown()
-        busy, first, last = {}, {}, {}
-        for inf in infos:
-            busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
-            first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
-            last[inf.tenant] = max(last.get(inf.tenant, 0), inf.t_done[2])
-        xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
-        jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
-        span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
+        runs = []
+        for rep in range(1 + args.config_repeats):
+            S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
+            ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+            t0 = time.perf_counter()
+            for sp in wl.jobs:
+                ins = [S.HostRef(hin[sp.tenant][i].data_ptr(), b) for i, b in enumerate(sp.h2d_sizes())]
+                outs = [S.HostRef(hout[sp.tenant].data_ptr(), b) for b in sp.d2h_sizes()]
+                S.submit_spec(ts[sp.tenant], sp, ins, outs)
+            st = S.drain()
+            wall = time.perf_counter() - t0
+            infos = [S.job_info(i) for i in range(len(wl.jobs))]
+            S.shutdown()
+            if rep == 0:
+                continue                    # warm-up
+            busy, first, last = {}, {}, {}
+            for inf in infos:
+                busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
+                first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
+                last[inf.tenant] = max(last.get(inf.tenant, 0), inf.t_done[2])
+            xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
+            jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+            span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
+            runs.append({"span": span, "wall": wall, "jain": jain, "status": st,
+                         "failed": sum(1 for i in infos if i.status != S.OK)})
+        # arrivals are submit times in MEASURED mode: the whole config is offered at t = 0
+        wl0 = dataclasses.replace(wl, jobs=[dataclasses.replace(j, arrival_ns=0) for j in wl.jobs])
+        tstar, terms = tstar_device(wl0, link, peaks["hbm_gbs"],
+                                    peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"],
+                                    kl_slots=max(1, (cfg.num_gpus + ngpu - 1) // ngpu) * cfg.partitions)
+        spans = [r["span"] for r in runs]
+        span = statistics.median(spans)
         print(json.dumps({"config": name, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
                           "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
                           "balancer": W.BALANCER_NAMES[cfg.balancer],
                           "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
-                          "status": st, "jobs_per_s": round(len(wl.jobs) / span, 1),
-                          "span_ms": round(span * 1e3, 2), "wall_ms": round(wall * 1e3, 2),
-                          "jain": round(jain, 4),
-                          "failed_jobs": sum(1 for i in infos if i.status != S.OK),
+                          "status": max((r["status"] for r in runs), key=abs),
+                          "failed_jobs": sum(r["failed"] for r in runs),
+                          "jobs_per_s": round(len(wl.jobs) / span, 1),
+                          "span_ms": round(span * 1e3, 2), "span_ms_min_max": [round(min(spans) * 1e3, 2),
+                                                                            round(max(spans) * 1e3, 2)],
+                          "runs": len(runs),
+                          "tstar_ms": round(tstar * 1e3, 3), "roofline_frac": round(tstar / span, 4),
+                          "tstar_terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()},
+                          "jain": round(statistics.median(r["jain"] for r in runs), 4),
+                          "host_link_gbs": {k: round(v, 2) for k, v in link.items()},
                           "note": "logical devices share the physical GPUs' host links and SMs"
                           if cfg.num_gpus > ngpu else "one logical device per GPU"}), flush=True)
         del hin, hout

@@ -136,7 +136,7 @@ typedef struct {
     uint64_t t_start[3], t_done[3];          /* per phase H2D, KL, D2H (library clock)       */
     int32_t  kl_slot;                        /* logical KL slot                               */
     int32_t  kl_partition;                   /* physical SM partition that ran the KL        */
-    uint64_t kl_gpu_start_ns, kl_gpu_end_ns; /* %globaltimer: partition claimed the item, last
+    uint64_t kl_gpu_start_ns, kl_gpu_end_ns; /* %globaltimer: partition leader saw the doorbell, last
                                                 CTA finished                                  */
     uint64_t kl_gpu_exec_ns;                 /* %globaltimer: the body started (after broadcast) */
     uint64_t kl_host_issue_ns;               /* CLOCK_REALTIME: item published in the ring     */
@@ -156,6 +156,9 @@ typedef struct {
     uint64_t issue_ns;                            /* part of decision_ns spent issuing woken ops
                                                      (cudaMemcpyAsync, stream writes, KL ring
                                                      publish); decision_ns - issue_ns = decisions */
+    int64_t  gpu_clock_offset_ns[8];              /* per physical GPU (first 8): %globaltimer minus
+                                                     CLOCK_REALTIME, calibrated at init (kl_gpu_*
+                                                     stamps - offset = host clock); 0 if unknown */
 } strings_stats_t;
 
 /* Initialise the runtime (gPool creation): enumerate the GPUs,

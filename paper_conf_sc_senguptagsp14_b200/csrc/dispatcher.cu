@@ -10,18 +10,15 @@
 // operands fit), split into NP = L*P partitions of contiguous CTAs.  Partition
 // q serves logical device q / P.  Its leader (CTA rank 0, thread 0):
 //   1. waits until the previous item is finished by every CTA (done_gen),
-//   2. polls its logical device's doorbell word in device memory (ld.acquire.gpu,
-//      nanosleep back-off; the host writes the ring tail there with
-//      cuStreamWriteValue32) and claims the next item with a CAS on the device
-//      claim counter, then reads the item from the host-mapped ring.  Polling
-//      L2 instead of host memory keeps the PCIe link free for the tenants'
-//      DMA: with 16 leaders polling host memory the copy engines lost 4x
-//      throughput (profiles/r01_doorbell.md),
-//   3. copies the item into the partition mailbox and publishes gen+1
-//      (st.release.gpu).
-// Every CTA of the partition waits for the new generation, runs its share of
-// the item, and the last CTA to finish writes the completion word and the
-// %globaltimer stamps back to host memory (st.release.sys).
+//   2. polls the next entry of its logical device's KL ring in device memory
+//      (ld.acquire.gpu, nanosleep back-off; the host publishes (seq, slot) with
+//      one cuStreamWriteValue64) and claims it with a CAS on the device claim
+//      counter.  The dispatch path never reads host memory (ctrl.hpp),
+//   3. publishes (slot, gen+1) in one 64-bit st.release.gpu.
+// Every CTA of the partition waits for the new generation, reads the job's item
+// from the device item table, runs its share of the item, and the last CTA to
+// finish writes the completion word and the %globaltimer stamps back to host
+// memory (gpu-scope fence + plain store).
 #include <cstdio>
 
 #include "ctrl.hpp"
@@ -43,6 +40,14 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint64_t ld_acquire_gpu_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
@@ -60,7 +65,7 @@ __device__ __forceinline__ void partition_of(int b, int NP, const int* part_star
 __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams p) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ KlItem s_item;
-  __shared__ uint32_t s_gen;
+  __shared__ uint32_t s_gen, s_slot;
   GemmSmem sm = carve_smem(smem);
   if ((smem_u32(smem) & 1023u) != 0) __trap();   // SWIZZLE_128B tiles need a 1 KB-aligned base
   const int NP = p.L * p.P;
@@ -69,54 +74,61 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   const int rank = blockIdx.x - start;
   const int ld = q / p.P;
   PartState* ps = p.parts + q;
+  const KlItem* table = p.items + (size_t)ld * p.M;
+  const uint64_t* ring = p.ring + (size_t)ld * kRing;
   const uint32_t tmem = cta_setup(sm);
   uint32_t mma_phase = 0;
   uint32_t seen = 0;
   for (;;) {
-    if (threadIdx.x == 0) {
-      if (rank == 0) {
+    if (threadIdx.x < 32) {                       // warp 0
+      const unsigned lane = threadIdx.x;
+      if (rank == 0 && lane == 0) {               // the partition leader
         while (ld_acquire_gpu(&ps->done_gen) != seen) __nanosleep(32);
-        uint32_t g;
         uint32_t backoff = 32;
-        const bool host_db = p.flags & 2u;
+        uint64_t pub;
         for (;;) {
-          const uint32_t tail = host_db ? ld_acquire_sys(&p.rings[ld].tail) : ld_acquire_gpu(&p.doorbells[32 * ld]);
           const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&p.heads[ld]);
-          if (h < tail) {
+          const uint64_t e = ld_acquire_gpu_u64(&ring[h % kRing]);
+          if ((uint32_t)(e >> 32) == h + 1) {     // entry h published
+            const uint64_t t_seen = globaltimer();
             if (atomicCAS(&p.heads[ld], h, h + 1) == h) {
-              const KlItem* src = &p.rings[ld].items[h % kRing];
-              // 16-B loads that bypass stale cached lines (.cv), issued back to back: one
-              // PCIe round trip for the whole item instead of one per 32-bit field
-              uint4 v[sizeof(KlItem) / 16];
-#pragma unroll
-              for (int w = 0; w < (int)(sizeof(KlItem) / 16); ++w)
-                asm volatile("ld.global.cv.v4.u32 {%0,%1,%2,%3}, [%4];"
-                             : "=r"(v[w].x), "=r"(v[w].y), "=r"(v[w].z), "=r"(v[w].w)
-                             : "l"(reinterpret_cast<const uint4*>(src) + w));
-              uint4* d4 = reinterpret_cast<uint4*>(&ps->item);
-#pragma unroll
-              for (int w = 0; w < (int)(sizeof(KlItem) / 16); ++w) d4[w] = v[w];
               ps->ring_idx = h % kRing;
-              ps->t_start = globaltimer();
-              g = seen + 1;
+              ps->seq = h + 1;
+              ps->t_start = t_seen;
+              pub = ((uint64_t)(uint32_t)e << 32) | (seen + 1);
               break;
             }
-            continue;
+            continue;                             // the other KL slot took it
           }
-          if (host_db ? ld_acquire_sys(&p.ctrl->shutdown) : ld_acquire_gpu(&p.doorbells[32 * p.L])) {
-            g = kStop;
+          if (ld_acquire_gpu(p.stop)) {
+            pub = kStop;
             break;
           }
           if (p.flags & 1u) continue;
           __nanosleep(backoff);
           if (backoff < p.poll_max_ns) backoff <<= 1;
         }
-        st_release_gpu(&ps->gen, g);
+        st_release_gpu_u64(&ps->gen, pub);
       }
-      uint32_t g;
-      while ((g = ld_acquire_gpu(&ps->gen)) == seen) __nanosleep(32);
-      s_gen = g;
-      if (g != kStop) s_item = ps->item;
+      uint64_t gw = 0;
+      if (lane == 0)                              // one poller per CTA
+        while ((uint32_t)(gw = ld_acquire_gpu_u64(&ps->gen)) == seen) __nanosleep(32);
+      __syncwarp();                               // orders lane 0's acquire before the item loads
+      gw = __shfl_sync(0xffffffffu, gw, 0);
+      const uint32_t g = (uint32_t)gw, slot = (uint32_t)(gw >> 32);
+      if (g != kStop) {
+        // the 512-B item straight from the device item table: one warp-wide L2 read
+        // (.cg: the copy engine wrote it, no stale L1 line)
+        uint4 v;
+        asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                     : "l"(reinterpret_cast<const uint4*>(table + slot) + lane) : "memory");
+        reinterpret_cast<uint4*>(&s_item)[lane] = v;
+      }
+      if (lane == 0) {
+        s_gen = g;
+        s_slot = slot;
+      }
     }
     __syncthreads();
     const uint32_t g = s_gen;
@@ -125,7 +137,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     const KlItem it = s_item;
     if (it.job == p.fault_job) __trap();          // fault injection (tests the watchdog)
     if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
-    run_item(it, &ps->item, true, rank, S, sm, tmem, mma_phase, &ps->sync);
+    run_item(it, table + s_slot, true, rank, S, sm, tmem, mma_phase, &ps->sync);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -142,7 +154,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         // DMA from device memory, so a gpu-scope fence + plain store is sufficient
         // (a sys-scope release costs ~3 us more per item, PCIe-fence round trip).
         __threadfence();
-        d->seq = it.seq;
+        d->seq = ps->seq;
         st_release_gpu(&ps->done_gen, seen);
       }
     }
@@ -167,6 +179,18 @@ __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_const
   if (gemm) cta_teardown(tmem);
 }
 
+// Clock calibration ping-pong: sample i is taken when the host raises flag to
+// i+1; the kernel answers with %globaltimer (host-mapped memory both ways).
+__global__ void clock_probe_kernel(const uint32_t* flag, uint64_t* out, int n) {
+  for (int i = 0; i < n; ++i) {
+    while (ld_acquire_sys(flag) != (uint32_t)(i + 1)) {
+    }
+    const uint64_t t = globaltimer();
+    *reinterpret_cast<volatile uint64_t*>(out + i) = t;
+    __threadfence_system();
+  }
+}
+
 }  // namespace strings_dev
 
 // ----------------------------------------------------------------- host side
@@ -178,6 +202,11 @@ cudaError_t launch_dispatcher(const strings_dev::DispatchParams& p, int grid, cu
                                        (int)strings_dev::kSmemGemm);
   if (e != cudaSuccess) return e;
   strings_dev::dispatcher_kernel<<<grid, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaStream_t s) {
+  strings_dev::clock_probe_kernel<<<1, 1, 0, s>>>(flag, out, n);
   return cudaGetLastError();
 }
 

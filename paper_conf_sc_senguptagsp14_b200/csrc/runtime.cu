@@ -39,12 +39,12 @@
 namespace strings {
 cudaError_t launch_dispatcher(const strings_dev::DispatchParams& p, int grid, cudaStream_t s);
 cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t s);
+cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaStream_t s);
 }  // namespace strings
 
 using strings_dev::HostCtrl;
 using strings_dev::KlDone;
 using strings_dev::KlItem;
-using strings_dev::KlRing;
 using strings_dev::kRing;
 
 namespace {
@@ -81,6 +81,8 @@ uint64_t mono_ns() {
 // Driver API entry points, fetched through the runtime (no libcuda link).
 typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 WriteValue32Fn g_write_value32 = nullptr;
+typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+WriteValue64Fn g_write_value64 = nullptr;
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -168,6 +170,7 @@ struct JobCtx {
   bool issued[3] = {false, false, false};
   bool phys_done[3] = {false, false, false};
   uint32_t kl_seq = 0;
+  bool item_ok = false;                // KL work item built (and staged) at H2D issue
   uint32_t copy_seq[3] = {0, 0, 0};
   int kl_idx = -1;
   int kl_partition = -1;
@@ -187,7 +190,9 @@ struct Logical {
   int next_kl_stream = 0;
   uint8_t* arena = nullptr;            // M slots of slot_bytes
   std::vector<int> free_slots;
-  KlRing* ring = nullptr;              // host pointer
+  KlItem* item_host = nullptr;         // [M] pinned staging of the slots' work items
+  CUdeviceptr item_dev = 0;            // [M] device copies (dispatcher reads them)
+  CUdeviceptr ring_dev = 0;            // [kRing] device ring entries (seq << 32 | slot)
   KlDone* done = nullptr;              // host pointer, kRing entries
   uint32_t tail = 0;                   // items published
   uint32_t completed = 0;              // items whose completion was consumed
@@ -211,11 +216,15 @@ struct Phys {
   cudaStream_t kstream = nullptr;
   // Copy streams shared by the logical devices hosted here (STRINGS_COPY_STREAMS=physical)
   cudaStream_t h2d = nullptr, d2h = nullptr;
-  // KL doorbells: ring tails + shutdown in device memory, written by stream
-  // memory ops on this stream, so the dispatcher polls L2, not host memory
+  // KL queue in device memory (ctrl.hpp): ring entries + doorbells written by
+  // stream memory ops on this stream, work items DMA'd by the H2D streams
   cudaStream_t dbstream = nullptr;
   uint8_t* doorbells = nullptr;
-  bool host_doorbell = false;          // STRINGS_DOORBELL=host: leaders poll the host ring tail
+  uint8_t* ring_dev = nullptr;         // [L][kRing] u64
+  uint8_t* items_dev = nullptr;        // [L][M] KlItem
+  KlItem* items_host = nullptr;        // [L][M] pinned staging
+  int64_t clock_offset_ns = 0;         // %globaltimer - CLOCK_REALTIME (ping-pong, min RTT)
+  uint64_t clock_rtt_ns = 0;
   bool kernel_running = false;
   std::vector<int> part_start;         // [L*P + 1] partition table (host copy)
   std::vector<cudaEvent_t> ev_pool;
@@ -523,10 +532,30 @@ class Runtime : public strings::Hooks {
       size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
       size_t table_bytes = sizeof(int) * ph->part_start.size();
       size_t db_off = align_up(heads_bytes + parts_bytes + table_bytes);
-      size_t db_bytes = 128 * ((size_t)ph->L + 1);
-      if (!cuda_ok(cudaMalloc(&ph->dev_state, db_off + db_bytes))) return STRINGS_ENOMEM;
-      if (!cuda_ok(cudaMemset(ph->dev_state, 0, db_off + db_bytes))) return STRINGS_ECUDA;
+      size_t db_bytes = 128;                                         // shutdown word
+      size_t ring_off = align_up(db_off + db_bytes);
+      size_t ring_bytes = sizeof(uint64_t) * kRing * ph->L;
+      size_t items_off = align_up(ring_off + ring_bytes);
+      size_t items_bytes = sizeof(KlItem) * (size_t)cfg.admit_cap * ph->L;
+      if (!cuda_ok(cudaMalloc(&ph->dev_state, items_off + items_bytes))) return STRINGS_ENOMEM;
+      if (!cuda_ok(cudaMemset(ph->dev_state, 0, items_off + items_bytes))) return STRINGS_ECUDA;
       ph->doorbells = ph->dev_state + db_off;
+      ph->ring_dev = ph->dev_state + ring_off;
+      ph->items_dev = ph->dev_state + items_off;
+      {
+        void* ih = nullptr;
+        if (!cuda_ok(cudaHostAlloc(&ih, items_bytes, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+        memset(ih, 0, items_bytes);
+        ph->items_host = static_cast<KlItem*>(ih);
+      }
+      if (!g_write_value64) {
+        cudaDriverEntryPointQueryResult q;
+        void* fn = nullptr;
+        if (!cuda_ok(cudaGetDriverEntryPoint("cuStreamWriteValue64", &fn, cudaEnableDefault, &q)) ||
+            q != cudaDriverEntryPointSuccess || !fn)
+          return STRINGS_ECUDA;
+        g_write_value64 = reinterpret_cast<WriteValue64Fn>(fn);
+      }
       if (!cuda_ok(cudaMemcpy(ph->dev_state + heads_bytes + parts_bytes, ph->part_start.data(), table_bytes,
                               cudaMemcpyHostToDevice)))
         return STRINGS_ECUDA;
@@ -547,11 +576,7 @@ class Runtime : public strings::Hooks {
       }
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->kstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->dbstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
-      const char* dbm = getenv("STRINGS_DOORBELL");
-      ph->host_doorbell = dbm && strcmp(dbm, "host") == 0;
-      uint8_t* base = static_cast<uint8_t*>(hp) + sizeof(HostCtrl);
-      KlRing* rings = reinterpret_cast<KlRing*>(base);
-      KlDone* dones = reinterpret_cast<KlDone*>(base + sizeof(KlRing) * ph->L);
+      KlDone* dones = reinterpret_cast<KlDone*>(static_cast<uint8_t*>(hp) + sizeof(HostCtrl));
       const char* cs = getenv("STRINGS_COPY_STREAMS");
       const bool shared_copy = cs && strcmp(cs, "physical") == 0;
       if (shared_copy) {
@@ -577,7 +602,9 @@ class Runtime : public strings::Hooks {
         }
         lg.arena = ph->arena + (size_t)lg.local * cfg.admit_cap * cfg.slot_bytes;
         for (int s = cfg.admit_cap - 1; s >= 0; --s) lg.free_slots.push_back(s);
-        lg.ring = rings + lg.local;
+        lg.item_host = ph->items_host + (size_t)lg.local * cfg.admit_cap;
+        lg.item_dev = reinterpret_cast<CUdeviceptr>(ph->items_dev) + sizeof(KlItem) * (size_t)lg.local * cfg.admit_cap;
+        lg.ring_dev = reinterpret_cast<CUdeviceptr>(ph->ring_dev) + sizeof(uint64_t) * (size_t)kRing * lg.local;
         lg.done = dones + (size_t)lg.local * kRing;
         lg.ctr = ph->ctrs + lg.local;
         lg.ctr_dev = reinterpret_cast<CUdeviceptr>(static_cast<CopyCounters*>(ph->ctrs_dev) + lg.local);
@@ -590,22 +617,23 @@ class Runtime : public strings::Hooks {
       if (kl_mode == 0) {
         strings_dev::DispatchParams dp;
         uint8_t* dbase = static_cast<uint8_t*>(ph->ctrl_dev);
-        dp.ctrl = reinterpret_cast<HostCtrl*>(dbase);
-        dp.rings = reinterpret_cast<KlRing*>(dbase + sizeof(HostCtrl));
-        dp.done = reinterpret_cast<KlDone*>(dbase + sizeof(HostCtrl) + sizeof(KlRing) * ph->L);
+        dp.done = reinterpret_cast<KlDone*>(dbase + sizeof(HostCtrl));
         dp.heads = reinterpret_cast<uint32_t*>(ph->dev_state);
         dp.parts = reinterpret_cast<strings_dev::PartState*>(ph->dev_state + heads_bytes);
         dp.part_start = reinterpret_cast<const int*>(ph->dev_state + heads_bytes + parts_bytes);
         dp.L = ph->L;
         dp.P = cfg.partitions;
+        dp.M = cfg.admit_cap;
+        dp.ring = reinterpret_cast<const uint64_t*>(ph->ring_dev);
+        dp.items = reinterpret_cast<const KlItem*>(ph->items_dev);
         const char* fl = getenv("STRINGS_DISPATCH_FLAGS");
         dp.flags = fl ? (uint32_t)strtoul(fl, nullptr, 0) : 0u;
         const char* fj = getenv("STRINGS_FAULT_JOB");
         dp.fault_job = fj ? (uint64_t)strtoull(fj, nullptr, 0) : ~0ull;
         const char* pm = getenv("STRINGS_POLL_MAX_NS");
         dp.poll_max_ns = pm ? (uint32_t)strtoul(pm, nullptr, 0) : 1024u;
-        dp.doorbells = reinterpret_cast<uint32_t*>(ph->doorbells);
-        if (ph->host_doorbell) dp.flags |= 2u;
+        dp.stop = reinterpret_cast<const uint32_t*>(ph->doorbells);
+        if (!calibrate_clock(ph.get())) return STRINGS_ECUDA;
         if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
       }
@@ -613,15 +641,53 @@ class Runtime : public strings::Hooks {
     return STRINGS_OK;
   }
 
+  // Offset between the device's %globaltimer (the dispatcher's KL stamps) and
+  // the host CLOCK_REALTIME (issue/observe stamps), so that strings_job_info's
+  // KL timestamps can be placed on one time line.  Best of 16 ping-pongs.
+  bool calibrate_clock(Phys* ph) {
+    void* hp = nullptr;
+    if (!cuda_ok(cudaHostAlloc(&hp, 256, cudaHostAllocMapped))) return false;
+    memset(hp, 0, 256);
+    void* dp = nullptr;
+    bool ok = cuda_ok(cudaHostGetDevicePointer(&dp, hp, 0));
+    volatile uint32_t* flag = static_cast<volatile uint32_t*>(hp);
+    volatile uint64_t* out = reinterpret_cast<volatile uint64_t*>(static_cast<uint8_t*>(hp) + 64);
+    const int n = 16;
+    ok = ok && cuda_ok(strings::launch_clock_probe(static_cast<const uint32_t*>(dp),
+                                                   reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(dp) + 64), n,
+                                                   ph->kstream));
+    uint64_t best_rtt = UINT64_MAX;
+    for (int i = 0; ok && i < n; ++i) {
+      const uint64_t t_send = real_ns();
+      std::atomic_thread_fence(std::memory_order_seq_cst);
+      *flag = (uint32_t)(i + 1);
+      const uint64_t deadline = mono_ns() + 2000000000ull;
+      while (out[i] == 0) {
+        if (mono_ns() > deadline) {
+          ok = false;
+          break;
+        }
+      }
+      const uint64_t t_recv = real_ns();
+      if (!ok) break;
+      const uint64_t rtt = t_recv - t_send;
+      if (rtt < best_rtt) {
+        best_rtt = rtt;
+        ph->clock_offset_ns = (int64_t)out[i] - (int64_t)(t_send + rtt / 2);
+      }
+    }
+    ok = ok && cuda_ok(cudaStreamSynchronize(ph->kstream));
+    ph->clock_rtt_ns = best_rtt;
+    cudaFreeHost(hp);
+    return ok;
+  }
+
   void teardown_gpus() {
     for (auto& ph : phys) {
       if (ph->L == 0) continue;
       cudaSetDevice(ph->dev);
       if (ph->kernel_running) {
-        ph->ctrl->shutdown = 1;
-        std::atomic_thread_fence(std::memory_order_seq_cst);
-        g_write_value32(reinterpret_cast<CUstream>(ph->dbstream),
-                        reinterpret_cast<CUdeviceptr>(ph->doorbells + 128 * (size_t)ph->L), 1, 0);
+        g_write_value32(reinterpret_cast<CUstream>(ph->dbstream), reinterpret_cast<CUdeviceptr>(ph->doorbells), 1, 0);
         cudaStreamSynchronize(ph->kstream);
         ph->kernel_running = false;
       }
@@ -646,6 +712,8 @@ class Runtime : public strings::Hooks {
       if (ph->arena && ph->arena_owned) cudaFree(ph->arena);
       if (ph->dev_state) cudaFree(ph->dev_state);
       if (ph->ctrl) cudaFreeHost(ph->ctrl);
+      if (ph->items_host) cudaFreeHost(ph->items_host);
+      ph->items_host = nullptr;
       if (ph->ctrs) cudaFreeHost(ph->ctrs);
       ph->ctrs = nullptr;
       ph->kstream = nullptr;
@@ -671,6 +739,23 @@ class Runtime : public strings::Hooks {
     issue_ns += mono_ns() - i0;
   }
 
+  // The job's KL work item (device pointers of its slot; GEMM tensor maps).
+  bool build_item(const strings::Job& j, const JobCtx* jc, KlItem& it) {
+    memset(&it, 0, sizeof it);
+    it.kclass = jc->desc.kclass;
+    it.job = j.id;
+    it.in0 = jc->dev_in[0];
+    it.in1 = jc->dev_in[1];
+    it.out0 = jc->dev_out;
+    it.n = jc->desc.n;
+    it.m = jc->desc.m;
+    it.k = jc->desc.k;
+    it.reps = jc->desc.reps ? jc->desc.reps : 1;
+    it.alpha = jc->desc.alpha;
+    it.seed = jc->desc.seed;
+    return it.kclass != STRINGS_GEMM || encode_gemm_maps(it);
+  }
+
   void issue(strings::Job& j, JobCtx* jc, int engine) {
     Logical& lg = logical[j.gid];
     Phys* ph = lg.phys;
@@ -693,6 +778,19 @@ class Runtime : public strings::Hooks {
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma,
                                        jc->in[i].bytes, cudaMemcpyHostToDevice, lg.h2d));
       ok = ok && signal_copy(lg, jc, engine, lg.h2d);
+      if (ok && kl_mode == 0) {
+        // The job's KL work item goes to the device item table (the dispatcher
+        // never reads host memory, ctrl.hpp) on the queue stream, after the input
+        // copies are queued and off the H2D stream; the KL's ring entry is written
+        // later on the same queue stream, hence after this copy.  The slot's
+        // previous item copy finished before the slot was freed (its KL ran).
+        KlItem& it = lg.item_host[jc->slot];
+        jc->item_ok = build_item(j, jc, it);
+        const size_t bytes = it.kclass == STRINGS_GEMM ? sizeof(KlItem) : offsetof(KlItem, tmap_a);
+        if (jc->item_ok)
+          ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(lg.item_dev + sizeof(KlItem) * jc->slot), &it, bytes,
+                                       cudaMemcpyHostToDevice, ph->dbstream));
+      }
     } else if (engine == strings::ENG_D2H) {
       uint64_t off = 0;
       for (size_t i = 0; i < jc->out.size() && ok; ++i) {
@@ -702,50 +800,30 @@ class Runtime : public strings::Hooks {
         off = align_up(off + jc->out[i].bytes);
       }
       ok = ok && signal_copy(lg, jc, engine, lg.d2h);
+    } else if (kl_mode == 0) {
+      if (!jc->item_ok || lg.tail - lg.completed >= (uint32_t)kRing) {
+        ok = false;   // bad item (fault localised to this job); a full ring cannot happen with A <= kRing
+      } else {
+        // one 64-bit stream memory op publishes ring entry (seq, slot); it is ordered
+        // after the item copy issued on the same stream at H2D time
+        const uint32_t idx = lg.tail % kRing;
+        const uint32_t seq = lg.tail + 1;
+        jc->kl_issue = real_ns();
+        jc->kl_seq = seq;
+        jc->kl_idx = (int)idx;
+        CUresult r = g_write_value64(reinterpret_cast<CUstream>(ph->dbstream), lg.ring_dev + sizeof(uint64_t) * idx,
+                                     ((uint64_t)seq << 32) | (uint32_t)jc->slot, 0);
+        if (r != CUDA_SUCCESS) {
+          g_last_cuda_error.store(10000 + (int32_t)r);
+          ok = false;
+        } else {
+          lg.tail = seq;
+        }
+      }
     } else {
       KlItem it;
-      memset(&it, 0, sizeof it);
-      it.kclass = jc->desc.kclass;
-      it.job = j.id;
-      it.in0 = jc->dev_in[0];
-      it.in1 = jc->dev_in[1];
-      it.out0 = jc->dev_out;
-      it.n = jc->desc.n;
-      it.m = jc->desc.m;
-      it.k = jc->desc.k;
-      it.reps = jc->desc.reps ? jc->desc.reps : 1;
-      it.alpha = jc->desc.alpha;
-      it.seed = jc->desc.seed;
-      if (it.kclass == STRINGS_GEMM && !encode_gemm_maps(it)) ok = false;
-      if (!ok) {
-        // leave the op failed (fault localised to this job)
-      } else if (kl_mode == 0) {
-        if (lg.tail - lg.completed >= (uint32_t)kRing) {
-          ok = false;  // cannot happen with A <= kRing; treat as a job fault
-        } else {
-          const uint32_t idx = lg.tail % kRing;
-          it.seq = lg.tail + 1;
-          it.t_issue = jc->kl_issue = real_ns();
-          KlItem* dst = &lg.ring->items[idx];
-          memcpy(dst, &it, sizeof it);
-          jc->kl_seq = it.seq;
-          jc->kl_idx = (int)idx;
-          std::atomic_thread_fence(std::memory_order_seq_cst);
-          lg.tail += 1;
-          lg.ring->tail = lg.tail;
-          std::atomic_thread_fence(std::memory_order_seq_cst);
-          if (!ph->host_doorbell) {
-            // doorbell: the new tail into device memory through a stream memory op
-            CUresult r = g_write_value32(reinterpret_cast<CUstream>(ph->dbstream),
-                                         reinterpret_cast<CUdeviceptr>(ph->doorbells + 128 * (size_t)lg.local),
-                                         lg.tail, 0);
-            if (r != CUDA_SUCCESS) {
-              g_last_cuda_error.store(10000 + (int32_t)r);
-              ok = false;
-            }
-          }
-        }
-      } else {
+      ok = build_item(j, jc, it);
+      if (ok) {
         const int si = lg.next_kl_stream;
         cudaStream_t s = lg.kl_streams[si];
         lg.next_kl_stream = (lg.next_kl_stream + 1) % (int)lg.kl_streams.size();
@@ -1337,6 +1415,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->decisions = r.core->decisions();
   st->decision_ns = r.decision_ns;
   st->issue_ns = r.issue_ns;
+  for (size_t i = 0; i < r.phys.size() && i < 8; ++i) st->gpu_clock_offset_ns[i] = r.phys[i]->clock_offset_ns;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

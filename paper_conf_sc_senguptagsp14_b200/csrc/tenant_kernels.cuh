@@ -16,10 +16,11 @@ namespace strings_dev {
 
 constexpr int kThreads = 256;
 
-// One KL work item (also the layout of the host-mapped KL ring entries).
-// GEMM items carry the TMA tensor maps of A and B (encoded on the host per job).
+// One KL work item: built by the host at the job's H2D issue and DMA'd into the
+// device item table with the job's inputs (ctrl.hpp).  GEMM items carry the TMA
+// tensor maps of A, B and C (encoded on the host per job).
 struct __align__(64) KlItem {
-  uint32_t seq;          // claim number (1-based, monotone per ring); written last by the host
+  uint32_t seq;          // claim number (1-based, monotone per ring); set by the claiming leader
   uint32_t kclass;
   uint64_t job;
   uint64_t in0, in1, out0;   // device pointers
@@ -28,7 +29,7 @@ struct __align__(64) KlItem {
   float alpha;
   uint32_t seed;
   uint32_t pad;
-  uint64_t t_issue;      // host CLOCK_REALTIME ns when the item was published (telemetry)
+  uint64_t t_issue;      // unused (telemetry is kept on the host)
   uint64_t sync;         // stand-alone launches: GroupSync* to use (0 = the default one)
   uint64_t pad3[4];
   uint8_t tmap_a[128];   // CUtensorMap of A (bf16 M x K, K-major, box 64 x 128, SWIZZLE_128B)

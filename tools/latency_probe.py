@@ -36,6 +36,7 @@ def main(n_jobs=300, n=1024):
             rtt.append((time.perf_counter() - t0) * 1e6)
         assert float(y[0]) == 3.0
         infos = [S.job_info(i) for i in range(n_jobs)][20:]
+        off = S.stats().gpu_clock_offset_ns[0]
     finally:
         S.shutdown()
     med = lambda v: round(statistics.median(v), 2)
@@ -47,12 +48,13 @@ def main(n_jobs=300, n=1024):
         "kl_device_us": med([(i.kl_gpu_end_ns - i.kl_gpu_start_ns) / 1e3 for i in infos]),
         "submit_to_done_us": med([(i.t_done[2] - i.t_arrival) / 1e3 for i in infos]),
         "sync_rtt_us": med(rtt[20:]),
-        # decomposition of the KL phase (host CLOCK_REALTIME vs device %globaltimer; meaningful
-        # only if the two clocks share an epoch -- check issue_to_claim >= 0)
-        "kl_issue_to_claim_us": med([(i.kl_gpu_start_ns - i.kl_host_issue_ns) / 1e3 for i in infos]),
+        # decomposition of the KL phase: device %globaltimer stamps moved onto the host
+        # CLOCK_REALTIME line with the offset the library calibrates at init (+-RTT/2)
+        "gpu_clock_offset_ns": off,
+        "kl_issue_to_claim_us": med([(i.kl_gpu_start_ns - off - i.kl_host_issue_ns) / 1e3 for i in infos]),
         "kl_claim_to_exec_us": med([(i.kl_gpu_exec_ns - i.kl_gpu_start_ns) / 1e3 for i in infos]),
         "kl_exec_to_end_us": med([(i.kl_gpu_end_ns - i.kl_gpu_exec_ns) / 1e3 for i in infos]),
-        "kl_end_to_observe_us": med([(i.kl_host_observe_ns - i.kl_gpu_end_ns) / 1e3 for i in infos]),
+        "kl_end_to_observe_us": med([(i.kl_host_observe_ns - (i.kl_gpu_end_ns - off)) / 1e3 for i in infos]),
         "kl_issue_to_observe_us": med([(i.kl_host_observe_ns - i.kl_host_issue_ns) / 1e3 for i in infos]),
     }
     print(json.dumps(out))
