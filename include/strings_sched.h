@@ -88,7 +88,7 @@ typedef struct {
     int32_t  timing_mode;    /* STRINGS_TIMING_*                                                */
     uint64_t quantum_ns;     /* LAS epoch Q; 0 -> 1,000,000 (R-5)                               */
     uint64_t slot_bytes;     /* device bytes per resident job slot; 0 -> 160 MiB                */
-    const char* trace_path;  /* if non-NULL the decision trace is written there at drain/shutdown */
+    const char* trace_path;  /* if non-NULL the decision trace is written there at drain/shutdown (string copied at init) */
     int32_t  trace_in_memory;/* 1 = keep the trace for strings_trace_copy; with trace_path NULL
                                 and trace_in_memory 0 no record is formatted (counters only)    */
     int32_t  kl_mode;        /* 0 = persistent dispatcher kernel (product); 1 = per-job launches of

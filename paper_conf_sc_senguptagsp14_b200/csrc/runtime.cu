@@ -360,6 +360,7 @@ std::mutex g_init_mu;
 class Runtime : public strings::Hooks {
  public:
   strings_config_t cfg{};
+  std::string trace_path;              // copied at init: the caller's string need not outlive it
   strings::CoreConfig ccfg;
   int kl_mode = 0;                     // 0 persistent, 1 launch (profiling)
   std::vector<uint32_t> weights;       // DST weight per logical device
@@ -404,6 +405,8 @@ class Runtime : public strings::Hooks {
   // ------------------------------------------------------------ init/fini
   strings_status_t init(const strings_config_t* c) {
     if (c) cfg = *c;
+    trace_path = cfg.trace_path ? cfg.trace_path : "";
+    cfg.trace_path = nullptr;
     if (cfg.partitions <= 0) cfg.partitions = 2;
     if (cfg.awake_budget <= 0) cfg.awake_budget = 2 + cfg.partitions;
     if (cfg.admit_cap <= 0) cfg.admit_cap = 2 * cfg.awake_budget;
@@ -434,7 +437,7 @@ class Runtime : public strings::Hooks {
     ccfg.joint = cfg.joint_select;
     ccfg.Q = cfg.quantum_ns;
     ccfg.tfs_slice = cfg.tfs_slice_ns;
-    ccfg.record_trace = cfg.trace_in_memory || cfg.trace_path;
+    ccfg.record_trace = cfg.trace_in_memory || !trace_path.empty();
     weights.assign(cfg.num_gpus, 1);
     if (cfg.device_weights) {
       for (int g = 0; g < cfg.num_gpus; ++g) {
@@ -1245,8 +1248,8 @@ class Runtime : public strings::Hooks {
   }
 
   void flush_trace() {
-    if (!cfg.trace_path) return;
-    FILE* f = fopen(cfg.trace_path, "w");
+    if (trace_path.empty()) return;
+    FILE* f = fopen(trace_path.c_str(), "w");
     if (!f) return;
     fwrite(core->trace().data(), 1, core->trace().size(), f);
     fclose(f);
