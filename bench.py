@@ -62,6 +62,12 @@ def parse_args():
                    help="run BASELINE configs C1-C5 at full size (node mode, logical devices if G > GPUs)")
     p.add_argument("--fig2", action="store_true",
                    help="Fig. 2 analogue: N identical requests sequential vs co-resident vs separate contexts")
+    p.add_argument("--open-loop", action="store_true",
+                   help="C4 open loop: jobs submitted at their Eq. (4) arrival times; p50/p99 latency per "
+                   "priority class, LAS+GUF vs arrival-order GMin+FIFO; not the driver line")
+    p.add_argument("--open-loop-dilate", type=float, default=0.0,
+                   help="arrival-time dilation (0 = logical devices per physical GPU, so the offered load "
+                   "per physical host link is the config's rho)")
     p.add_argument("--sweep", action="store_true",
                    help="policy comparison on C2 (device policies x balancers) vs static; not the driver line")
     return p.parse_args()
@@ -787,8 +793,140 @@ def run_configs(args) -> None:
         del hin, hout
 
 
+def _pct(xs, q):
+    xs = sorted(xs)
+    return xs[min(len(xs) - 1, int(q * len(xs)))] if xs else None
+
+
+def open_loop(args) -> None:
+    """C4 as the open-loop system SURVEY §8(d) describes: 64 tenants whose jobs
+    arrive by Eq. (4) at offered load rho = 0.9 per device, skewed
+    priorities w = 8/4/2/1.  A submitter thread of this process calls
+    strings_submit at each job's arrival time (MEASURED timing, caller-pinned
+    buffers), so a job's latency is done - submit on the library clock.  On a box
+    with fewer GPUs than the config's 8 devices the arrival times are dilated by
+    the number of logical devices per GPU, which keeps the offered load per
+    physical host link at rho.  Two schedulers see the same arrivals:
+    the config's (weighted-LAS admission + GUF placement, LAS wake order) and an
+    arrival-order baseline (GMin placement, FIFO wake order).  Reported per
+    priority class: jobs, p50 / p99 / mean latency; plus jobs/s (bounded by the
+    arrival rate), T*/span with T* including the arrival-bound term, Jain, and
+    the submitter's lateness."""
+    import threading
+
+    import torch
+
+    import strings_workload as W
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+
+    ngpu = torch.cuda.device_count()
+    peaks = measured_peaks()
+    link = host_link_peaks(torch)
+    base = W.CONFIGS["C4"]()
+    lpg = max(1, (base.config.num_gpus + ngpu - 1) // ngpu)
+    dil = args.open_loop_dilate or float(lpg)
+    wl = dataclasses.replace(base, jobs=[dataclasses.replace(j, arrival_ns=int(j.arrival_ns * dil))
+                                         for j in base.jobs])
+    need_in, need_out = {}, {}
+    for sp in wl.jobs:
+        need_in[sp.tenant] = [max(a, b) for a, b in zip(need_in.get(sp.tenant, [0, 0]), (sp.h2d_sizes() + [0])[:2])]
+        need_out[sp.tenant] = max(need_out.get(sp.tenant, 0), sum(sp.d2h_sizes()))
+    hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
+    hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
+    refs = [([S.HostRef(hin[sp.tenant][i].data_ptr(), b) for i, b in enumerate(sp.h2d_sizes())],
+             [S.HostRef(hout[sp.tenant].data_ptr(), b) for b in sp.d2h_sizes()]) for sp in wl.jobs]
+    tstar, terms = tstar_device(wl, link, peaks["hbm_gbs"], peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"],
+                                kl_slots=lpg * wl.config.partitions)
+    variants = [("LAS admission + GUF / LAS (C4)", wl.config.resolved()),
+                ("arrival order + GMin / FIFO", dataclasses.replace(wl.config, balancer=W.GMIN, las_admission=0,
+                                                                    device_policy=W.FIFO).resolved())]
+    weight_of = {t: ten.weight for t, ten in enumerate(wl.tenants)}
+    # Third row: the same scheduler in INJECTED timing on the undilated arrivals --
+    # decisions in virtual time with the nominal per-device phase durations
+    # (SURVEY §8(d)), i.e. the latencies an 8-device box at nominal rates would
+    # see; every op still runs on the GPU.
+    variants.append(("LAS admission + GUF / LAS (C4), INJECTED virtual time, 8 devices at nominal rates",
+                     wl.config.resolved()))
+    for vi, (name, cfg) in enumerate(variants):
+        injected = vi == 2
+        run_wl = base if injected else wl
+        with ClockSampler(torch.cuda.current_device()) as clk:
+            S.init_from_config(cfg, timing_mode=S.INJECTED if injected else S.MEASURED, physical_gpus=ngpu,
+                               trace_in_memory=False)
+            ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+            late = []
+            ids = [None] * len(wl.jobs)
+
+            def submitter():
+                if injected:               # arrival_ns is virtual: submit everything, then drain
+                    for i, sp in enumerate(base.jobs):
+                        ids[i] = S.submit_spec(ts[sp.tenant], sp, refs[i][0], refs[i][1])
+                        late.append(0)
+                    return
+                t0 = time.perf_counter_ns()
+                for i, sp in enumerate(wl.jobs):
+                    due = t0 + sp.arrival_ns
+                    while time.perf_counter_ns() < due:
+                        pass
+                    late.append(time.perf_counter_ns() - due)
+                    ids[i] = S.submit_spec(ts[sp.tenant], sp, refs[i][0], refs[i][1])
+
+            th = threading.Thread(target=submitter)
+            th.start()
+            th.join()
+            st = S.drain()
+            infos = [S.job_info(j) for j in ids]
+            S.shutdown()
+        dump = os.environ.get("BENCH_OPEN_LOOP_DUMP")
+        if dump:                           # per-job records for offline analysis
+            with open(f"{dump}.{vi}.jsonl", "w") as f:
+                for sp, inf in zip(run_wl.jobs, infos):
+                    f.write(json.dumps({"tenant": sp.tenant, "cls": W.CLASS_NAMES[sp.kclass], "gid": inf.gid,
+                                        "arr": inf.t_arrival, "place": inf.t_place, "start": list(inf.t_start),
+                                        "done": list(inf.t_done)}) + "\n")
+        lat = {}
+        for sp, inf in zip(run_wl.jobs, infos):
+            lat.setdefault(weight_of[sp.tenant], []).append((inf.t_done[2] - inf.t_arrival) / 1e6)
+        per_class = {f"w={w}": {"jobs": len(v), "p50_ms": round(_pct(v, 0.5), 3), "p99_ms": round(_pct(v, 0.99), 3),
+                                "mean_ms": round(sum(v) / len(v), 3)} for w, v in sorted(lat.items(), reverse=True)}
+        busy, first, last = {}, {}, {}
+        for inf in infos:
+            busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
+            first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
+            last[inf.tenant] = max(last.get(inf.tenant, 0), inf.t_done[2])
+        xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
+        jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+        span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
+        print(json.dumps({"config": "C4 open loop", "scheduler": name, "status": st,
+                          "failed_jobs": sum(1 for i in infos if i.status != S.OK),
+                          "jobs": len(wl.jobs), "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
+                          "timing": "INJECTED (virtual)" if injected else "MEASURED",
+                          "arrival_dilation": 1.0 if injected else dil, "rho_per_device": 0.9,
+                          "jobs_per_s": round(len(wl.jobs) / span, 1), "span_ms": round(span * 1e3, 2),
+                          "last_arrival_ms": round(run_wl.jobs[-1].arrival_ns / 1e6, 2),
+                          "tstar_ms": None if injected else round(tstar * 1e3, 3),
+                          "roofline_frac": None if injected else round(tstar / span, 4),
+                          "tstar_terms_ms": None if injected else {k: round(v * 1e3, 3) for k, v in terms.items()},
+                          "latency_by_priority": per_class,
+                          "latency_all": {"p50_ms": round(_pct([x for v in lat.values() for x in v], 0.5), 3),
+                                          "p99_ms": round(_pct([x for v in lat.values() for x in v], 0.99), 3)},
+                          "jain_weighted_service": round(jain, 4),
+                          "submit_lateness_us": {"p50": round(_pct(late, 0.5) / 1e3, 1),
+                                                 "p99": round(_pct(late, 0.99) / 1e3, 1),
+                                                 "max": round(max(late) / 1e3, 1)},
+                          "clocks": clk.summary(),
+                          "note": "latency = JOB_DONE - arrival; priority class = tenant weight; " + (
+                              "virtual clock: each logical device has its own nominal engines" if injected else
+                              "logical devices share the physical GPU's host link and SMs"
+                              if cfg.num_gpus > ngpu else "one logical device per GPU")}), flush=True)
+    del hin, hout
+
+
 def main():
     args = parse_args()
+    if args.open_loop:
+        open_loop(args)
+        return
     if args.configs:
         run_configs(args)
         return

@@ -46,6 +46,7 @@ def main():
     ap.add_argument("--policy", default=None)
     ap.add_argument("--gpus", type=int, default=0, help="logical devices (0 = the config's)")
     ap.add_argument("--repeats", type=int, default=2)
+    ap.add_argument("--trace", default=None, help="write the last repeat's decision trace here")
     args = ap.parse_args()
     wl = W.CONFIGS[args.config]()
     cfg = wl.config
@@ -65,7 +66,8 @@ def main():
     hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
     hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
     for rep in range(args.repeats):
-        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
+        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False,
+                           trace_path=args.trace if rep == args.repeats - 1 else None)
         ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
         t0 = time.perf_counter()
         for sp in wl.jobs:
