@@ -170,14 +170,14 @@ def kernel_rooflines(torch, S, peaks) -> list:
     out = []
     st = torch.cuda.current_stream()
 
-    def time_launch(desc, ins, outs, iters=10):
-        S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs],
+    def time_launch(desc, ins, outs, iters=10, ctas=0):
+        S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], ctas=ctas,
                         stream=st.cuda_stream)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(st)
         for _ in range(iters):
-            S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs],
+            S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], ctas=ctas,
                             stream=st.cuda_stream)
         e1.record(st)
         torch.cuda.synchronize()
@@ -193,6 +193,30 @@ def kernel_rooflines(torch, S, peaks) -> list:
                     "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                     "frac": round(gbs / peaks["hbm_gbs"], 4), "ms": round(t * 1e3, 4)})
     del x, y
+    # the C2 work item's size on one P=2 partition: what the same body achieves as a
+    # stand-alone launch (the ceiling the dispatcher item is judged against)
+    n24 = 1 << 24
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    xs = [torch.randint(0, 1 << 30, (n24,), dtype=torch.int32, device="cuda") for _ in range(4)]
+    ys = [torch.empty_like(x) for x in xs]         # 4 rotating pairs: 512 MiB > L2
+    d24 = S.make_desc(S.XFER, n=n24, seed=7)
+    for ctas in (sms // 2, sms):
+        for i in range(4):
+            S.kernel_launch(0, d24, [xs[i].data_ptr()], [ys[i].data_ptr()], ctas=ctas, stream=st.cuda_stream)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        for i in range(20):
+            S.kernel_launch(0, d24, [xs[i % 4].data_ptr()], [ys[i % 4].data_ptr()], ctas=ctas,
+                            stream=st.cuda_stream)
+        e1.record(st)
+        torch.cuda.synchronize()
+        t = e0.elapsed_time(e1) / 1e3 / 20
+        gbs = 8 * n24 / t / 1e9
+        out.append({"kernel": "XFER", "bound": "hbm", "size": f"n=2^24 (128 MiB moved) on {ctas} CTAs",
+                    "ctas": ctas, "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                    "frac": round(gbs / peaks["hbm_gbs"], 4), "ms": round(t * 1e3, 4)})
+    del xs, ys
     m, nn, k, reps = 128 * 148, 256, 256, 64
     a = torch.randint(-2, 3, (m, k), device="cuda").to(torch.bfloat16)
     b = torch.randint(-2, 3, (k, nn), device="cuda").to(torch.bfloat16)
@@ -422,7 +446,7 @@ def run_strings(args, rank, world, torch, gloo):
                      "unit": "GB/s", "frac": round(link_gbs / link["bidir_gbs"], 4), "traffic": None,
                      "resource": "copy engines H2D+D2H (the step's dominant resource)",
                      "peak_source": "measured in this run: concurrent pinned H2D+D2H cudaMemcpyAsync 256 MiB"},
-        "roofline_kernel": _kernel_roofline(kl_lat, wl, peaks),
+        "roofline_kernel": _kernel_roofline(kl_lat, wl, peaks, krl),
         "overlapped_roofline": {"tstar_ms": round(tstar * 1e3, 3), "span_ms": round(span_step * 1e3, 3),
                                 "frac": round(tstar / span_step, 4),
                                 "terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()}},
@@ -453,23 +477,42 @@ def run_strings(args, rank, world, torch, gloo):
     return res, wl
 
 
-def _kernel_roofline(kl_lat, wl, peaks) -> dict:
+def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
     """The dominant kernel work inside the timed step: XFER items run by the
     persistent dispatcher on one P=2 SM partition (74 SMs), HBM-bound.
     achieved = algorithmic bytes per item (read + write) / median device time
-    of the item (%globaltimer claim -> last CTA done)."""
+    of the item (%globaltimer claim -> last CTA done).  Beside it: the same body
+    launched stand-alone on the same CTA count at the same size (measured in
+    this run, kernel_rooflines) -- a 128 MiB pass on 74 SMs does not reach the
+    2 GiB full-GPU rate -- and the ncu DRAM traffic of that launch."""
     import strings_workload as W
     x = kl_lat.get("XFER")
     n = [j for j in wl.jobs if j.kclass == W.XFER][0].n
     if not x:
         return None
     gbs = 8 * n / (x["kl_device_us_p50"] * 1e3)
-    return {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline)", "bound": "hbm",
-            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
-            "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": None,
-            "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (74 of 148 SMs); the other "
-            "partition often runs an item concurrently and shares HBM; device time includes the partition "
-            "broadcast and completion publish (stand-alone full-GPU runs: kernel_rooflines)"}
+    out = {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline)", "bound": "hbm",
+           "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+           "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": _XFER_ITEM_NCU["dram_bytes"],
+           "traffic_source": _XFER_ITEM_NCU["source"],
+           "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (74 of 148 SMs); the other "
+           "partition often runs an item concurrently and shares HBM; device time includes the partition "
+           "broadcast and completion publish (stand-alone full-GPU runs: kernel_rooflines)"}
+    same = sorted((k for k in (krl or []) if k.get("ctas") and k["kernel"] == "XFER"), key=lambda k: k["ctas"])
+    if same:
+        out["same_work_standalone"] = {"ctas": same[0]["ctas"], "GBps": same[0]["achieved"],
+                                       "us": round(same[0]["ms"] * 1e3, 2),
+                                       "item_vs_standalone": round(gbs / same[0]["achieved"], 4)}
+    return out
+
+
+# ncu --set full of the C2 work item's body as a stand-alone launch (XFER 2^24 u32
+# on 74 CTAs, `tools/kernel_probe.py xfer_item`): dram__bytes_read.sum +
+# dram__bytes_write.sum per launch; see profiles/r01_kernels.md.
+# Reads 67.18 MB = the 64 MiB input exactly; writes 20.27 MB of 67.1 MB: at this size
+# most of the output is still in the 126 MB L2 when the launch ends (no re-reads).
+_XFER_ITEM_NCU = {"dram_bytes": 67181056 + 20273664,
+                  "source": "profiles/r01_kernels.md (xfer_item: ncu --set full, XFER 2^24 on 74 CTAs)"}
 
 
 def max_over(gloo, x: float) -> float:

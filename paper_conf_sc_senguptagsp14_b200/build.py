@@ -16,6 +16,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-Wall,-Wno-unused-function",
          "-I", os.path.join(ROOT, "include"), "--expt-relaxed-constexpr"]
+# experiments only (e.g. STRINGS_NVCC_EXTRA="-DSTRINGS_STREAM_STAGES=6 -DSTRINGS_STREAM_CHUNK_KB=32")
+FLAGS += os.environ.get("STRINGS_NVCC_EXTRA", "").split()
 
 
 def _stale() -> bool:

@@ -123,8 +123,15 @@ __device__ void stream_ldg(const uint32_t* __restrict__ x, uint32_t* __restrict_
   for (uint64_t e = e0 + nvec * 4 + tid; e < e1; e += nthreads) y[e] = elem_op<KCLASS>(x[e], alpha, seed);
 }
 
-constexpr int kStreamStages = 4;
-constexpr uint32_t kStreamChunk = 48 * 1024;             // bytes per stage (4 x 48 KB = 192 KB)
+#ifndef STRINGS_STREAM_STAGES
+#define STRINGS_STREAM_STAGES 4
+#endif
+#ifndef STRINGS_STREAM_CHUNK_KB
+#define STRINGS_STREAM_CHUNK_KB 48
+#endif
+constexpr int kStreamStages = STRINGS_STREAM_STAGES;                 // stage count (<= 12 mbarriers in the tail)
+constexpr uint32_t kStreamChunk = STRINGS_STREAM_CHUNK_KB * 1024;    // bytes per stage (4 x 48 KB = 192 KB)
+static_assert(kStreamStages >= 3 && kStreamStages <= 12, "stream stages");
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(
@@ -218,7 +225,8 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
 constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
 constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
 constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
-constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 64;     // + mbarriers / tmem slot (tail, see carve_smem)
+constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 128;    // + mbarriers / tmem slot (tail, see carve_smem)
+static_assert(kStreamStages * kStreamChunk <= kSmemA + kSmemB, "streaming stages alias the GEMM operand smem");
 constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
 constexpr uint32_t kSlabA = 128 * 128;                   // 16 KB
 constexpr uint32_t kSlabB = 256 * 128;                   // 32 KB
@@ -597,7 +605,7 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
   }
 }
 
-// smem: [A 64 KB][B 128 KB][tail 64 B: GEMM mbarrier @0, TMEM slot @8, 4 stream mbarriers @16..48]
+// smem: [A 64 KB][B 128 KB][tail 128 B: GEMM mbarrier @0, TMEM slot @8, <= 14 stream/fill mbarriers @16..]
 __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   GemmSmem s;
   s.a = base;

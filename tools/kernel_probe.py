@@ -3,7 +3,8 @@
     ncu --set full --clock-control none --import-source on -k regex:oneshot -c 6 \
         -o gpurun_out/prof python tools/kernel_probe.py
 
-Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2).
+Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2);
+`xfer_item`: XFER n=2^24 on 74 CTAs (x2), the C2 work item on one P=2 partition.
 The persistent dispatcher runs exactly these device bodies on its SM partitions.
 """
 import os
@@ -28,6 +29,16 @@ def main():
                 for _ in range(2):
                     S.kernel_launch(0, S.make_desc(cls, n=n, alpha=1.001, seed=7), [x.data_ptr()], [y.data_ptr()],
                                     stream=st)
+        torch.cuda.synchronize()
+        del x, y
+    if "xfer_item" in which:
+        # the C2 work item as the dispatcher runs it: XFER 2^24 u32 on a 74-SM partition
+        n24 = 1 << 24
+        x = torch.randint(0, 1 << 30, (n24,), dtype=torch.int32, device="cuda")
+        y = torch.empty_like(x)
+        for _ in range(2):
+            S.kernel_launch(0, S.make_desc(S.XFER, n=n24, seed=7), [x.data_ptr()], [y.data_ptr()], ctas=74,
+                            stream=st)
         torch.cuda.synchronize()
         del x, y
     if "gemm" in which:
