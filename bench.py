@@ -432,13 +432,7 @@ def run_strings(args, rank, world, torch, gloo):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt_max / args.steps * 1e3, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16/f32/u32",
         "data": "synthetic (seeded; strings_workload)",
-        "config": {"workload": "C2: 16 tenants (8 GEMM 256^3 R=64, 8 XFER 2^24 u32) x 8 jobs, 1 B200 per rank, "
-                               "DTF joint placement, PS dispatch, measured timing",
-                   "jobs_per_step_per_gpu": jobs_step, "partitions": cfg.partitions,
-                   "awake_budget": cfg.awake_budget, "admit_cap": cfg.admit_cap,
-                   "l2": "inputs larger than L2 (4 GiB H2D + 4 GiB D2H per step)",
-                   "kl_mode": "persistent dispatcher" if args.kl_mode == 0 else "per-job launches",
-                   "parallelism": f"placement only, {world} rank(s) x 1 GPU"},
+        "config": arm_config(cfg, jobs_step, world, args.kl_mode),
         "continuous": {"value": round(jobs_step * args.steps * world / dt_cont, 3), "unit": "jobs/s",
                        "frac_host_link": round(moved * args.steps / dt_cont / 1e9 / link["bidir_gbs"], 4),
                        "note": "same K batches submitted back to back, one drain (no per-step fill/drain)"},
@@ -475,6 +469,17 @@ def run_strings(args, rank, world, torch, gloo):
         with open(args.trace_out, "w") as f:
             f.write("\n".join(trace) + "\n")
     return res, wl
+
+
+def arm_config(cfg, jobs_step: int, world: int, kl_mode: int) -> dict:
+    """The `config` object of the JSON line (both arms print the same one)."""
+    return {"workload": "C2: 16 tenants (8 GEMM 256^3 R=64, 8 XFER 2^24 u32) x 8 jobs, 1 B200 per rank, "
+                        "DTF joint placement, PS dispatch, measured timing",
+            "jobs_per_step_per_gpu": jobs_step, "partitions": cfg.partitions,
+            "awake_budget": cfg.awake_budget, "admit_cap": cfg.admit_cap,
+            "l2": "inputs larger than L2 (4 GiB H2D + 4 GiB D2H per step)",
+            "kl_mode": "persistent dispatcher" if kl_mode == 0 else "per-job launches",
+            "parallelism": f"placement only, {world} rank(s) x 1 GPU"}
 
 
 def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
@@ -600,7 +605,9 @@ def run_reference(args):
             "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64/f32/u32 (numpy)", "data": "synthetic",
             "impl": "reference",
-            "config": {"workload": "C2 (16 tenants, 8 GEMM 256^3 R=64 + 8 XFER 2^24), oracle on the host"},
+            "config": arm_config(wl.config.resolved(), len(wl.jobs), args.gpus, args.kl_mode),
+            "reference_note": "the oracle (oracle/, plain numpy, one host core) runs the same C2 jobs: copy-in, "
+                              "CPU kernel, copy-out; each step times a 16-job sample (one job per tenant)",
             "cpu_baseline": {"value": v, "unit": "jobs/s", "cores": 1, "kind": "oracle",
                              "sample": "16 jobs of C2 per step (one per tenant)"},
             "e2e": {"value": v, "unit": "jobs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
