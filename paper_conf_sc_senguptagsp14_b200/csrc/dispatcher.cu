@@ -201,8 +201,14 @@ cudaError_t launch_dispatcher(const strings_dev::DispatchParams& p, int grid, cu
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)strings_dev::kSmemGemm);
   if (e != cudaSuccess) return e;
-  strings_dev::dispatcher_kernel<<<grid, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(p);
-  return cudaGetLastError();
+  // Every CTA must be resident at once (partition leaders and followers poll each
+  // other, and the last CTA of a partition completes its item): a cooperative
+  // launch guarantees co-residency or fails, instead of hanging when other work
+  // holds some SMs at launch time.
+  strings_dev::DispatchParams arg = p;
+  void* args[] = {&arg};
+  return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(strings_dev::dispatcher_kernel), dim3(grid),
+                                     dim3(strings_dev::kThreads), args, strings_dev::kSmemGemm, s);
 }
 
 cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaStream_t s) {
