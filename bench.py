@@ -80,8 +80,8 @@ class ClockSampler:
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, index: int):
-        self.index = index
+    def __init__(self, index):
+        self.index = index                 # nvidia-smi --id (index, bus id or UUID)
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         self.p = None
 
@@ -320,7 +320,9 @@ def run_strings(args, rank, world, torch, gloo):
     trace_start = len(S.trace()) if args.trace_out else 0
     gloo_barrier(gloo)
     stream.synchronize()
-    with ClockSampler(int(os.environ.get("LOCAL_RANK", 0)) if world > 1 else 0) as clk:
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    gpu_id = par.physical_gpu(par.rank_info())      # nvidia-smi id of this rank's GPU
+    with ClockSampler(gpu_id) as clk:
         ev0.record(stream)
         t_wall = time.perf_counter()
         for _ in range(args.steps):
@@ -479,7 +481,9 @@ def arm_config(cfg, jobs_step: int, world: int, kl_mode: int) -> dict:
             "awake_budget": cfg.awake_budget, "admit_cap": cfg.admit_cap,
             "l2": "inputs larger than L2 (4 GiB H2D + 4 GiB D2H per step)",
             "kl_mode": "persistent dispatcher" if kl_mode == 0 else "per-job launches",
-            "parallelism": f"placement only, {world} rank(s) x 1 GPU"}
+            "parallelism": f"placement only, {world} rank(s) x 1 GPU" + (
+                " (TEST MODE: all ranks share one GPU, SM-limited dispatchers; not a reported number)"
+                if os.environ.get("STRINGS_BENCH_SHARE_GPU") == "1" else "")}
 
 
 def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:

@@ -484,6 +484,10 @@ class Runtime : public strings::Hooks {
       cudaDeviceProp prop;
       if (!cuda_ok(cudaGetDeviceProperties(&prop, ph->dev))) return STRINGS_ECUDA;
       ph->sms = prop.multiProcessorCount;
+      // test knob: run the dispatcher on fewer SMs (e.g. two library instances
+      // sharing one GPU to exercise the multi-rank bench path on a 1-GPU box)
+      if (const char* lim = getenv("STRINGS_SM_LIMIT"))
+        if (atoi(lim) > 0) ph->sms = std::min(ph->sms, atoi(lim));
       if (ph->L * cfg.partitions > ph->sms) return STRINGS_EINVAL;
       // SM shares: logical devices of this GPU get CTAs in proportion to their
       // weights, each share split evenly into P partitions (one per KL slot)

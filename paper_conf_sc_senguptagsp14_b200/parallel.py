@@ -34,9 +34,34 @@ def rank_info() -> RankInfo:
 
 
 def isolate_gpu(info: RankInfo) -> None:
-    """Make this rank's GPU the only visible one (must run before CUDA init)."""
+    """Make this rank's GPU the only visible one (must run before CUDA init).
+    The rank takes the local_rank-th entry of an inherited CUDA_VISIBLE_DEVICES
+    list (so a launcher that hands out e.g. "4,5,6,7" is respected), else the
+    device with index local_rank."""
     if info.world > 1:
-        os.environ["CUDA_VISIBLE_DEVICES"] = str(info.local_rank)
+        os.environ["CUDA_VISIBLE_DEVICES"] = physical_gpu(info)
+        if shared_gpu_test():
+            # every rank on the first device, each dispatcher on its own share of the SMs
+            os.environ.setdefault("STRINGS_SM_LIMIT", str(148 // info.world))
+
+
+def shared_gpu_test() -> bool:
+    """STRINGS_BENCH_SHARE_GPU=1: all ranks share the first visible GPU (a test of
+    the multi-rank plumbing on a 1-GPU box; NCCL refuses two ranks per device, so
+    the default group is gloo).  Never used for reported numbers."""
+    return os.environ.get("STRINGS_BENCH_SHARE_GPU") == "1"
+
+
+def physical_gpu(info: RankInfo) -> str:
+    """The device id this rank uses, as the launcher numbers devices."""
+    vis = [d.strip() for d in os.environ.get("STRINGS_INHERITED_CVD", os.environ.get("CUDA_VISIBLE_DEVICES", ""))
+           .split(",") if d.strip()]
+    os.environ.setdefault("STRINGS_INHERITED_CVD", ",".join(vis))
+    if shared_gpu_test():
+        return vis[0] if vis else "0"
+    if vis and info.local_rank < len(vis):
+        return vis[info.local_rank]
+    return str(info.local_rank)
 
 
 def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl"):
@@ -46,7 +71,7 @@ def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl"):
         return None
     import torch
     import torch.distributed as dist
-    if device_backend == "nccl" and torch.cuda.is_available():
+    if device_backend == "nccl" and torch.cuda.is_available() and not shared_gpu_test():
         torch.cuda.set_device(0)
         dist.init_process_group("nccl", device_id=torch.device("cuda:0"))
         return dist.new_group(backend="gloo")
