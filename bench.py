@@ -291,16 +291,20 @@ def run_strings(args, rank, world, torch, gloo):
     if args.balancer >= 0:
         wl.config.balancer = args.balancer
     cfg = wl.config.resolved()
-    # inputs resident in pinned host memory before timing (the H2D phase is part of the job, S4)
-    ins, outs = [], []
+    # inputs resident in pinned host memory before timing (the H2D phase is part of the job, S4).
+    # One input and one output set per tenant, shared by the tenant's jobs: c_t = 1, so a
+    # tenant's jobs never overlap, and every job still moves its own bytes each way
+    # (1.1 GB of host buffers per rank instead of 8.6 GB; output parity of this configuration
+    # with per-job inputs is checked by tests/test_gpu_scheduler.py).
+    per_tenant = {}
     for spec in wl.jobs:
-        src = W.job_inputs(spec)
-        pins = []
-        for a in src:
-            p = torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory()
-            pins.append(p)
-        ins.append(pins)
-        outs.append([torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
+        if spec.tenant not in per_tenant:
+            per_tenant[spec.tenant] = (
+                [torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory() for a in W.job_inputs(spec)],
+                [torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
+    assert all(t.max_inflight == 1 for t in wl.tenants)
+    ins = [per_tenant[spec.tenant][0] for spec in wl.jobs]
+    outs = [per_tenant[spec.tenant][1] for spec in wl.jobs]
     arenas = S.torch_arenas(cfg.num_gpus, 1, cfg.admit_cap)      # PyTorch provides the device memory
     S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1, kl_mode=args.kl_mode,
                        trace_in_memory=bool(args.trace_out), arenas=arenas)
@@ -352,8 +356,10 @@ def run_strings(args, rank, world, torch, gloo):
     # (pageable) numpy arrays: the library stages them through its pinned PMT
     # (MOT) and copies results back into the caller's arrays.
     if not args.no_e2e:
-        np_ins = [[a.numpy().copy() for a in row] for row in ins]
-        np_outs = [[np.empty(o.numel(), dtype=np.uint8) for o in row] for row in outs]
+        np_t = {t: ([a.numpy().copy() for a in i], [np.empty(o.numel(), dtype=np.uint8) for o in o_])
+                for t, (i, o_) in per_tenant.items()}
+        np_ins = [np_t[spec.tenant][0] for spec in wl.jobs]
+        np_outs = [np_t[spec.tenant][1] for spec in wl.jobs]
         for i, spec in enumerate(wl.jobs):          # warm the staging pool once
             S.submit_spec(tenants[spec.tenant], spec, np_ins[i], np_outs[i])
         assert S.drain() == S.OK
