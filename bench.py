@@ -1004,10 +1004,12 @@ def main():
             run_reference(args)
         return
     par.isolate_gpu(info)                 # one process per GPU (before CUDA init)
+    numa = par.bind_to_gpu_numa_node(par.physical_gpu(info))
     import torch
     gloo = par.init_groups(info, device_backend="nccl")
     res, wl = run_strings(args, rank, world, torch, gloo)
     if rank == 0:
+        res["config"]["host_numa"] = numa
         if world == 1 and not args.no_static:
             from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
             sb = run_static(wl, num_gpus=1, repeats=args.static_repeats)

@@ -64,6 +64,36 @@ def physical_gpu(info: RankInfo) -> str:
     return str(info.local_rank)
 
 
+def bind_to_gpu_numa_node(gpu_id: str) -> dict:
+    """Restrict this process (and the library threads it will start) to the CPUs
+    of the NUMA node the GPU hangs off, so pinned buffers are first-touched on
+    that node and the copy engines DMA without crossing the socket link (SURVEY
+    §8(e): host DRAM and PCIe root complexes are shared).  No-op when the node
+    cannot be determined; returns what was done."""
+    import subprocess
+    try:
+        bus = subprocess.run(["nvidia-smi", f"--id={gpu_id}", "--query-gpu=pci.bus_id", "--format=csv,noheader"],
+                             capture_output=True, text=True, timeout=30).stdout.strip().splitlines()[0]
+        dom, rest = bus.split(":", 1)
+        sysfs = f"/sys/bus/pci/devices/{dom[-4:]}:{rest}".lower()
+        with open(sysfs + "/local_cpulist") as f:
+            spec = f.read().strip()
+        with open(sysfs + "/numa_node") as f:
+            node = int(f.read().strip())
+        cpus = set()
+        for part in spec.split(","):
+            a, _, b = part.partition("-")
+            cpus.update(range(int(a), int(b or a) + 1))
+        allowed = os.sched_getaffinity(0)
+        use = cpus & allowed
+        if not use or use == allowed:
+            return {"numa_node": node, "cpus": len(allowed), "bound": False}
+        os.sched_setaffinity(0, use)
+        return {"numa_node": node, "cpus": len(use), "bound": True}
+    except Exception as e:  # noqa: BLE001 - best effort
+        return {"bound": False, "why": type(e).__name__}
+
+
 def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl"):
     """Default process group (NCCL when a GPU is present) plus a gloo group for
     host-side coordination.  Returns the gloo group (None for world == 1)."""
