@@ -245,3 +245,27 @@ def test_device_fault_fails_tenants_instead_of_hanging(tmp_path):
     assert line, p.stdout + p.stderr
     f = line[0].split()
     assert int(f[1]) == S.ECUDA and int(f[3]) != 0 and float(f[5]) < 30
+
+
+def test_job_exactly_filling_its_slot():
+    # maximum size: one XFER job of 2^26 u32 (256 MiB in + 256 MiB out) in a slot of
+    # exactly 512 MiB runs and is exact on sampled elements; 4 more bytes of input
+    # do not fit and are rejected at submit (EINVAL), with nothing queued
+    n = 1 << 26
+    wl = W.Workload("max-slot", W.SystemConfig(num_gpus=1, device_policy=W.PS), [W.TenantSpec()],
+                    [W.JobSpec(tenant=0, kclass=W.XFER, n=n, seed=0x9E3779B9, data_seed=5)])
+    r = run_workload(wl, timing_mode=S.MEASURED, slot_bytes=8 * n, keep_inputs=True)
+    assert r.status == S.OK
+    x, y = r.inputs[0][0], r.outputs[0][0]
+    rng = np.random.default_rng(3)
+    idx = np.concatenate([np.arange(64), n - 1 - np.arange(64), rng.integers(0, n, 1 << 16)])
+    assert np.array_equal(y[idx], K.xfer(x[idx], wl.jobs[0].seed))
+    S.init(num_gpus=1, timing_mode=S.MEASURED, slot_bytes=8 * n, physical_gpus=1)
+    try:
+        t = S.register_tenant()
+        with pytest.raises(S.StringsError) as e:
+            S.submit(t, S.make_desc(S.XFER, n=n + 1), [S.HostRef(1, 4 * (n + 1))], [S.HostRef(1, 4 * (n + 1))])
+        assert e.value.status == S.EINVAL
+        assert S.drain() == S.OK and S.stats().jobs_submitted == 0
+    finally:
+        S.shutdown()
