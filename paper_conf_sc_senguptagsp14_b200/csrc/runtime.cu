@@ -14,6 +14,7 @@
 //   poisons that GPU's tenants (STRINGS_ECUDA at sync) instead of hanging.
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <emmintrin.h>
 #include <time.h>
 #include <unistd.h>
 
@@ -230,6 +231,47 @@ struct Phys {
   std::vector<cudaEvent_t> ev_pool;
 };
 
+// One part of a PMT staging copy.  Large parts use non-temporal stores
+// (SSE2 movntdq, then sfence before the part counts as done): a regular store
+// first reads the destination line from DRAM (read-for-ownership), so a copy
+// costs 3 bytes of host-DRAM traffic per byte instead of 2, and the e2e
+// (pageable) path is host-DRAM bound.  The staged bytes are read
+// next by the copy engine or the caller, never by this thread, so caching them
+// buys nothing.  STRINGS_NT_COPY=0 keeps plain memcpy.
+bool nt_copy_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("STRINGS_NT_COPY");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+void pmt_copy_part(void* dst, const void* src, uint64_t n) {
+  if (n < (256u << 10) || !nt_copy_enabled()) {
+    memcpy(dst, src, n);
+    return;
+  }
+  char* d = static_cast<char*>(dst);
+  const char* s = static_cast<const char*>(src);
+  const uint64_t head = (uint64_t)(-(uintptr_t)d) & 63;   // n >= 256 KiB > head
+  memcpy(d, s, head);
+  d += head;
+  s += head;
+  n -= head;
+  for (uint64_t i = 0, nv = n / 64; i < nv; ++i, d += 64, s += 64) {
+    const __m128i a = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s));
+    const __m128i b = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 16));
+    const __m128i c = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 32));
+    const __m128i e = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 48));
+    _mm_stream_si128(reinterpret_cast<__m128i*>(d), a);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 16), b);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 32), c);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 48), e);
+  }
+  memcpy(d, s, n & 63);
+  _mm_sfence();                                  // NT stores visible before the part is reported done
+}
+
 // Parallel host memcpy for PMT staging (one host thread copies ~6-10 GB/s;
 // a 64 MiB pageable buffer is split over a small worker pool).
 class CopyPool {
@@ -248,7 +290,7 @@ class CopyPool {
   void copy(void* dst, const void* src, uint64_t bytes) {
     constexpr uint64_t kChunk = 4ull << 20;
     if (bytes <= kChunk || th_.empty()) {
-      memcpy(dst, src, bytes);
+      pmt_copy_part(dst, src, bytes);
       return;
     }
     uint64_t parts = std::min<uint64_t>((bytes + kChunk - 1) / kChunk, th_.size() + 1);
@@ -264,7 +306,7 @@ class CopyPool {
       for (auto& t : tasks) q_.push_back(t);
     }
     cv_.notify_all();
-    memcpy(dst, src, std::min(per, bytes));        // the caller copies the first part
+    pmt_copy_part(dst, src, std::min(per, bytes));   // the caller copies the first part
     while (left.load(std::memory_order_acquire) > 0) std::this_thread::yield();
   }
 
@@ -283,7 +325,7 @@ class CopyPool {
       Task t = q_.front();
       q_.pop_front();
       lk.unlock();
-      memcpy(t.dst, t.src, t.n);
+      pmt_copy_part(t.dst, t.src, t.n);
       t.left->fetch_sub(1, std::memory_order_release);
       lk.lock();
     }

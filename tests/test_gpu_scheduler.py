@@ -184,6 +184,25 @@ def test_pageable_buffers_are_staged():
     check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("n", [65_537, 1_000_003, 6_000_011])
+def test_pageable_misaligned_ragged_buffers(n):
+    # PMT staging of pageable arrays that start off any 16/64-B boundary and end
+    # on a ragged tail: the staging copy (one part, or split over the copy pool,
+    # non-temporal stores above 256 KiB) and the copy-back must be exact
+    S.init(num_gpus=1, physical_gpus=1)
+    try:
+        t = S.register_tenant()
+        rng = np.random.default_rng(n)
+        xs = rng.integers(0, 1 << 32, n + 1, dtype=np.uint32)[1:]      # 4 B past the allocation start
+        ys = np.zeros(n + 3, np.uint32)[3:]
+        assert xs.ctypes.data % 16 and ys.ctypes.data % 16
+        S.submit(t, S.make_desc(S.XFER, n=n, seed=77), [xs], [ys])
+        assert S.sync(t) == S.OK
+        assert np.array_equal(ys, K.xfer(xs, 77))
+    finally:
+        S.shutdown()
+
+
 def test_full_size_c2_measured_sampled_parity():
     # BASELINE configs[1] at full size, in the launch configuration bench.py
     # times (MEASURED, persistent dispatcher): every GEMM output in full, XFER
