@@ -14,7 +14,7 @@
 //   poisons that GPU's tenants (STRINGS_ECUDA at sync) instead of hanging.
 #include <cuda.h>
 #include <cuda_runtime.h>
-#include <emmintrin.h>
+#include <immintrin.h>
 #include <time.h>
 #include <unistd.h>
 
@@ -232,22 +232,62 @@ struct Phys {
 };
 
 // One part of a PMT staging copy.  Large parts use non-temporal stores
-// (SSE2 movntdq, then sfence before the part counts as done): a regular store
-// first reads the destination line from DRAM (read-for-ownership), so a copy
-// costs 3 bytes of host-DRAM traffic per byte instead of 2, and the e2e
+// (movntdq / vmovntdq, then sfence before the part counts as done): a regular
+// store first reads the destination line from DRAM (read-for-ownership), so a
+// copy costs 3 bytes of host-DRAM traffic per byte instead of 2, and the e2e
 // (pageable) path is host-DRAM bound.  The staged bytes are read
 // next by the copy engine or the caller, never by this thread, so caching them
-// buys nothing.  STRINGS_NT_COPY=0 keeps plain memcpy.
-bool nt_copy_enabled() {
-  static const bool on = [] {
-    const char* e = getenv("STRINGS_NT_COPY");
-    return !(e && e[0] == '0');
+// buys nothing.  STRINGS_NT_COPY selects the loop: 0 = plain memcpy, 1 = SSE2
+// (default), 2 = AVX2, 3 = AVX-512.  The wider loops copy faster in isolation
+// (tools/host_ntcopy_probe.cpp) but lose in the e2e path on the B200 host
+// (SSE2 747, AVX2 642, AVX-512 345-591 jobs/s; profiles/r01_ntcopy.jsonl).
+__attribute__((target("avx2"))) void nt_loop_avx2(char* d, const char* s, uint64_t nv) {
+  for (uint64_t i = 0; i < nv; ++i, d += 128, s += 128) {
+    const __m256i a = _mm256_loadu_si256(reinterpret_cast<const __m256i*>(s));
+    const __m256i b = _mm256_loadu_si256(reinterpret_cast<const __m256i*>(s + 32));
+    const __m256i c = _mm256_loadu_si256(reinterpret_cast<const __m256i*>(s + 64));
+    const __m256i e = _mm256_loadu_si256(reinterpret_cast<const __m256i*>(s + 96));
+    _mm256_stream_si256(reinterpret_cast<__m256i*>(d), a);
+    _mm256_stream_si256(reinterpret_cast<__m256i*>(d + 32), b);
+    _mm256_stream_si256(reinterpret_cast<__m256i*>(d + 64), c);
+    _mm256_stream_si256(reinterpret_cast<__m256i*>(d + 96), e);
+  }
+}
+
+__attribute__((target("avx512f"))) void nt_loop_avx512(char* d, const char* s, uint64_t nv) {
+  for (uint64_t i = 0; i < nv; ++i, d += 128, s += 128) {
+    const __m512i a = _mm512_loadu_si512(s);
+    const __m512i b = _mm512_loadu_si512(s + 64);
+    _mm512_stream_si512(reinterpret_cast<__m512i*>(d), a);
+    _mm512_stream_si512(reinterpret_cast<__m512i*>(d + 64), b);
+  }
+}
+
+void nt_loop_sse2(char* d, const char* s, uint64_t nv) {
+  for (uint64_t i = 0; i < nv; ++i, d += 128, s += 128) {
+    __m128i v[8];
+    for (int k = 0; k < 8; ++k) v[k] = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 16 * k));
+    for (int k = 0; k < 8; ++k) _mm_stream_si128(reinterpret_cast<__m128i*>(d + 16 * k), v[k]);
+  }
+}
+
+using NtLoop = void (*)(char*, const char*, uint64_t);
+NtLoop nt_loop() {
+  static const NtLoop f = []() -> NtLoop {
+    int want = 1;
+    if (const char* e = getenv("STRINGS_NT_COPY")) want = atoi(e);
+    __builtin_cpu_init();
+    if (want >= 3 && __builtin_cpu_supports("avx512f")) return nt_loop_avx512;
+    if (want >= 2 && __builtin_cpu_supports("avx2")) return nt_loop_avx2;
+    if (want >= 1) return nt_loop_sse2;
+    return nullptr;
   }();
-  return on;
+  return f;
 }
 
 void pmt_copy_part(void* dst, const void* src, uint64_t n) {
-  if (n < (256u << 10) || !nt_copy_enabled()) {
+  const NtLoop loop = nt_loop();
+  if (n < (256u << 10) || !loop) {
     memcpy(dst, src, n);
     return;
   }
@@ -258,17 +298,8 @@ void pmt_copy_part(void* dst, const void* src, uint64_t n) {
   d += head;
   s += head;
   n -= head;
-  for (uint64_t i = 0, nv = n / 64; i < nv; ++i, d += 64, s += 64) {
-    const __m128i a = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s));
-    const __m128i b = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 16));
-    const __m128i c = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 32));
-    const __m128i e = _mm_loadu_si128(reinterpret_cast<const __m128i*>(s + 48));
-    _mm_stream_si128(reinterpret_cast<__m128i*>(d), a);
-    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 16), b);
-    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 32), c);
-    _mm_stream_si128(reinterpret_cast<__m128i*>(d + 48), e);
-  }
-  memcpy(d, s, n & 63);
+  loop(d, s, n / 128);                           // 64-B aligned destination, 128 B per iteration
+  memcpy(d + (n & ~uint64_t(127)), s + (n & ~uint64_t(127)), n & 127);
   _mm_sfence();                                  // NT stores visible before the part is reported done
 }
 
