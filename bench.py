@@ -462,7 +462,10 @@ def run_strings(args, rank, world, torch, gloo):
         "gpu_launches_note": "KL work items executed by the persistent dispatcher kernel (launched once at init)"
                              if args.kl_mode == 0 else "per-job tenant kernel launches",
         "clocks": clk.summary(),
-        "decisions_per_step": (stats.decisions // (args.warmup + args.steps)),
+        "decisions_per_step": (stats.decisions // (args.warmup + 2 * args.steps)),   # warm-up + timed + continuous
+        "sm_copy_ops_per_step": (stats.sm_copy_ops // (args.warmup + 2 * args.steps)),
+        "sm_copy_note": "H2D/D2H ops of small jobs served by the dispatcher's copy partition (zero-copy SM "
+                        "copies over PCIe) instead of the copy engines",
         "decision_us_per_job": round((stats.decision_ns - stats.issue_ns) / 1e3 / max(1, stats.jobs_done), 3),
         "issue_us_per_job": round(stats.issue_ns / 1e3 / max(1, stats.jobs_done), 3),
         "decision_note": "engine-thread time per job: decision core (placement, wake/start passes, epochs, "
@@ -806,6 +809,7 @@ def run_configs(args) -> None:
             st = S.drain()
             wall = time.perf_counter() - t0
             infos = [S.job_info(i) for i in range(len(wl.jobs))]
+            sm_ops = S.stats().sm_copy_ops
             S.shutdown()
             if rep == 0:
                 continue                    # warm-up
@@ -817,7 +821,7 @@ def run_configs(args) -> None:
             xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
             jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
             span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
-            runs.append({"span": span, "wall": wall, "jain": jain, "status": st,
+            runs.append({"span": span, "wall": wall, "jain": jain, "status": st, "sm_copy_ops": sm_ops,
                          "failed": sum(1 for i in infos if i.status != S.OK)})
         # arrivals are submit times in MEASURED mode: the whole config is offered at t = 0
         wl0 = dataclasses.replace(wl, jobs=[dataclasses.replace(j, arrival_ns=0) for j in wl.jobs])
@@ -837,7 +841,7 @@ def run_configs(args) -> None:
                           "jobs_per_s": round(len(wl.jobs) / span, 1),
                           "span_ms": round(span * 1e3, 2), "span_ms_min_max": [round(min(spans) * 1e3, 2),
                                                                             round(max(spans) * 1e3, 2)],
-                          "runs": len(runs),
+                          "runs": len(runs), "sm_copy_ops": runs[-1]["sm_copy_ops"],
                           "tstar_ms": round(tstar * 1e3, 3), "roofline_frac": round(tstar / span, 4),
                           "tstar_terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()},
                           "copy_replay_ms": round(replay * 1e3, 3),

@@ -159,6 +159,10 @@ typedef struct {
     int64_t  gpu_clock_offset_ns[8];              /* per physical GPU (first 8): %globaltimer minus
                                                      CLOCK_REALTIME, calibrated at init (kl_gpu_*
                                                      stamps - offset = host clock); 0 if unknown */
+    uint64_t sm_copy_ops;                         /* H2D/D2H ops served as zero-copy SM copies by the
+                                                     dispatcher's copy partition (small ops with mapped
+                                                     pinned host buffers; STRINGS_COPY_CTAS,
+                                                     STRINGS_SM_COPY_MAX) instead of the copy engines */
 } strings_stats_t;
 
 /* Initialise the runtime (gPool creation): enumerate the GPUs,

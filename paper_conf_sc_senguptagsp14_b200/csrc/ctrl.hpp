@@ -25,7 +25,7 @@ struct __align__(32) KlDone {
 // Host-mapped part (cudaHostAlloc mapped): the completion words the GPU writes.
 struct HostCtrl {
   uint32_t pad[16];
-  // followed by KlDone[L][kRing]
+  // followed by KlDone[L][kRing], then the copy partition's KlDone[kRing] and CopyItem[kRing]
 };
 
 // Device-memory part: claim counters and per-partition mailboxes.
@@ -52,6 +52,65 @@ struct __align__(128) PartState {
 //                    published when its seq == i + 1 (mod kRing reuse: seq is
 //                    monotone and the host never overwrites an unclaimed entry);
 //   stop             shutdown word, stream memory op at teardown.
+// Small host-link copies on SMs (the copy partition).  The copy engines serve
+// mixed-size traffic badly: a 128-256 KiB copy queued among 4-64 MiB copies
+// waits for them and costs ~14 us of engine time more than alone
+// (tools/mix_probe.cu, profiles/r01_mix_probe.jsonl).  So H2D/D2H ops of up to
+// STRINGS_SM_COPY_MAX bytes whose host buffers are mapped pinned memory run on
+// a partition of the persistent dispatcher instead: 16-B zero-copy loads and
+// stores over PCIe, concurrent with the engines' large copies.  The host
+// writes a CopyItem into a host-mapped table and publishes (seq, index) into a
+// device-memory ring with one stream memory op (no copy-engine operation on
+// this path); the partition leader claims it, the item is read once from host
+// memory, and the last CTA writes a KlDone word into host memory.
+struct CopySeg {
+  uint64_t src, dst, bytes;           // device-visible addresses; 16-B aligned, bytes % 16 == 0
+};
+constexpr int kCopySegs = 4;
+struct __align__(128) CopyItem {
+  uint64_t job;
+  uint32_t nseg;
+  uint32_t to_host;                   // 1: destinations are host memory (D2H): system-scope fence
+  CopySeg seg[kCopySegs];
+};
+static_assert(sizeof(CopyItem) == 128, "CopyItem layout");
+
+__device__ __forceinline__ uint4 ld_cv_v4(const uint4* p) {     // host memory: never a stale cached line
+  uint4 r;
+  asm volatile("ld.global.cv.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+  return r;
+}
+__device__ __forceinline__ uint4 ld_cg_v4(const uint4* p) {     // device memory another SM wrote
+  uint4 r;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+  return r;
+}
+
+// One copy item on the partition's S CTAs: every segment cut into 16-B words
+// dealt round-robin over S*256 threads, 8 independent loads in flight per
+// thread (32 KB per CTA) to cover the PCIe round trip.
+__device__ __forceinline__ void copy_body(const CopyItem& c, int rank, int S) {
+  const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x;
+  const uint64_t nthr = (uint64_t)S * kThreads;
+  constexpr int U = 8;
+  for (uint32_t g = 0; g < c.nseg; ++g) {
+    const uint4* src = reinterpret_cast<const uint4*>(c.seg[g].src);
+    uint4* dst = reinterpret_cast<uint4*>(c.seg[g].dst);
+    const uint64_t n16 = c.seg[g].bytes / 16;
+    uint64_t i = tid;
+    for (; i + (U - 1) * nthr < n16; i += U * nthr) {
+      uint4 v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) v[u] = c.to_host ? ld_cg_v4(src + i + u * nthr) : ld_cv_v4(src + i + u * nthr);
+#pragma unroll
+      for (int u = 0; u < U; ++u) dst[i + u * nthr] = v[u];
+    }
+    for (; i < n16; i += nthr) dst[i] = c.to_host ? ld_cg_v4(src + i) : ld_cv_v4(src + i);
+  }
+}
+
 struct DispatchParams {
   KlDone* done;                       // [L * kRing] host-mapped completion words
   uint32_t* heads;                    // [L] device-memory claim counters
@@ -64,8 +123,16 @@ struct DispatchParams {
   uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
   uint32_t poll_max_ns;               // idle-poll back-off cap (STRINGS_POLL_MAX_NS)
   uint64_t fault_job;                 // fault injection (STRINGS_FAULT_JOB): trap on this job id
+  // copy partition (partition index L*P, CTAs [part_start[L*P], part_start[L*P+1])) when copy_ctas > 0;
+  // its claim counter is heads[L] and its PartState parts[L*P]
+  int copy_ctas;
+  const uint64_t* cring;              // [kRing] device ring entries (seq << 32) | index
+  const CopyItem* citems;             // [kRing] host-mapped copy items (device view)
+  KlDone* cdone;                      // [kRing] host-mapped completion words
 };
 
-inline size_t host_ctrl_bytes(int L) { return sizeof(HostCtrl) + sizeof(KlDone) * kRing * L; }
+inline size_t host_ctrl_bytes(int L) {
+  return sizeof(HostCtrl) + sizeof(KlDone) * kRing * (L + 1) + sizeof(CopyItem) * kRing + 128;
+}
 
 }  // namespace strings_dev

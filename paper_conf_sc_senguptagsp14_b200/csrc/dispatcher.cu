@@ -19,6 +19,9 @@
 // from the device item table, runs its share of the item, and the last CTA to
 // finish writes the completion word and the %globaltimer stamps back to host
 // memory (gpu-scope fence + plain store).
+// With copy_ctas > 0 the last partition serves small H2D/D2H copies instead
+// (ctrl.hpp, CopyItem): same claim/broadcast/completion protocol on its own
+// ring, the item read from host memory, the body a zero-copy PCIe copy.
 #include <cstdio>
 
 #include "ctrl.hpp"
@@ -65,17 +68,20 @@ __device__ __forceinline__ void partition_of(int b, int NP, const int* part_star
 __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams p) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ KlItem s_item;
+  __shared__ CopyItem s_citem;
   __shared__ uint32_t s_gen, s_slot;
   GemmSmem sm = carve_smem(smem);
   if ((smem_u32(smem) & 1023u) != 0) __trap();   // SWIZZLE_128B tiles need a 1 KB-aligned base
-  const int NP = p.L * p.P;
+  const int NK = p.L * p.P;                       // KL partitions; the copy partition (if any) is NK
+  const int NP = NK + (p.copy_ctas > 0 ? 1 : 0);
   int q, start, S;
   partition_of(blockIdx.x, NP, p.part_start, &q, &start, &S);
   const int rank = blockIdx.x - start;
-  const int ld = q / p.P;
+  const bool cpart = q == NK;
+  const int ld = cpart ? p.L : q / p.P;           // claim counter heads[ld]
   PartState* ps = p.parts + q;
-  const KlItem* table = p.items + (size_t)ld * p.M;
-  const uint64_t* ring = p.ring + (size_t)ld * kRing;
+  const KlItem* table = p.items + (size_t)(cpart ? 0 : ld) * p.M;
+  const uint64_t* ring = cpart ? p.cring : p.ring + (size_t)ld * kRing;
   const uint32_t tmem = cta_setup(sm);
   uint32_t mma_phase = 0;
   uint32_t seen = 0;
@@ -116,7 +122,11 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
       __syncwarp();                               // orders lane 0's acquire before the item loads
       gw = __shfl_sync(0xffffffffu, gw, 0);
       const uint32_t g = (uint32_t)gw, slot = (uint32_t)(gw >> 32);
-      if (g != kStop) {
+      if (g != kStop && cpart) {
+        // the 128-B copy item from the host-mapped table: one PCIe read by 8 lanes
+        if (lane < sizeof(CopyItem) / 16)
+          reinterpret_cast<uint4*>(&s_citem)[lane] = ld_cv_v4(reinterpret_cast<const uint4*>(p.citems + slot) + lane);
+      } else if (g != kStop) {
         // the 512-B item straight from the device item table: one warp-wide L2 read
         // (.cg: the copy engine wrote it, no stale L1 line)
         uint4 v;
@@ -134,17 +144,26 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     const uint32_t g = s_gen;
     if (g == kStop) break;
     seen = g;
-    const KlItem it = s_item;
-    if (it.job == p.fault_job) __trap();          // fault injection (tests the watchdog)
     if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
-    run_item(it, table + s_slot, true, rank, S, sm, tmem, mma_phase, &ps->sync);
+    if (cpart) {
+      copy_body(s_citem, rank, S);
+    } else {
+      const KlItem it = s_item;
+      if (it.job == p.fault_job) __trap();        // fault injection (tests the watchdog)
+      run_item(it, table + s_slot, true, rank, S, sm, tmem, mma_phase, &ps->sync);
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
-      __threadfence();
+      // D2H copy items wrote host memory: their stores must be visible system-wide
+      // before the completion word; everything else only needs gpu scope
+      if (cpart && s_citem.to_host)
+        __threadfence_system();
+      else
+        __threadfence();
       const uint32_t old = atomicAdd(&ps->done_cnt, 1u);
       if (old == (uint32_t)S - 1) {
         ps->done_cnt = 0;
-        KlDone* d = &p.done[ld * kRing + ps->ring_idx];
+        KlDone* d = cpart ? &p.cdone[ps->ring_idx] : &p.done[ld * kRing + ps->ring_idx];
         d->partition = (uint32_t)q;
         d->t_start = ps->t_start;
         d->t_exec = ps->t_exec;

@@ -46,6 +46,7 @@ cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaS
 using strings_dev::HostCtrl;
 using strings_dev::KlDone;
 using strings_dev::KlItem;
+using strings_dev::CopyItem;
 using strings_dev::kRing;
 
 namespace {
@@ -156,6 +157,7 @@ struct HostBuf {
   void* user = nullptr;     // caller's buffer
   uint64_t bytes = 0;
   void* dma = nullptr;      // pinned address used by the copy engine
+  uint64_t dev_view = 0;    // device-visible address of dma (mapped pinned memory), 0 = not mapped
   bool staged = false;      // dma is library-owned staging (PMT entry)
 };
 
@@ -173,6 +175,9 @@ struct JobCtx {
   uint32_t kl_seq = 0;
   bool item_ok = false;                // KL work item built (and staged) at H2D issue
   uint32_t copy_seq[3] = {0, 0, 0};
+  bool smcopy[3] = {false, false, false};          // op runs on the dispatcher's copy partition
+  uint32_t cseq[3] = {0, 0, 0};
+  int cidx[3] = {-1, -1, -1};
   int kl_idx = -1;
   int kl_partition = -1;
   uint64_t kl_t0 = 0, kl_t1 = 0, kl_exec = 0;     // device %globaltimer: claim, end, body start
@@ -224,6 +229,19 @@ struct Phys {
   uint8_t* ring_dev = nullptr;         // [L][kRing] u64
   uint8_t* items_dev = nullptr;        // [L][M] KlItem
   KlItem* items_host = nullptr;        // [L][M] pinned staging
+  uint64_t items_host_dev = 0;         // device view of items_host (mapped)
+  // copy partition (ctrl.hpp CopyItem): small H2D/D2H ops as zero-copy SM copies
+  int copy_ctas = 0;
+  uint8_t* cring_dev = nullptr;        // [kRing] u64 ring entries (device memory)
+  CopyItem* citems = nullptr;          // [kRing] host-mapped items
+  KlDone* cdone = nullptr;             // [kRing] host-mapped completion words
+  uint32_t ctail = 0, ccompleted = 0;
+  // ring index still owned by an op whose completion the engine has not consumed:
+  // ops of different logical devices / directions are consumed out of ring order
+  // (in INJECTED timing an op may be issued long before its virtual DONE), so an
+  // index is reused only after its own op was observed, never by count alone
+  std::vector<uint8_t> cbusy = std::vector<uint8_t>(kRing, 0);
+  cudaStream_t cpstream = nullptr;     // stream memory ops publishing copy ring entries
   int64_t clock_offset_ns = 0;         // %globaltimer - CLOCK_REALTIME (ping-pong, min RTT)
   uint64_t clock_rtt_ns = 0;
   bool kernel_running = false;
@@ -384,7 +402,7 @@ class StagingPool {
       return p;
     }
     void* p = nullptr;
-    if (!cuda_ok(cudaHostAlloc(&p, (size_t)1 << c, cudaHostAllocPortable))) return nullptr;
+    if (!cuda_ok(cudaHostAlloc(&p, (size_t)1 << c, cudaHostAllocPortable | cudaHostAllocMapped))) return nullptr;
     all_.push_back(p);
     return p;
   }
@@ -417,6 +435,17 @@ struct Tenant {
   uint32_t next_seq = 0;
   bool active = true;
 };
+
+// Copy partition size (CTAs = SMs of the persistent dispatcher serving small
+// H2D/D2H ops; 0 = every copy on the copy engines) and the largest op it takes.
+int copy_ctas_env() {
+  const char* e = getenv("STRINGS_COPY_CTAS");
+  return e ? std::max(0, atoi(e)) : 4;
+}
+uint64_t sm_copy_max_env() {
+  const char* e = getenv("STRINGS_SM_COPY_MAX");
+  return e ? strtoull(e, nullptr, 0) : (1ull << 20);
+}
 
 // PMT staging copy threads: most of the host's cores (the engine thread and the
 // caller keep one each); STRINGS_COPY_THREADS overrides.
@@ -453,6 +482,14 @@ class Runtime : public strings::Hooks {
   uint64_t first_submit = 0, last_done = 0;
   uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
   uint64_t decision_ns = 0;            // time inside Core::step (decisions + op issue)
+  uint64_t sm_copies = 0;              // H2D/D2H ops served by the copy partition
+  uint64_t last_progress = 0;
+  bool stall_dumped = false;
+  const uint64_t stall_dump_ns = [] {
+    const char* e = getenv("STRINGS_STALL_DUMP_S");
+    return (uint64_t)((e ? atof(e) : 20.0) * 1e9);
+  }();
+  const uint64_t sm_copy_max = sm_copy_max_env();
   uint64_t issue_ns = 0;               // of which: issuing woken ops (on_wake)
   // in-flight physical ops (measured mode): (job, engine)
   std::vector<std::pair<JobCtx*, int>> inflight;
@@ -562,6 +599,10 @@ class Runtime : public strings::Hooks {
       if (const char* lim = getenv("STRINGS_SM_LIMIT"))
         if (atoi(lim) > 0) ph->sms = std::min(ph->sms, atoi(lim));
       if (ph->L * cfg.partitions > ph->sms) return STRINGS_EINVAL;
+      // the copy partition takes the last copy_ctas SMs when enough remain for the KL partitions
+      ph->copy_ctas = kl_mode == 0 ? copy_ctas_env() : 0;
+      if (ph->L * cfg.partitions > ph->sms - ph->copy_ctas) ph->copy_ctas = 0;
+      const int sms_kl = ph->sms - ph->copy_ctas;
       // SM shares: logical devices of this GPU get CTAs in proportion to their
       // weights, each share split evenly into P partitions (one per KL slot)
       {
@@ -574,15 +615,16 @@ class Runtime : public strings::Hooks {
         for (size_t i = 0; i < lds.size(); ++i) {
           const int lo = ph->part_start.back();
           wacc += weights[lds[i]];
-          int hi = (int)((uint64_t)ph->sms * wacc / wsum);
+          int hi = (int)((uint64_t)sms_kl * wacc / wsum);
           hi = std::max(hi, lo + cfg.partitions);
           const int remaining_ld = (int)(lds.size() - 1 - i);
-          hi = std::min(hi, ph->sms - remaining_ld * cfg.partitions);
-          if (i + 1 == lds.size()) hi = ph->sms;
+          hi = std::min(hi, sms_kl - remaining_ld * cfg.partitions);
+          if (i + 1 == lds.size()) hi = sms_kl;
           for (int p = 1; p <= cfg.partitions; ++p)
             ph->part_start.push_back(lo + (int)((int64_t)(hi - lo) * p / cfg.partitions));
           logical[lds[i]].ctas = hi - lo;
         }
+        if (ph->copy_ctas) ph->part_start.push_back(ph->sms);     // the copy partition
       }
       // host-mapped control block
       size_t cb = strings_dev::host_ctrl_bytes(ph->L);
@@ -592,6 +634,13 @@ class Runtime : public strings::Hooks {
       memset(hp, 0, cb);
       ph->ctrl = static_cast<HostCtrl*>(hp);
       if (!cuda_ok(cudaHostGetDevicePointer(&ph->ctrl_dev, hp, 0))) return STRINGS_ECUDA;
+      {
+        uint8_t* cb0 = static_cast<uint8_t*>(hp) + sizeof(HostCtrl) + sizeof(KlDone) * kRing * ph->L;
+        ph->cdone = reinterpret_cast<KlDone*>(cb0);
+        uint8_t* ci = cb0 + sizeof(KlDone) * kRing;
+        ci += (128 - reinterpret_cast<uintptr_t>(ci) % 128) % 128;
+        ph->citems = reinterpret_cast<CopyItem*>(ci);
+      }
       void* cp = nullptr;
       if (!cuda_ok(cudaHostAlloc(&cp, sizeof(CopyCounters) * ph->L, cudaHostAllocMapped | cudaHostAllocPortable)))
         return STRINGS_ENOMEM;
@@ -606,10 +655,10 @@ class Runtime : public strings::Hooks {
           return STRINGS_ECUDA;
         g_write_value32 = reinterpret_cast<WriteValue32Fn>(fn);
       }
-      // device state: heads[L] (padded) + parts[L*P] + partition table + doorbells
-      // (one 128-B line per logical device's ring tail, one for shutdown)
-      size_t heads_bytes = 128 * (size_t)ph->L;
-      size_t parts_bytes = sizeof(strings_dev::PartState) * ph->L * cfg.partitions;
+      // device state: heads[L + 1] (padded; [L] = copy ring) + parts[L*P + 1] + partition
+      // table + doorbells (one 128-B line per logical device's ring tail, one for shutdown)
+      size_t heads_bytes = 128 * (size_t)(ph->L + 1);
+      size_t parts_bytes = sizeof(strings_dev::PartState) * (ph->L * cfg.partitions + 1);
       size_t table_bytes = sizeof(int) * ph->part_start.size();
       size_t db_off = align_up(heads_bytes + parts_bytes + table_bytes);
       size_t db_bytes = 128;                                         // shutdown word
@@ -617,16 +666,23 @@ class Runtime : public strings::Hooks {
       size_t ring_bytes = sizeof(uint64_t) * kRing * ph->L;
       size_t items_off = align_up(ring_off + ring_bytes);
       size_t items_bytes = sizeof(KlItem) * (size_t)cfg.admit_cap * ph->L;
-      if (!cuda_ok(cudaMalloc(&ph->dev_state, items_off + items_bytes))) return STRINGS_ENOMEM;
-      if (!cuda_ok(cudaMemset(ph->dev_state, 0, items_off + items_bytes))) return STRINGS_ECUDA;
+      size_t cring_off = align_up(items_off + items_bytes);
+      size_t cring_bytes = sizeof(uint64_t) * kRing;
+      if (!cuda_ok(cudaMalloc(&ph->dev_state, cring_off + cring_bytes))) return STRINGS_ENOMEM;
+      if (!cuda_ok(cudaMemset(ph->dev_state, 0, cring_off + cring_bytes))) return STRINGS_ECUDA;
       ph->doorbells = ph->dev_state + db_off;
       ph->ring_dev = ph->dev_state + ring_off;
       ph->items_dev = ph->dev_state + items_off;
+      ph->cring_dev = ph->dev_state + cring_off;
       {
         void* ih = nullptr;
-        if (!cuda_ok(cudaHostAlloc(&ih, items_bytes, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+        if (!cuda_ok(cudaHostAlloc(&ih, items_bytes, cudaHostAllocPortable | cudaHostAllocMapped)))
+          return STRINGS_ENOMEM;
         memset(ih, 0, items_bytes);
         ph->items_host = static_cast<KlItem*>(ih);
+        void* ihd = nullptr;
+        if (!cuda_ok(cudaHostGetDevicePointer(&ihd, ih, 0))) return STRINGS_ECUDA;
+        ph->items_host_dev = reinterpret_cast<uint64_t>(ihd);
       }
       if (!g_write_value64) {
         cudaDriverEntryPointQueryResult q;
@@ -656,6 +712,7 @@ class Runtime : public strings::Hooks {
       }
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->kstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
       if (!cuda_ok(cudaStreamCreateWithFlags(&ph->dbstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+      if (!cuda_ok(cudaStreamCreateWithFlags(&ph->cpstream, cudaStreamNonBlocking))) return STRINGS_ECUDA;
       KlDone* dones = reinterpret_cast<KlDone*>(static_cast<uint8_t*>(hp) + sizeof(HostCtrl));
       const char* cs = getenv("STRINGS_COPY_STREAMS");
       const bool shared_copy = cs && strcmp(cs, "physical") == 0;
@@ -713,6 +770,12 @@ class Runtime : public strings::Hooks {
         const char* pm = getenv("STRINGS_POLL_MAX_NS");
         dp.poll_max_ns = pm ? (uint32_t)strtoul(pm, nullptr, 0) : 1024u;
         dp.stop = reinterpret_cast<const uint32_t*>(ph->doorbells);
+        dp.copy_ctas = ph->copy_ctas;
+        dp.cring = reinterpret_cast<const uint64_t*>(ph->cring_dev);
+        dp.citems = reinterpret_cast<const CopyItem*>(dbase + (reinterpret_cast<uint8_t*>(ph->citems) -
+                                                               reinterpret_cast<uint8_t*>(ph->ctrl)));
+        dp.cdone = reinterpret_cast<KlDone*>(dbase + (reinterpret_cast<uint8_t*>(ph->cdone) -
+                                                      reinterpret_cast<uint8_t*>(ph->ctrl)));
         if (!calibrate_clock(ph.get())) return STRINGS_ECUDA;
         if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
@@ -783,6 +846,11 @@ class Runtime : public strings::Hooks {
       }
       if (ph->dbstream) cudaStreamSynchronize(ph->dbstream), cudaStreamDestroy(ph->dbstream);
       ph->dbstream = nullptr;
+      if (ph->cpstream) cudaStreamSynchronize(ph->cpstream), cudaStreamDestroy(ph->cpstream);
+      ph->cpstream = nullptr;
+      ph->copy_ctas = 0;
+      ph->ctail = ph->ccompleted = 0;
+      std::fill(ph->cbusy.begin(), ph->cbusy.end(), 0);
       if (ph->h2d) cudaStreamSynchronize(ph->h2d), cudaStreamDestroy(ph->h2d);
       if (ph->d2h) cudaStreamSynchronize(ph->d2h), cudaStreamDestroy(ph->d2h);
       ph->h2d = ph->d2h = nullptr;
@@ -853,6 +921,29 @@ class Runtime : public strings::Hooks {
         }
         jc->dev_out = reinterpret_cast<uint64_t>(base + off);
       }
+      if (sm_copy_eligible(jc->in, ph)) {
+        // small inputs (+ the KL work item) as one zero-copy item on the copy partition
+        CopyItem ci;
+        memset(&ci, 0, sizeof ci);
+        ci.job = j.id;
+        for (size_t i = 0; i < jc->in.size(); ++i)
+          if (jc->in[i].bytes) ci.seg[ci.nseg++] = {jc->in[i].dev_view, jc->dev_in[i], jc->in[i].bytes};
+        KlItem& it = lg.item_host[jc->slot];
+        jc->item_ok = build_item(j, jc, it);
+        if (jc->item_ok) {
+          const uint64_t off = sizeof(KlItem) * (size_t)(&it - ph->items_host);
+          ci.seg[ci.nseg++] = {ph->items_host_dev + off, lg.item_dev + sizeof(KlItem) * jc->slot,
+                               it.kclass == STRINGS_GEMM ? sizeof(KlItem) : offsetof(KlItem, tmap_a)};
+        }
+        ok = publish_copy(ph, jc, engine, ci);
+        jc->issued[engine] = true;
+        if (!ok) {
+          fail_job(jc);
+          jc->phys_done[engine] = true;
+        }
+        if (!virtual_clock()) inflight.push_back({jc, engine});
+        return;
+      }
       for (size_t i = 0; i < jc->in.size() && ok; ++i)
         if (jc->in[i].bytes)
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma,
@@ -871,6 +962,17 @@ class Runtime : public strings::Hooks {
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(lg.item_dev + sizeof(KlItem) * jc->slot), &it, bytes,
                                        cudaMemcpyHostToDevice, ph->dbstream));
       }
+    } else if (engine == strings::ENG_D2H && sm_copy_eligible(jc->out, ph)) {
+      CopyItem ci;
+      memset(&ci, 0, sizeof ci);
+      ci.job = j.id;
+      ci.to_host = 1;
+      uint64_t off = 0;
+      for (size_t i = 0; i < jc->out.size(); ++i) {
+        if (jc->out[i].bytes) ci.seg[ci.nseg++] = {jc->dev_out + off, jc->out[i].dev_view, jc->out[i].bytes};
+        off = align_up(off + jc->out[i].bytes);
+      }
+      ok = publish_copy(ph, jc, engine, ci);
     } else if (engine == strings::ENG_D2H) {
       uint64_t off = 0;
       for (size_t i = 0; i < jc->out.size() && ok; ++i) {
@@ -987,6 +1089,46 @@ class Runtime : public strings::Hooks {
     }
   }
 
+  // An H2D/D2H op goes to the copy partition when it is small, every host buffer
+  // is mapped pinned memory, every address and size is 16-B aligned, there is a
+  // segment left for the KL work item, and the copy ring has room.
+  bool sm_copy_eligible(const std::vector<HostBuf>& bufs, const Phys* ph) const {
+    if (!ph->copy_ctas || kl_mode != 0) return false;
+    uint64_t total = 0;
+    int nseg = 0;
+    for (const auto& b : bufs) {
+      if (!b.bytes) continue;
+      if (!b.dev_view || ((b.dev_view | b.bytes) & 15)) return false;
+      total += b.bytes;
+      ++nseg;
+    }
+    return total > 0 && total <= sm_copy_max && nseg + 1 <= strings_dev::kCopySegs &&
+           !ph->cbusy[ph->ctail % kRing];
+  }
+
+  // Write the item into the host-mapped table, then publish (seq, index) into the
+  // device ring with one stream memory op (no copy-engine operation).
+  bool publish_copy(Phys* ph, JobCtx* jc, int engine, const CopyItem& ci) {
+    const uint32_t idx = ph->ctail % kRing;
+    const uint32_t seq = ph->ctail + 1;
+    ph->citems[idx] = ci;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    CUresult r = g_write_value64(reinterpret_cast<CUstream>(ph->cpstream),
+                                 reinterpret_cast<CUdeviceptr>(ph->cring_dev) + sizeof(uint64_t) * idx,
+                                 ((uint64_t)seq << 32) | idx, 0);
+    if (r != CUDA_SUCCESS) {
+      g_last_cuda_error.store(10000 + (int32_t)r);
+      return false;
+    }
+    ph->ctail = seq;
+    ph->cbusy[idx] = 1;
+    jc->smcopy[engine] = true;
+    jc->cseq[engine] = seq;
+    jc->cidx[engine] = (int)idx;
+    sm_copies += 1;
+    return true;
+  }
+
   // Append "done[engine] = seq" to the copy stream (ordered after the copies).
   bool signal_copy(Logical& lg, JobCtx* jc, int engine, cudaStream_t s) {
     const uint32_t seq = ++lg.issued[engine];
@@ -1031,6 +1173,16 @@ class Runtime : public strings::Hooks {
       jc->kl_exec = d->t_exec;
       jc->kl_observe = real_ns();
       lg.completed += 1;
+      jc->phys_done[engine] = true;
+      return true;
+    }
+    if (jc->smcopy[engine]) {
+      Phys* ph = lg.phys;
+      volatile KlDone* d = &ph->cdone[jc->cidx[engine]];
+      if (d->seq != jc->cseq[engine]) return false;
+      std::atomic_thread_fence(std::memory_order_acquire);
+      ph->ccompleted += 1;
+      ph->cbusy[jc->cidx[engine]] = 0;
       jc->phys_done[engine] = true;
       return true;
     }
@@ -1130,10 +1282,23 @@ class Runtime : public strings::Hooks {
       // decides, the GPU still does the work)
       for (auto& c : batch) {
         JobCtx* jc = jobs[c.job].get();
+        const uint64_t w0 = mono_ns();
         while (!phys_complete(jc, c.engine)) {
           if (!healthy()) {
             stop = true;
             return;
+          }
+          if (!stall_dumped && mono_ns() - w0 > stall_dump_ns) {
+            stall_dumped = true;
+            fprintf(stderr, "[strings] injected: waiting for job %llu engine %d (t = %llu)\n",
+                    (unsigned long long)c.job, c.engine, (unsigned long long)t);
+            for (size_t k = 0; k < jobs.size(); ++k) {
+              JobCtx* o = jobs[k].get();
+              for (int e = 0; e < 3; ++e)
+                if (o->issued[e] && !o->phys_done[e]) inflight.push_back({o, e});
+            }
+            dump_state();
+            inflight.clear();
           }
           lk.unlock();
           std::this_thread::yield();
@@ -1150,6 +1315,7 @@ class Runtime : public strings::Hooks {
 
   // One real-time batch in MEASURED mode.
   void measured_step(std::unique_lock<std::mutex>& lk) {
+    if (inflight.empty()) last_progress = mono_ns();
     std::vector<JobCtx*> news;
     take_inbox(news);
     uint64_t t = now();
@@ -1179,6 +1345,7 @@ class Runtime : public strings::Hooks {
           ++i;
         }
       }
+      if (!batch.empty()) last_progress = mono_ns();
       if (batch.empty() && !first) break;
       if (batch.empty() && !progressed && core->next_epoch() != t) break;
       const uint64_t d0 = mono_ns();
@@ -1192,9 +1359,39 @@ class Runtime : public strings::Hooks {
         stop = true;
         return;
       }
+      if (!inflight.empty() && !stall_dumped && mono_ns() - last_progress > stall_dump_ns) {
+        stall_dumped = true;
+        dump_state();
+      }
       lk.unlock();
       std::this_thread::yield();
       lk.lock();
+    }
+  }
+
+  // Diagnostics: no op completed for STRINGS_STALL_DUMP_S seconds (default 20)
+  // while ops are in flight -> print the in-flight ops and queue states once.
+  void dump_state() {
+    fprintf(stderr, "[strings] stall: %zu ops in flight, %llu/%llu jobs done\n", inflight.size(),
+            (unsigned long long)done_count, (unsigned long long)submitted);
+    for (auto& ph : phys)
+      fprintf(stderr, "[strings]  gpu %d: copy ring tail %u completed %u, copy ctas %d\n", ph->dev, ph->ctail,
+              ph->ccompleted, ph->copy_ctas);
+    for (auto& lg : logical)
+      fprintf(stderr, "[strings]  ld %d: KL tail %u completed %u, copies issued h2d %u d2h %u, done h2d %u d2h %u\n",
+              lg.gid, lg.tail, lg.completed, lg.issued[0], lg.issued[2], lg.ctr ? lg.ctr->done[0] : 0,
+              lg.ctr ? lg.ctr->done[2] : 0);
+    for (auto& f : inflight) {
+      JobCtx* jc = f.first;
+      const int e = f.second;
+      const strings::Job& j = jc->job;
+      uint32_t cd = 0;
+      if (jc->smcopy[e]) cd = logical[j.gid].phys->cdone[jc->cidx[e]].seq;
+      fprintf(stderr,
+              "[strings]  job %llu gid %d engine %d phase %d slot %d started %d sm %d cseq %u cidx %d cdone %u "
+              "copy_seq %u kl_seq %u kl_idx %d\n",
+              (unsigned long long)j.id, j.gid, e, j.phase, j.slot[e], (int)(j.phase == e && j.slot[e] >= 0),
+              (int)jc->smcopy[e], jc->cseq[e], jc->cidx[e], cd, jc->copy_seq[e], jc->kl_seq, jc->kl_idx);
     }
   }
 
@@ -1260,12 +1457,18 @@ class Runtime : public strings::Hooks {
       cudaError_t e = cudaPointerGetAttributes(&a, b.host);
       if (e != cudaSuccess) cudaGetLastError();
       bool pinned = e == cudaSuccess && a.type == cudaMemoryTypeHost;
-      if (pinned) return STRINGS_OK;
+      if (pinned) {
+        hb.dev_view = reinterpret_cast<uint64_t>(a.devicePointer);   // null unless mapped
+        return STRINGS_OK;
+      }
       void* p = staging.get(b.bytes);
       if (!p) return STRINGS_ENOMEM;
       if (is_in) copier.copy(p, b.host, b.bytes);
       hb.dma = p;
       hb.staged = true;
+      void* dv = nullptr;
+      if (cudaHostGetDevicePointer(&dv, p, 0) == cudaSuccess) hb.dev_view = reinterpret_cast<uint64_t>(dv);
+      else cudaGetLastError();
       return STRINGS_OK;
     };
     jc->in.resize(n_h2d);
@@ -1430,7 +1633,7 @@ strings_status_t strings_shutdown(void) {
 
 strings_status_t strings_host_alloc(uint64_t bytes, void** p) {
   if (!p) return STRINGS_EINVAL;
-  if (!cuda_ok(cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable))) return STRINGS_ENOMEM;
+  if (!cuda_ok(cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable | cudaHostAllocMapped))) return STRINGS_ENOMEM;
   return STRINGS_OK;
 }
 
@@ -1496,6 +1699,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->decision_ns = r.decision_ns;
   st->issue_ns = r.issue_ns;
   for (size_t i = 0; i < r.phys.size() && i < 8; ++i) st->gpu_clock_offset_ns[i] = r.phys[i]->clock_offset_ns;
+  st->sm_copy_ops = r.sm_copies;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

@@ -67,7 +67,8 @@ class Stats(C.Structure):
                 ("decision_ns", C.c_uint64),
                 ("engine_busy_ns", (C.c_uint64 * 3) * 8), ("num_gpus", C.c_int32),
                 ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32),
-                ("issue_ns", C.c_uint64), ("gpu_clock_offset_ns", C.c_int64 * 8)]
+                ("issue_ns", C.c_uint64), ("gpu_clock_offset_ns", C.c_int64 * 8),
+                ("sm_copy_ops", C.c_uint64)]
 
 
 def _load() -> C.CDLL:

@@ -203,6 +203,60 @@ def test_pageable_misaligned_ragged_buffers(n):
         S.shutdown()
 
 
+@pytest.mark.parametrize("copy_ctas", ["0", "1", "4", "16"])
+def test_small_copies_on_the_copy_partition(copy_ctas, monkeypatch):
+    # GEMM jobs' 2 x 128 KiB H2D and 256 KiB D2H are small enough for the
+    # dispatcher's copy partition (zero-copy SM copies, ctrl.hpp CopyItem); VSCALE's
+    # 4 MiB copies stay on the copy engines.  Outputs exact either way, measured
+    # invariants hold, and the stats say which path ran.
+    monkeypatch.setenv("STRINGS_COPY_CTAS", copy_ctas)
+    wl = W.config_c1(reps=2)
+    r = run_workload(wl, timing_mode=S.MEASURED)
+    assert r.status == S.OK
+    assert invariants.check(r.trace, wl) == []
+    check_outputs(wl, r)
+    n_gemm = sum(1 for j in wl.jobs if j.kclass == W.GEMM)
+    if copy_ctas == "0":
+        assert r.stats.sm_copy_ops == 0
+    else:
+        assert r.stats.sm_copy_ops == 2 * n_gemm        # H2D and D2H of every GEMM job
+
+
+def test_small_copies_injected_parity_and_threshold(monkeypatch):
+    # the physical copy path never changes decisions: INJECTED traces stay
+    # byte-identical to the oracle with every op small enough for the partition
+    monkeypatch.setenv("STRINGS_SM_COPY_MAX", str(64 << 20))
+    wl = W.config_c3(scale=4)
+    r = run_workload(wl, timing_mode=S.INJECTED)
+    assert r.status == S.OK
+    assert r.trace == run_oracle(wl).trace
+    check_outputs(wl, r)
+    assert r.stats.sm_copy_ops == 2 * len(wl.jobs)
+
+
+def test_misaligned_pinned_buffers_use_the_copy_engines():
+    # a caller-pinned buffer off a 16-B boundary cannot take the 16-B zero-copy path
+    S.init(num_gpus=1, physical_gpus=1)
+    try:
+        t = S.register_tenant()
+        n = 4097
+        xs = S.pinned_array((n + 1,), np.uint32)[1:]
+        ys = S.pinned_array((n + 1,), np.uint32)[1:]
+        xs[...] = np.arange(n, dtype=np.uint32) * 2654435761
+        S.submit(t, S.make_desc(S.XFER, n=n, seed=5), [xs], [ys])
+        assert S.sync(t) == S.OK
+        assert np.array_equal(ys, K.xfer(xs, 5))
+        assert S.stats().sm_copy_ops == 0
+        a = S.pinned_array((n,), np.uint32)
+        b = S.pinned_array((n + 3,), np.uint32)      # 16-B aligned start, ragged size -> not % 16
+        a[...] = 7
+        S.submit(t, S.make_desc(S.XFER, n=n, seed=5), [a], [b[:n]])
+        assert S.sync(t) == S.OK
+        assert np.array_equal(b[:n], K.xfer(a, 5))
+    finally:
+        S.shutdown()
+
+
 def test_full_size_c2_measured_sampled_parity():
     # BASELINE configs[1] at full size, in the launch configuration bench.py
     # times (MEASURED, persistent dispatcher): every GEMM output in full, XFER
