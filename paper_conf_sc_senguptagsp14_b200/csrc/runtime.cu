@@ -176,6 +176,8 @@ struct JobCtx {
   bool item_ok = false;                // KL work item built (and staged) at H2D issue
   uint32_t copy_seq[3] = {0, 0, 0};
   bool smcopy[3] = {false, false, false};          // op runs on the dispatcher's copy partition
+  uint32_t item_cseq = 0;                          // KL work item copied by the copy partition
+  int item_cidx = -1;                              //   (CE-path H2D jobs), consumed at KL issue
   uint32_t cseq[3] = {0, 0, 0};
   int cidx[3] = {-1, -1, -1};
   int kl_idx = -1;
@@ -490,6 +492,14 @@ class Runtime : public strings::Hooks {
     return (uint64_t)((e ? atof(e) : 20.0) * 1e9);
   }();
   const uint64_t sm_copy_max = sm_copy_max_env();
+  // STRINGS_ITEM_VIA_COPY=1: the KL work item of a copy-engine job goes through the
+  // copy partition too.  Off by default: C3 6% slower (the KL issue must wait for
+  // the item behind the ring's 256 KiB copies), C1/C2/C4 within noise
+  // (profiles/r01_item_path_ab.jsonl).
+  const bool item_via_copy = [] {
+    const char* e = getenv("STRINGS_ITEM_VIA_COPY");
+    return e && e[0] == '1';
+  }();
   uint64_t issue_ns = 0;               // of which: issuing woken ops (on_wake)
   // in-flight physical ops (measured mode): (job, engine)
   std::vector<std::pair<JobCtx*, int>> inflight;
@@ -951,16 +961,25 @@ class Runtime : public strings::Hooks {
       ok = ok && signal_copy(lg, jc, engine, lg.h2d);
       if (ok && kl_mode == 0) {
         // The job's KL work item goes to the device item table (the dispatcher
-        // never reads host memory, ctrl.hpp) on the queue stream, after the input
-        // copies are queued and off the H2D stream; the KL's ring entry is written
-        // later on the same queue stream, hence after this copy.  The slot's
-        // previous item copy finished before the slot was freed (its KL ran).
+        // never reads host memory, ctrl.hpp): optionally through the copy
+        // partition (item_via_copy), else on the queue stream,
+        // where the KL's ring entry is written later, hence after this copy.  The
+        // slot's previous item copy finished before the slot was freed (its KL ran).
         KlItem& it = lg.item_host[jc->slot];
         jc->item_ok = build_item(j, jc, it);
         const size_t bytes = it.kclass == STRINGS_GEMM ? sizeof(KlItem) : offsetof(KlItem, tmap_a);
-        if (jc->item_ok)
+        if (jc->item_ok && item_via_copy && ph->copy_ctas && !ph->cbusy[ph->ctail % kRing]) {
+          CopyItem ci;
+          memset(&ci, 0, sizeof ci);
+          ci.job = j.id;
+          ci.nseg = 1;
+          ci.seg[0] = {ph->items_host_dev + sizeof(KlItem) * (size_t)(&it - ph->items_host),
+                       lg.item_dev + sizeof(KlItem) * jc->slot, bytes};
+          ok = publish_copy_item(ph, ci, &jc->item_cseq, &jc->item_cidx);
+        } else if (jc->item_ok) {
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(lg.item_dev + sizeof(KlItem) * jc->slot), &it, bytes,
                                        cudaMemcpyHostToDevice, ph->dbstream));
+        }
       }
     } else if (engine == strings::ENG_D2H && sm_copy_eligible(jc->out, ph)) {
       CopyItem ci;
@@ -983,7 +1002,9 @@ class Runtime : public strings::Hooks {
       }
       ok = ok && signal_copy(lg, jc, engine, lg.d2h);
     } else if (kl_mode == 0) {
-      if (!jc->item_ok || lg.tail - lg.completed >= (uint32_t)kRing) {
+      if (!await_item_copy(ph, jc)) {
+        ok = false;
+      } else if (!jc->item_ok || lg.tail - lg.completed >= (uint32_t)kRing) {
         ok = false;   // bad item (fault localised to this job); a full ring cannot happen with A <= kRing
       } else {
         // one 64-bit stream memory op publishes ring entry (seq, slot); it is ordered
@@ -1036,6 +1057,7 @@ class Runtime : public strings::Hooks {
     bool staged_out = false;
     if (has_gpu()) {
       Logical& lg = logical[j.gid];
+      if (jc->item_cidx >= 0) await_item_copy(lg.phys, jc);   // KL never issued (failed job): free the index
       if (jc->slot >= 0) {              // the D2H finished: the device slot is free now
         lg.free_slots.push_back(jc->slot);
         jc->slot = -1;
@@ -1108,7 +1130,7 @@ class Runtime : public strings::Hooks {
 
   // Write the item into the host-mapped table, then publish (seq, index) into the
   // device ring with one stream memory op (no copy-engine operation).
-  bool publish_copy(Phys* ph, JobCtx* jc, int engine, const CopyItem& ci) {
+  bool publish_copy_item(Phys* ph, const CopyItem& ci, uint32_t* seq_out, int* idx_out) {
     const uint32_t idx = ph->ctail % kRing;
     const uint32_t seq = ph->ctail + 1;
     ph->citems[idx] = ci;
@@ -1122,10 +1144,35 @@ class Runtime : public strings::Hooks {
     }
     ph->ctail = seq;
     ph->cbusy[idx] = 1;
+    *seq_out = seq;
+    *idx_out = (int)idx;
+    return true;
+  }
+  bool publish_copy(Phys* ph, JobCtx* jc, int engine, const CopyItem& ci) {
+    if (!publish_copy_item(ph, ci, &jc->cseq[engine], &jc->cidx[engine])) return false;
     jc->smcopy[engine] = true;
-    jc->cseq[engine] = seq;
-    jc->cidx[engine] = (int)idx;
     sm_copies += 1;
+    return true;
+  }
+  bool copy_item_done(Phys* ph, uint32_t seq, int idx) {
+    volatile KlDone* d = &ph->cdone[idx];
+    if (d->seq != seq) return false;
+    std::atomic_thread_fence(std::memory_order_acquire);
+    ph->ccompleted += 1;
+    ph->cbusy[idx] = 0;
+    return true;
+  }
+  // The KL work item of a copy-engine H2D job was sent through the copy ring at
+  // H2D issue; its KL ring entry may be published only after it landed.  It was
+  // issued at least one H2D op earlier, so this normally returns at once.
+  bool await_item_copy(Phys* ph, JobCtx* jc) {
+    if (jc->item_cidx < 0) return true;
+    const uint64_t t0 = mono_ns();
+    while (!copy_item_done(ph, jc->item_cseq, jc->item_cidx)) {
+      if (mono_ns() - t0 > 2000000000ull || !healthy()) return false;
+      std::this_thread::yield();
+    }
+    jc->item_cidx = -1;
     return true;
   }
 
@@ -1177,12 +1224,7 @@ class Runtime : public strings::Hooks {
       return true;
     }
     if (jc->smcopy[engine]) {
-      Phys* ph = lg.phys;
-      volatile KlDone* d = &ph->cdone[jc->cidx[engine]];
-      if (d->seq != jc->cseq[engine]) return false;
-      std::atomic_thread_fence(std::memory_order_acquire);
-      ph->ccompleted += 1;
-      ph->cbusy[jc->cidx[engine]] = 0;
+      if (!copy_item_done(lg.phys, jc->cseq[engine], jc->cidx[engine])) return false;
       jc->phys_done[engine] = true;
       return true;
     }
