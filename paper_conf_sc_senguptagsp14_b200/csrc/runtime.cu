@@ -1163,8 +1163,9 @@ class Runtime : public strings::Hooks {
     return true;
   }
   // The KL work item of a copy-engine H2D job was sent through the copy ring at
-  // H2D issue; its KL ring entry may be published only after it landed.  It was
-  // issued at least one H2D op earlier, so this normally returns at once.
+  // H2D issue; its KL ring entry may be published only after it landed.  The
+  // H2D's completion already waits for it (phys_complete), so this only matters
+  // for a job whose H2D failed.
   bool await_item_copy(Phys* ph, JobCtx* jc) {
     if (jc->item_cidx < 0) return true;
     const uint64_t t0 = mono_ns();
@@ -1231,6 +1232,12 @@ class Runtime : public strings::Hooks {
     if (engine != strings::ENG_KL) {
       const uint32_t d = lg.ctr->done[engine];
       if ((int32_t)(d - jc->copy_seq[engine]) < 0) return false;
+      // an H2D whose KL work item went through the copy partition is complete
+      // only once the item landed too (so the KL issue never waits for it)
+      if (engine == strings::ENG_H2D && jc->item_cidx >= 0) {
+        if (!copy_item_done(lg.phys, jc->item_cseq, jc->item_cidx)) return false;
+        jc->item_cidx = -1;
+      }
       std::atomic_thread_fence(std::memory_order_acquire);
       jc->phys_done[engine] = true;
       return true;

@@ -3,9 +3,10 @@
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 rm -f gpurun_out/item_ab.jsonl
+STRINGS_ITEM_VIA_COPY=1 timeout 600 python -m pytest tests -m gpu -x -q -k "small_copies or full_size" --timeout 300 --timeout-method=thread > gpurun_out/pt.log 2>&1; echo "pytest exit $?" >> gpurun_out/pt.log; tail -2 gpurun_out/pt.log
 for r in 1 2; do
   for v in 1 0; do
-    STRINGS_ITEM_VIA_COPY=$v BENCH_CONFIGS=C1,C3,C4,C2 timeout 900 python bench.py --configs --config-repeats 3 > gpurun_out/item_ab.log 2>&1
+    STRINGS_ITEM_VIA_COPY=$v STRINGS_STALL_DUMP_S=30 BENCH_CONFIGS=C1,C3,C4,C2 timeout 900 python bench.py --configs --config-repeats 3 > gpurun_out/item_ab.log 2>&1
     python - gpurun_out/item_ab.log $v $r >> gpurun_out/item_ab.jsonl <<'PY'
 import json,sys
 for l in open(sys.argv[1]):
