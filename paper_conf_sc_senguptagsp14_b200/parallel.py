@@ -43,6 +43,11 @@ def isolate_gpu(info: RankInfo) -> None:
         if shared_gpu_test():
             # every rank on the first device, each dispatcher on its own share of the SMs
             os.environ.setdefault("STRINGS_SM_LIMIT", str(148 // info.world))
+            # processes sharing a GPU time-slice their persistent kernels (separate
+            # contexts, no MPS): a copy-partition op waits for its context's slice
+            # (2 ranks: 1136-1193 jobs/s with copy engines only, 680-700 with the
+            # copy partition), so the shared-GPU test keeps every copy on the engines
+            os.environ.setdefault("STRINGS_COPY_CTAS", "0")
 
 
 def shared_gpu_test() -> bool:
