@@ -434,7 +434,9 @@ def run_strings(args, rank, world, torch, gloo):
             kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
                             "kl_host_us_p50": round(host[len(host) // 2], 1),
                             "h2d_host_us_p50": round(h2d[len(h2d) // 2], 1)}
-    kl_items = jobs_step * args.steps
+    # work items the persistent dispatcher executed in the timed steps: one KL item per
+    # job plus the copy partition's items (small H2D/D2H ops), an equal share per step
+    kl_items = jobs_step * args.steps + (stats.sm_copy_ops // (args.warmup + 2 * args.steps)) * args.steps
     res = {
         "metric": METRIC, "value": round(value, 3), "unit": "jobs/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt_max / args.steps * 1e3, 3),
@@ -459,7 +461,8 @@ def run_strings(args, rank, world, torch, gloo):
         "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step)",
         "phase_latency": kl_lat,
         "gpu_launches": kl_items,
-        "gpu_launches_note": "KL work items executed by the persistent dispatcher kernel (launched once at init)"
+        "gpu_launches_note": "work items executed by the persistent dispatcher kernel (launched once at init): "
+                             "KL items plus copy-partition items"
                              if args.kl_mode == 0 else "per-job tenant kernel launches",
         "clocks": clk.summary(),
         "decisions_per_step": (stats.decisions // (args.warmup + 2 * args.steps)),   # warm-up + timed + continuous
