@@ -405,7 +405,8 @@ def run_strings(args, rank, world, torch, gloo):
         first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
         lastd[inf.tenant] = max(lastd.get(inf.tenant, 0), inf.t_done[2])
     xs = [busy[t] / max(1, lastd[t] - first[t]) / wl.tenants[t].weight for t in busy]
-    jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par_
+    jain = par_.jain(par_.gather_over_ranks(gloo, xs))       # over the tenants of all ranks
     # mean completion latency per tenant in the last timed step (all jobs
     # submitted at the start of the step), for the weighted speedup
     step_t0 = min(inf.t_arrival for inf in last)
@@ -420,6 +421,7 @@ def run_strings(args, rank, world, torch, gloo):
     for cls, name in ((W.GEMM, "GEMM"), (W.XFER, "XFER")):
         rows = [inf for inf, spec in zip(timed, wl.jobs * args.steps) if spec.kclass == cls]
         dev = sorted((r.kl_gpu_end_ns - r.kl_gpu_start_ns) / 1e3 for r in rows)
+        body = sorted((r.kl_gpu_end_ns - r.kl_gpu_exec_ns) / 1e3 for r in rows if r.kl_gpu_exec_ns)
         host = sorted((r.t_done[1] - r.t_start[1]) / 1e3 for r in rows)
         h2d = sorted((r.t_done[0] - r.t_start[0]) / 1e3 for r in rows)
         if dev and name == "XFER":
@@ -432,6 +434,7 @@ def run_strings(args, rank, world, torch, gloo):
                                             "half_bidir_peak": round(link["bidir_gbs"] / 2, 2)}
         if dev:
             kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
+                            "kl_body_us_p50": round(body[len(body) // 2], 1) if body else None,
                             "kl_host_us_p50": round(host[len(host) // 2], 1),
                             "h2d_host_us_p50": round(h2d[len(h2d) // 2], 1)}
     # work items the persistent dispatcher executed in the timed steps: one KL item per
@@ -458,7 +461,8 @@ def run_strings(args, rank, world, torch, gloo):
         "kernel_rooflines": krl,
         "_mean_latency_s_by_tenant": mlat,
         "jain": round(jain, 4),
-        "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step)",
+        "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step), "
+                           "all tenants of all ranks",
         "phase_latency": kl_lat,
         "gpu_launches": kl_items,
         "gpu_launches_note": "work items executed by the persistent dispatcher kernel (launched once at init): "
@@ -500,7 +504,8 @@ def arm_config(cfg, jobs_step: int, world: int, kl_mode: int) -> dict:
 
 def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
     """The dominant kernel work inside the timed step: XFER items run by the
-    persistent dispatcher on one P=2 SM partition (74 SMs), HBM-bound.
+    persistent dispatcher on one P=2 SM partition (72 SMs beside the 4-CTA copy
+    partition), HBM-bound.
     achieved = algorithmic bytes per item (read + write) / median device time
     of the item (%globaltimer claim -> last CTA done).  Beside it: the same body
     launched stand-alone on the same CTA count at the same size (measured in
@@ -516,9 +521,15 @@ def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
            "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": _XFER_ITEM_NCU["dram_bytes"],
            "traffic_source": _XFER_ITEM_NCU["source"],
-           "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (74 of 148 SMs); the other "
+           "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (72 of 148 SMs); the other "
            "partition often runs an item concurrently and shares HBM; device time includes the partition "
            "broadcast and completion publish (stand-alone full-GPU runs: kernel_rooflines)"}
+    if x.get("kl_body_us_p50"):
+        # the body alone (leader's body start -> last CTA done): without the claim and
+        # the partition broadcast, which are dispatch cost, not kernel work
+        bg = 8 * n / (x["kl_body_us_p50"] * 1e3)
+        out["body_only"] = {"achieved": round(bg, 1), "frac": round(bg / peaks["hbm_gbs"], 4),
+                            "us": x["kl_body_us_p50"]}
     same = sorted((k for k in (krl or []) if k.get("ctas") and k["kernel"] == "XFER"), key=lambda k: k["ctas"])
     if same:
         out["same_work_standalone"] = {"ctas": same[0]["ctas"], "GBps": same[0]["achieved"],

@@ -142,6 +142,22 @@ def sum_over_ranks(group, x: float) -> float:
     return float(t.item())
 
 
+def gather_over_ranks(group, xs: List[float]) -> List[float]:
+    """Concatenation of every rank's list (rank order), e.g. per-tenant fairness
+    inputs, so whole-job metrics (Jain over all N x 16 tenants) are computed once."""
+    if group is None:
+        return list(xs)
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, list(xs), group=group)
+    return [x for part in out for x in part]
+
+
+def jain(xs: List[float]) -> float:
+    """Jain's index (Eq. 3, reading R-2): (sum x)^2 / (n sum x^2), in [1/n, 1]."""
+    return sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs)) if xs else 1.0
+
+
 def shard_tenants(num_tenants: int, world: int, rank: int) -> List[int]:
     """Tenants of this rank under strong scaling (round robin, like GRR)."""
     return [t for t in range(num_tenants) if t % world == rank]

@@ -50,6 +50,8 @@ def _worker(rank, world, port, q):
         span = max(i.t_done[2] for i in r.infos)
         mx = par.max_over_ranks(g, float(span))
         tot = par.sum_over_ranks(g, float(len(wl.jobs)))
+        allx = par.gather_over_ranks(g, [float(rank)] * (rank + 1))
+        assert allx == [0.0, 1.0, 1.0], allx                 # rank order, every rank's entries
         q.put((rank, same, span, mx, tot, r.stats.jobs_done))
         import torch.distributed as dist
         dist.destroy_process_group()
@@ -81,3 +83,14 @@ def test_shard_tenants_partition():
         parts = [par.shard_tenants(64, world, r) for r in range(world)]
         flat = sorted(t for p in parts for t in p)
         assert flat == list(range(64))
+
+
+def test_whole_job_jain_helper():
+    # the bench's whole-job Jain (Eq. 3, reading R-2): equal shares -> 1, one
+    # tenant served of n -> 1/n, scale-invariant; single-rank gather is identity
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    assert par.jain([0.3] * 7) == pytest.approx(1.0)
+    assert par.jain([0.0, 0.0, 2.5, 0.0]) == pytest.approx(0.25)
+    xs = [0.1, 0.4, 0.2]
+    assert par.jain(xs) == pytest.approx(par.jain([10 * x for x in xs]))
+    assert par.gather_over_ranks(None, xs) == xs
