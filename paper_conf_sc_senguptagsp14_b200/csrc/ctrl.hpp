@@ -109,6 +109,9 @@ __device__ __forceinline__ void copy_body(const CopyItem& c, int rank, int S) {
     }
     for (; i < n16; i += nthr) dst[i] = c.to_host ? ld_cg_v4(src + i) : ld_cv_v4(src + i);
   }
+  // every thread orders its own host-memory stores before the CTA counts in (the
+  // last CTA's completion word must not overtake any of them over PCIe)
+  if (c.to_host) __threadfence_system();
 }
 
 struct DispatchParams {
