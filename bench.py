@@ -1023,6 +1023,10 @@ def main():
         return
     par.isolate_gpu(info)                 # one process per GPU (before CUDA init)
     numa = par.bind_to_gpu_numa_node(par.physical_gpu(info))
+    if world > 1 and "STRINGS_COPY_THREADS" not in os.environ:
+        # ranks bound to the same CPUs share them: each rank's PMT copy pool gets its share
+        os.environ["STRINGS_COPY_THREADS"] = str(par.copy_threads_per_rank(info))
+        numa["copy_threads"] = int(os.environ["STRINGS_COPY_THREADS"])
     import torch
     gloo = par.init_groups(info, device_backend="nccl")
     res, wl = run_strings(args, rank, world, torch, gloo)

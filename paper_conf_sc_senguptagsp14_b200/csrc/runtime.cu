@@ -15,6 +15,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <immintrin.h>
+#include <sched.h>
 #include <time.h>
 #include <unistd.h>
 
@@ -449,11 +450,16 @@ uint64_t sm_copy_max_env() {
   return e ? strtoull(e, nullptr, 0) : (1ull << 20);
 }
 
-// PMT staging copy threads: most of the host's cores (the engine thread and the
-// caller keep one each); STRINGS_COPY_THREADS overrides.
+// PMT staging copy threads: most of the cores this process may run on (its
+// affinity mask, e.g. the GPU's NUMA node; the engine thread and the caller
+// keep one each); STRINGS_COPY_THREADS overrides (bench.py divides a node's
+// cores among the ranks that share it).
 int copy_threads() {
   if (const char* e = getenv("STRINGS_COPY_THREADS")) return std::max(0, atoi(e));
-  const int hw = (int)std::thread::hardware_concurrency();
+  int hw = (int)std::thread::hardware_concurrency();
+  cpu_set_t set;
+  CPU_ZERO(&set);
+  if (sched_getaffinity(0, sizeof set, &set) == 0 && CPU_COUNT(&set) > 0) hw = CPU_COUNT(&set);
   return std::min(12, std::max(2, hw - 4));
 }
 

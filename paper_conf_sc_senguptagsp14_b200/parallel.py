@@ -26,11 +26,14 @@ class RankInfo:
     rank: int
     world: int
     local_rank: int
+    local_world: int = 1          # ranks on this node (torchrun's LOCAL_WORLD_SIZE)
 
 
 def rank_info() -> RankInfo:
-    return RankInfo(int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
-                    int(os.environ.get("LOCAL_RANK", os.environ.get("RANK", "0"))))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    return RankInfo(int(os.environ.get("RANK", "0")), world,
+                    int(os.environ.get("LOCAL_RANK", os.environ.get("RANK", "0"))),
+                    int(os.environ.get("LOCAL_WORLD_SIZE", str(world))))
 
 
 def isolate_gpu(info: RankInfo) -> None:
@@ -140,6 +143,17 @@ def sum_over_ranks(group, x: float) -> float:
     t = torch.tensor([x], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return float(t.item())
+
+
+def copy_threads_per_rank(info: RankInfo) -> int:
+    """PMT staging threads for one rank when several ranks run on one node: the
+    CPUs this rank may use, shared by the node's ranks bound to the same CPUs
+    (all local ranks when the NUMA binding was a no-op), minus the engine and
+    caller threads; at most the library's default of 12."""
+    cpus = len(os.sched_getaffinity(0))
+    total = max(cpus, os.cpu_count() or cpus)
+    sharing = max(1, round(info.local_world * cpus / total))   # ranks bound to these same CPUs
+    return max(2, min(12, cpus // sharing - 2))
 
 
 def gather_over_ranks(group, xs: List[float]) -> List[float]:

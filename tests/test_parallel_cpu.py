@@ -94,3 +94,17 @@ def test_whole_job_jain_helper():
     xs = [0.1, 0.4, 0.2]
     assert par.jain(xs) == pytest.approx(par.jain([10 * x for x in xs]))
     assert par.gather_over_ranks(None, xs) == xs
+
+
+def test_copy_threads_per_rank(monkeypatch):
+    # 8 ranks on one node share its CPUs: each PMT copy pool gets its share
+    from paper_conf_sc_senguptagsp14_b200 import parallel as par
+    monkeypatch.setattr(par.os, "sched_getaffinity", lambda pid: set(range(224)))
+    monkeypatch.setattr(par.os, "cpu_count", lambda: 224)
+    assert par.copy_threads_per_rank(par.RankInfo(0, 8, 0, 8)) == 12          # 28 CPUs each -> capped
+    monkeypatch.setattr(par.os, "sched_getaffinity", lambda pid: set(range(112)))   # bound to 1 of 2 nodes
+    assert par.copy_threads_per_rank(par.RankInfo(0, 8, 0, 8)) == 12
+    monkeypatch.setattr(par.os, "sched_getaffinity", lambda pid: set(range(16)))
+    monkeypatch.setattr(par.os, "cpu_count", lambda: 16)
+    assert par.copy_threads_per_rank(par.RankInfo(0, 4, 0, 4)) == 2            # 4 CPUs each
+    assert par.copy_threads_per_rank(par.RankInfo(0, 1, 0, 1)) == 12
