@@ -37,6 +37,14 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "tenant jobs/sec (8xB200) vs static CUDA provisioning; Jain fairness"
+# The paper's headline ratios, quoted with their hardware as context only.
+PAPER_CONTEXT = {
+    "weighted_speedup_vs_cuda_runtime": {"PS": 6.41, "DTF": 8.06, "MBF": 8.70},
+    "fairness_gain_vs_cuda_runtime": "13% (TFS-Strings, average Jain 91%)",
+    "hardware": "2 nodes x 2 Fermi GPUs (Quadro 2000/4000, Tesla C2050/C2070), CUDA 5.0, 4-GPU supernode "
+                "over GigE; CUDA SDK/Rodinia app pairs",
+    "citations": "PAPER.md L29, L43, L879, L957, L1155",
+    "note": "relative figures on other hardware and workloads: context, not a target (vs_baseline is null)"}
 
 
 def parse_args():
@@ -1032,6 +1040,7 @@ def main():
     res, wl = run_strings(args, rank, world, torch, gloo)
     if rank == 0:
         res["config"]["host_numa"] = numa
+        res["paper_context"] = PAPER_CONTEXT
         if world == 1 and not args.no_static:
             from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
             sb = run_static(wl, num_gpus=1, repeats=args.static_repeats)
