@@ -20,6 +20,26 @@
  *    library (per-GPU arena of resident job slots).
  *  - Times are ns on the library clock: CLOCK_MONOTONIC since strings_init in
  *    MEASURED mode, the virtual clock in INJECTED / DECISIONS_ONLY mode.
+ *
+ * Environment knobs (read at strings_init; none changes a decision, only how
+ * the decided ops execute; DESIGN.md §2 and §11 give the measurements):
+ *   STRINGS_COPY_CTAS=n      SMs of the persistent kernel serving small H2D/D2H
+ *                            ops as zero-copy SM copies (default 4; 0 = every
+ *                            copy on the copy engines)
+ *   STRINGS_SM_COPY_MAX=b    largest op (bytes, all buffers) sent to those SMs
+ *                            (default 1 MiB); host buffers must be mapped pinned
+ *                            memory, 16-B aligned, sizes multiples of 16
+ *   STRINGS_ITEM_VIA_COPY=1  also send KL work items of copy-engine jobs there
+ *   STRINGS_COPY_STREAMS=physical  one H2D and one D2H stream per GPU instead of
+ *                            per logical device
+ *   STRINGS_COPY_THREADS=n   host threads of the pageable-buffer staging pool
+ *   STRINGS_NT_COPY=0|1|2|3  staging copy loop: memcpy | SSE2 (default) | AVX2 |
+ *                            AVX-512 non-temporal stores
+ *   STRINGS_SM_LIMIT=n       run the persistent kernel on n SMs (tests)
+ *   STRINGS_POLL_MAX_NS=ns   idle-poll back-off cap of partition leaders (1024)
+ *   STRINGS_STALL_DUMP_S=s   print in-flight ops to stderr if none completes
+ *                            for s seconds (default 20)
+ *   STRINGS_FAULT_JOB=id     inject a device fault in that job's KL (tests)
  */
 #ifndef STRINGS_SCHED_H
 #define STRINGS_SCHED_H
