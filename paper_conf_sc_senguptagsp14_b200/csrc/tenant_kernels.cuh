@@ -123,15 +123,31 @@ __device__ void stream_ldg(const uint32_t* __restrict__ x, uint32_t* __restrict_
   for (uint64_t e = e0 + nvec * 4 + tid; e < e1; e += nthreads) y[e] = elem_op<KCLASS>(x[e], alpha, seed);
 }
 
+// 6 x 32 KB stages, loads 4 chunks ahead, one bulk store allowed in flight
+// while its stage is refilled two iterations later (profiles/r01_stream_lead.jsonl:
+// the fastest race-free shape, XFER 2^24 on 74 SMs 29.2 us, 2^28 on 148 SMs 0.95
+// of peak; 4 x 48 KB with a 3-chunk lead must wait for every store to read out
+// (34.8 us)).
 #ifndef STRINGS_STREAM_STAGES
-#define STRINGS_STREAM_STAGES 4
+#define STRINGS_STREAM_STAGES 6
 #endif
 #ifndef STRINGS_STREAM_CHUNK_KB
-#define STRINGS_STREAM_CHUNK_KB 48
+#define STRINGS_STREAM_CHUNK_KB 32
+#endif
+#ifndef STRINGS_STREAM_LEAD
+#define STRINGS_STREAM_LEAD (STRINGS_STREAM_STAGES - 2)
 #endif
 constexpr int kStreamStages = STRINGS_STREAM_STAGES;                 // stage count (<= 12 mbarriers in the tail)
-constexpr uint32_t kStreamChunk = STRINGS_STREAM_CHUNK_KB * 1024;    // bytes per stage (4 x 48 KB = 192 KB)
+constexpr uint32_t kStreamChunk = STRINGS_STREAM_CHUNK_KB * 1024;    // bytes per stage (6 x 32 KB = 192 KB)
+// Loads run kStreamLead chunks ahead of the chunk being processed.  The stage a
+// new load refills was last stored by the chunk kStreamStages - kStreamLead
+// iterations back; before the load overwrites it, that bulk store must have
+// finished READING shared memory, i.e. at most kStreamStages - kStreamLead - 1
+// newer store groups may still be pending (cp.async.bulk.wait_group.read N).
+constexpr int kStreamLead = STRINGS_STREAM_LEAD;
+constexpr int kStreamStoreSlack = kStreamStages - kStreamLead - 1;
 static_assert(kStreamStages >= 3 && kStreamStages <= 12, "stream stages");
+static_assert(kStreamLead >= 1 && kStreamLead < kStreamStages, "stream lead");
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(
@@ -148,12 +164,12 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
-// Streaming body: the buffer is cut into 48 KB chunks; chunk c belongs to CTA
-// (c mod S).  Each CTA runs a 4-stage TMA bulk-copy pipeline through shared
+// Streaming body: the buffer is cut into 32 KB chunks; chunk c belongs to CTA
+// (c mod S).  Each CTA runs a 6-stage TMA bulk-copy pipeline through shared
 // memory (cp.async.bulk global->smem with mbarrier completion, the element op
-// in smem, cp.async.bulk smem->global), keeping ~192 KB of loads in flight per
-// SM: one half-GPU partition saturates HBM.  Unaligned buffers and the tail
-// use the LDG path.
+// in smem, cp.async.bulk smem->global), keeping 4 chunks (128 KB) of loads in
+// flight per SM while the previous chunk's store drains.  Unaligned buffers
+// and the tail use the LDG path.
 template <int KCLASS>
 __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
                             float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar) {
@@ -170,19 +186,21 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
     const uint8_t* xb = reinterpret_cast<const uint8_t*>(x);
     uint8_t* yb = reinterpret_cast<uint8_t*>(y);
     if (threadIdx.x == 0)
-      for (int s = 0; s < kStreamStages - 1 && (uint64_t)s < my; ++s) {
+      for (int s = 0; s < kStreamLead && (uint64_t)s < my; ++s) {
         mbar_expect_tx(&sbar[s], kStreamChunk);
         bulk_g2s(stage + s * kStreamChunk, xb + (rank + (uint64_t)s * S) * kStreamChunk, kStreamChunk, &sbar[s]);
       }
     for (uint64_t i = 0; i < my; ++i) {
       const int s = (int)(i % kStreamStages);
       const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
-      if (threadIdx.x == 0 && i + kStreamStages - 1 < my) {
-        const int s2 = (int)((i + kStreamStages - 1) % kStreamStages);
-        // the bulk store that last used stage s2 (issued at iteration i-1) must have read smem
-        asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStages - 2) : "memory");
+      if (threadIdx.x == 0 && i + kStreamLead < my) {
+        const int s2 = (int)((i + kStreamLead) % kStreamStages);
+        // stage s2 was last stored at iteration i + kStreamLead - kStreamStages: that
+        // store must have finished reading smem before the load overwrites it
+        if (i + kStreamLead >= (uint64_t)kStreamStages)
+          asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStoreSlack) : "memory");
         mbar_expect_tx(&sbar[s2], kStreamChunk);
-        bulk_g2s(stage + s2 * kStreamChunk, xb + (rank + (i + kStreamStages - 1) * S) * kStreamChunk,
+        bulk_g2s(stage + s2 * kStreamChunk, xb + (rank + (i + kStreamLead) * S) * kStreamChunk,
                  kStreamChunk, &sbar[s2]);
       }
       mbar_wait(&sbar[s], ph);
