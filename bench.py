@@ -437,8 +437,8 @@ def run_strings(args, rank, world, torch, gloo):
             # (>= 90% of the measured pinned peak; here vs half the bidir peak)
             d2h = sorted((r.t_done[2] - r.t_start[2]) / 1e3 for r in rows)
             nb = 4 * [j for j in wl.jobs if j.kclass == W.XFER][0].n
-            kl_lat["XFER_copy_GBps_p50"] = {"h2d": round(nb / (h2d[len(h2d) // 2] * 1e3), 2),
-                                            "d2h": round(nb / (d2h[len(d2h) // 2] * 1e3), 2),
+            kl_lat["XFER_copy_GBps_p50"] = {"h2d": round(nb / max(1e-3, h2d[len(h2d) // 2] * 1e3), 2),
+                                            "d2h": round(nb / max(1e-3, d2h[len(d2h) // 2] * 1e3), 2),
                                             "half_bidir_peak": round(link["bidir_gbs"] / 2, 2)}
         if dev:
             kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
@@ -549,9 +549,9 @@ def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
 # ncu --set full of the C2 work item's body as a stand-alone launch (XFER 2^24 u32
 # on 74 CTAs, `tools/kernel_probe.py xfer_item`): dram__bytes_read.sum +
 # dram__bytes_write.sum per launch; see profiles/r01_kernels.md.
-# Reads 67.18 MB = the 64 MiB input exactly; writes 20.27 MB of 67.1 MB: at this size
+# Reads 67.18 MB = the 64 MiB input exactly; writes 21.33 MB of 67.1 MB: at this size
 # most of the output is still in the 126 MB L2 when the launch ends (no re-reads).
-_XFER_ITEM_NCU = {"dram_bytes": 67181056 + 20273664,
+_XFER_ITEM_NCU = {"dram_bytes": 67181056 + 21326336,
                   "source": "profiles/r01_kernels.md (xfer_item: ncu --set full, XFER 2^24 on 74 CTAs)"}
 
 
