@@ -243,8 +243,12 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
 constexpr int kTileM = 128, kTileN = 256, kMaxK = 256;
 constexpr uint32_t kSmemA = kTileM * kMaxK * 2;          // 64 KB
 constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
-constexpr uint32_t kSmemGemm = kSmemA + kSmemB + 128;    // + mbarriers / tmem slot (tail, see carve_smem)
-static_assert(kStreamStages * kStreamChunk <= kSmemA + kSmemB, "streaming stages alias the GEMM operand smem");
+// The streaming stages alias the GEMM operand smem (and may extend past it); the
+// 128-B tail of mbarriers / TMEM slot sits after the larger of the two.
+constexpr uint32_t kSmemMain = (kStreamStages * kStreamChunk > kSmemA + kSmemB) ? kStreamStages * kStreamChunk
+                                                                                 : kSmemA + kSmemB;
+constexpr uint32_t kSmemGemm = kSmemMain + 128;          // dynamic smem of the dispatcher / one-shot kernels
+static_assert(kSmemGemm + 2048 <= 227 * 1024, "dynamic + static smem must fit one CTA per SM");
 constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
 constexpr uint32_t kSlabA = 128 * 128;                   // 16 KB
 constexpr uint32_t kSlabB = 256 * 128;                   // 32 KB
@@ -628,7 +632,7 @@ __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   GemmSmem s;
   s.a = base;
   s.b = base + kSmemA;
-  uint8_t* tail = base + kSmemA + kSmemB;
+  uint8_t* tail = base + kSmemMain;
   s.bar = reinterpret_cast<uint64_t*>(tail);
   s.tmem_slot = reinterpret_cast<uint32_t*>(tail + 8);
   s.stage = base;

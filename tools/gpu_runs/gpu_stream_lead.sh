@@ -4,7 +4,7 @@ cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 : > gpurun_out/stream_lead.jsonl
 cp /dev/null gpurun_out/stream_lead2.jsonl
-for v in "6 32 4" "6 32 3" "7 27 5" "5 38 3" "12 16 10" "4 48 2"; do
+for v in "6 32 4" "7 32 5" "7 32 4" "6 36 4" "4 56 2"; do
   set -- $v
   export STRINGS_NVCC_EXTRA="-DSTRINGS_STREAM_STAGES=$1 -DSTRINGS_STREAM_CHUNK_KB=$2 -DSTRINGS_STREAM_LEAD=$3"
   python -m paper_conf_sc_senguptagsp14_b200.build --force > /dev/null 2>&1 || { echo "{\"build_failed\": \"$v\"}" >> gpurun_out/stream_lead.jsonl; continue; }
