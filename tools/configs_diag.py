@@ -95,6 +95,22 @@ def main():
         iv = [(i.t_start[x], i.t_done[x]) for i in infos if i.t_done[x] > i.t_start[x]]
         res[f"{name}_union_occupancy"] = round(union_len(iv) / span, 4)
         res[f"{name}_mean_concurrency"] = round(sum(e - s for s, e in iv) / max(1, union_len(iv)), 2)
+    # KL path under load: host issue -> leader claim -> body start -> last CTA -> host observe
+    off = stats.gpu_clock_offset_ns[0]
+    for cname in sorted({W.CLASS_NAMES[sp.kclass] for sp in wl.jobs}):
+        ii = [i for sp, i in zip(wl.jobs, infos) if W.CLASS_NAMES[sp.kclass] == cname and i.kl_gpu_start_ns]
+        if not ii or not off:
+            continue
+
+        def med(v):
+            v = sorted(v)
+            return round(v[len(v) // 2] / 1e3, 1)
+        res[f"{cname}_kl_path_us_p50"] = {
+            "issue_to_claim": med([i.kl_gpu_start_ns - off - i.kl_host_issue_ns for i in ii]),
+            "claim_to_exec": med([i.kl_gpu_exec_ns - i.kl_gpu_start_ns for i in ii]),
+            "exec_to_end": med([i.kl_gpu_end_ns - i.kl_gpu_exec_ns for i in ii]),
+            "end_to_observe": med([i.kl_host_observe_ns - (i.kl_gpu_end_ns - off) for i in ii]),
+            "model_start_to_done": med([i.t_done[1] - i.t_start[1] for i in ii])}
     by = {}
     for sp, i in zip(wl.jobs, infos):
         d = by.setdefault(W.CLASS_NAMES[sp.kclass], {"h2d": [], "kl": [], "d2h": [], "wait": [], "bytes": sum(sp.h2d_sizes())})
