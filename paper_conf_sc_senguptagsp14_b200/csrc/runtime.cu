@@ -1347,13 +1347,13 @@ class Runtime : public strings::Hooks {
             stall_dumped = true;
             fprintf(stderr, "[strings] injected: waiting for job %llu engine %d (t = %llu)\n",
                     (unsigned long long)c.job, c.engine, (unsigned long long)t);
+            std::vector<std::pair<JobCtx*, int>> pending;
             for (size_t k = 0; k < jobs.size(); ++k) {
               JobCtx* o = jobs[k].get();
               for (int e = 0; e < 3; ++e)
-                if (o->issued[e] && !o->phys_done[e]) inflight.push_back({o, e});
+                if (o->issued[e] && !o->phys_done[e]) pending.push_back({o, e});
             }
-            dump_state();
-            inflight.clear();
+            dump_state(pending);
           }
           lk.unlock();
           std::this_thread::yield();
@@ -1416,7 +1416,7 @@ class Runtime : public strings::Hooks {
       }
       if (!inflight.empty() && !stall_dumped && mono_ns() - last_progress > stall_dump_ns) {
         stall_dumped = true;
-        dump_state();
+        dump_state(inflight);
       }
       lk.unlock();
       std::this_thread::yield();
@@ -1426,8 +1426,8 @@ class Runtime : public strings::Hooks {
 
   // Diagnostics: no op completed for STRINGS_STALL_DUMP_S seconds (default 20)
   // while ops are in flight -> print the in-flight ops and queue states once.
-  void dump_state() {
-    fprintf(stderr, "[strings] stall: %zu ops in flight, %llu/%llu jobs done\n", inflight.size(),
+  void dump_state(const std::vector<std::pair<JobCtx*, int>>& ops) {
+    fprintf(stderr, "[strings] stall: %zu ops in flight, %llu/%llu jobs done\n", ops.size(),
             (unsigned long long)done_count, (unsigned long long)submitted);
     for (auto& ph : phys)
       fprintf(stderr, "[strings]  gpu %d: copy ring tail %u completed %u, copy ctas %d\n", ph->dev, ph->ctail,
@@ -1436,7 +1436,7 @@ class Runtime : public strings::Hooks {
       fprintf(stderr, "[strings]  ld %d: KL tail %u completed %u, copies issued h2d %u d2h %u, done h2d %u d2h %u\n",
               lg.gid, lg.tail, lg.completed, lg.issued[0], lg.issued[2], lg.ctr ? lg.ctr->done[0] : 0,
               lg.ctr ? lg.ctr->done[2] : 0);
-    for (auto& f : inflight) {
+    for (auto& f : ops) {
       JobCtx* jc = f.first;
       const int e = f.second;
       const strings::Job& j = jc->job;
