@@ -178,7 +178,7 @@ struct JobCtx {
   uint32_t copy_seq[3] = {0, 0, 0};
   bool smcopy[3] = {false, false, false};          // op runs on the dispatcher's copy partition
   uint32_t item_cseq = 0;                          // KL work item copied by the copy partition
-  int item_cidx = -1;                              //   (CE-path H2D jobs), consumed at KL issue
+  int item_cidx = -1;                              //   (CE-path H2D jobs; STRINGS_ITEM_VIA_COPY), consumed with the H2D
   uint32_t cseq[3] = {0, 0, 0};
   int cidx[3] = {-1, -1, -1};
   int kl_idx = -1;
