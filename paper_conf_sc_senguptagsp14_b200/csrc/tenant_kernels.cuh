@@ -144,7 +144,14 @@ constexpr uint32_t kStreamChunk = STRINGS_STREAM_CHUNK_KB * 1024;    // bytes pe
 // iterations back; before the load overwrites it, that bulk store must have
 // finished READING shared memory, i.e. at most kStreamStages - kStreamLead - 1
 // newer store groups may still be pending (cp.async.bulk.wait_group.read N).
+// Minimum chunks per CTA for the pipeline (below: LDG path).  0 = always the
+// pipeline: at 4 MiB on 18-72 CTAs the two paths are within +-10% either way, only
+// 16 MiB on 72 CTAs gains from the LDG path (profiles/r01_small_item.jsonl).
+#ifndef STRINGS_STREAM_MIN_CHUNKS
+#define STRINGS_STREAM_MIN_CHUNKS 0
+#endif
 constexpr int kStreamLead = STRINGS_STREAM_LEAD;
+constexpr int kStreamMinChunks = STRINGS_STREAM_MIN_CHUNKS;
 constexpr int kStreamStoreSlack = kStreamStages - kStreamLead - 1;
 static_assert(kStreamStages >= 3 && kStreamStages <= 12, "stream stages");
 static_assert(kStreamLead >= 1 && kStreamLead < kStreamStages, "stream lead");
@@ -175,7 +182,10 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
                             float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar) {
   const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   const uint64_t bytes = n * 4;
-  const uint64_t nchunks = aligned ? bytes / kStreamChunk : 0;
+  // items too small to fill the pipeline (fewer than kStreamMinChunks chunks per CTA)
+  // take the LDG path, whose first loads go out without a pipeline fill
+  const uint64_t nchunks =
+      aligned && bytes / kStreamChunk >= (uint64_t)S * kStreamMinChunks ? bytes / kStreamChunk : 0;
   if (nchunks) {
     const uint64_t my = (uint64_t)rank < nchunks ? (nchunks - 1 - rank) / S + 1 : 0;
     if (threadIdx.x == 0) {
