@@ -222,3 +222,23 @@ def test_product_path_never_imports_the_oracle():
         for node in ast.walk(fn):
             if isinstance(node, ast.ImportFrom) and node.module and node.module.split(".")[0] == "oracle":
                 assert fn.name in allowed, fn.name
+
+
+@pytest.mark.parametrize("pyname,cname", [("Config", "strings_config_t"), ("KernelDesc", "strings_kernel_desc_t"),
+                                          ("Buf", "strings_buf_t"), ("JobInfo", "strings_job_info_t"),
+                                          ("Stats", "strings_stats_t")])
+def test_binding_structs_match_the_header_layout(pyname, cname, tmp_path):
+    # the ctypes mirrors in strings.py must have the C structs' size and every
+    # field at the C offset (a drifted binding would read or write past the struct)
+    st = getattr(S, pyname)
+    names = [f[0] for f in st._fields_]
+    src = tmp_path / "layout.c"
+    body = "\n".join(f'  printf("%zu\\n", offsetof({cname}, {n}));' for n in names)
+    src.write_text(f'#include <stdio.h>\n#include <stddef.h>\n#include "strings_sched.h"\n'
+                   f'int main(void) {{\n  printf("%zu\\n", sizeof({cname}));\n{body}\n  return 0;\n}}\n')
+    exe = tmp_path / "layout"
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include")
+    subprocess.run(["gcc", "-std=c11", "-I", inc, str(src), "-o", str(exe)], check=True)
+    out = [int(v) for v in subprocess.run([str(exe)], check=True, capture_output=True, text=True).stdout.split()]
+    assert out[0] == ctypes.sizeof(st), (cname, out[0], ctypes.sizeof(st))
+    assert out[1:] == [getattr(st, n).offset for n in names], cname
