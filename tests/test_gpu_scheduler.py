@@ -342,3 +342,26 @@ def test_job_exactly_filling_its_slot():
         assert S.drain() == S.OK and S.stats().jobs_submitted == 0
     finally:
         S.shutdown()
+
+
+def _ngpus():
+    import torch
+    return torch.cuda.device_count()
+
+
+@pytest.mark.parametrize("timing", [S.INJECTED, S.MEASURED])
+def test_node_mode_on_several_physical_gpus(timing):
+    # node mode across physical GPUs (the level-1 balancer places jobs on distinct
+    # devices, each with its own dispatcher, streams and copy partition): C3's four
+    # logical devices on min(4, #GPUs) GPUs.  Runs on multi-GPU boxes only.
+    n = _ngpus()
+    if n < 2:
+        pytest.skip("needs >= 2 GPUs")
+    wl = W.config_c3(scale=4)
+    r = run_workload(wl, timing_mode=timing, physical_gpus=min(4, n))
+    assert r.status == S.OK
+    if timing == S.INJECTED:
+        assert r.trace == run_oracle(wl).trace
+    assert invariants.check(r.trace, wl) == []
+    check_outputs(wl, r)
+    assert r.stats.physical_gpus == min(4, n)
