@@ -515,15 +515,40 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
   return v;
 }
 
+// Tiles of 256 threads x 32 consecutive elements (32 KB): each thread loads its
+// 32 with eight 16-B loads (all in flight at once), scans them in registers,
+// and the warp / CTA totals give its offset; chunks are whole tiles, so every
+// CTA's loads stay 16-B aligned when the buffers are.
+constexpr int kScanPT = 32;
 __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
                                  int S, GroupSync* gs, uint8_t* stage) {
   uint32_t* wsum = reinterpret_cast<uint32_t*>(stage);           // [8] warp totals + [1] broadcast
-  const uint64_t chunk = ((n + S - 1) / S + 7) & ~7ull;
+  constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;
+  const uint64_t chunk = ((n + S - 1) / S + kTile - 1) / kTile * kTile;
   const uint64_t b0 = min(n, (uint64_t)rank * chunk), b1 = min(n, b0 + chunk);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  // 1. chunk sum
+  const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
+  // 1. chunk sum (8 independent 16-B loads in flight per thread)
   uint32_t s = 0;
-  for (uint64_t e = b0 + threadIdx.x; e < b1; e += kThreads) s += x[e];
+  uint64_t tail = b0;
+  if (vec) {
+    const uint4* x4 = reinterpret_cast<const uint4*>(x + b0);
+    const uint64_t n4 = (b1 - b0) / 4;
+    uint64_t i = threadIdx.x;
+    for (; i + 7 * kThreads < n4; i += 8 * kThreads) {
+      uint4 q[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) q[u] = ld_stream(x4 + i + u * kThreads);
+#pragma unroll
+      for (int u = 0; u < 8; ++u) s += q[u].x + q[u].y + q[u].z + q[u].w;
+    }
+    for (; i < n4; i += kThreads) {
+      const uint4 q = ld_stream(x4 + i);
+      s += q.x + q.y + q.z + q.w;
+    }
+    tail = b0 + n4 * 4;
+  }
+  for (uint64_t e = tail + threadIdx.x; e < b1; e += kThreads) s += x[e];
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   if (lane == 0) wsum[warp] = s;
@@ -543,14 +568,24 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
   __syncthreads();
   uint32_t carry = wsum[8];
   __syncthreads();
-  // 3. tiles of 256 threads x 8 consecutive elements
-  for (uint64_t base = b0; base < b1; base += kThreads * 8) {
-    const uint64_t e0 = base + (uint64_t)threadIdx.x * 8;
-    uint32_t v[8];
+  // 3. tiles
+  for (uint64_t base = b0; base < b1; base += kTile) {
+    const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
+    const bool full = vec && e0 + kScanPT <= b1;
+    uint32_t v[kScanPT];
+    if (full) {
+#pragma unroll
+      for (int u = 0; u < kScanPT / 4; ++u) {
+        const uint4 q = reinterpret_cast<const uint4*>(x + e0)[u];
+        v[4 * u] = q.x; v[4 * u + 1] = q.y; v[4 * u + 2] = q.z; v[4 * u + 3] = q.w;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < kScanPT; ++i) v[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
+    }
     uint32_t run = 0;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      v[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
+    for (int i = 0; i < kScanPT; ++i) {
       run += v[i];
       v[i] = run;                                                   // thread-local inclusive
     }
@@ -563,10 +598,17 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
       if (w < warp) wpre += t;
       tile += t;
     }
-    const uint32_t excl = carry + wpre + incl - run;               // sum before this thread's 8
+    const uint32_t excl = carry + wpre + incl - run;               // sum before this thread's elements
+    if (full) {
 #pragma unroll
-    for (int i = 0; i < 8; ++i)
-      if (e0 + i < b1) y[e0 + i] = excl + v[i];
+      for (int u = 0; u < kScanPT / 4; ++u)
+        reinterpret_cast<uint4*>(y + e0)[u] =
+            make_uint4(excl + v[4 * u], excl + v[4 * u + 1], excl + v[4 * u + 2], excl + v[4 * u + 3]);
+    } else {
+#pragma unroll
+      for (int i = 0; i < kScanPT; ++i)
+        if (e0 + i < b1) y[e0 + i] = excl + v[i];
+    }
     carry += tile;
     __syncthreads();
   }
@@ -574,33 +616,79 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
 
 // ------------------------------------------- SORT (Table I: SN, batch sort)
 // Each consecutive segment of 2048 u32 keys is sorted ascending by a bitonic
-// sorting network in shared memory (CUDA SDK "sortingNetworks" shape).
+// sorting network (the CUDA SDK "sortingNetworks" workload shape).  Thread t
+// keeps keys [8t, 8t + 8) of the segment in registers for the whole network:
+// compare-exchange distance j < 8 is inside the thread, 8 <= j < 256 between
+// lanes of one warp (shuffles), and only j >= 256 (6 of the 66 stages) goes
+// through shared memory (padded one word per 32: conflict-free).  The element
+// at index a with partner a ^ j keeps min(v, p) when it is the lower index of
+// an ascending block ((a & k) == 0) or the higher index of a descending one.
 constexpr int kSortSeg = 2048;
+__device__ __forceinline__ int sort_pad(int a) { return a + (a >> 5); }
+
 __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
                                  int S, uint8_t* stage) {
-  uint32_t* key = reinterpret_cast<uint32_t*>(stage);
+  static_assert(kSortSeg == 8 * kThreads, "8 keys per thread");
+  uint32_t* key = reinterpret_cast<uint32_t*>(stage);            // [2048 + 64] padded
   const uint64_t nseg = n / kSortSeg;
+  const int t = threadIdx.x;
+  const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   for (uint64_t seg = rank; seg < nseg; seg += S) {
-    const uint32_t* src = x + seg * kSortSeg;
-    for (int i = threadIdx.x; i < kSortSeg; i += kThreads) key[i] = src[i];
-    __syncthreads();
-    for (int k = 2; k <= kSortSeg; k <<= 1) {
-      for (int j = k >> 1; j > 0; j >>= 1) {
-        for (int i = threadIdx.x; i < kSortSeg / 2; i += kThreads) {
-          const int a = ((i / j) * 2 * j) + (i % j), b = a + j;
-          const bool up = (a & k) == 0;
-          const uint32_t ka = key[a], kb = key[b];
-          if ((ka > kb) == up) {
-            key[a] = kb;
-            key[b] = ka;
+    const uint32_t* src = x + seg * kSortSeg + 8 * t;
+    uint32_t v[8];
+    if (vec) {
+      const uint4 q0 = ld_stream(reinterpret_cast<const uint4*>(src));
+      const uint4 q1 = ld_stream(reinterpret_cast<const uint4*>(src) + 1);
+      v[0] = q0.x; v[1] = q0.y; v[2] = q0.z; v[3] = q0.w;
+      v[4] = q1.x; v[5] = q1.y; v[6] = q1.z; v[7] = q1.w;
+    } else {
+#pragma unroll
+      for (int r = 0; r < 8; ++r) v[r] = src[r];
+    }
+#pragma unroll
+    for (int lk = 1; lk <= 11; ++lk) {
+      const int k = 1 << lk;
+#pragma unroll
+      for (int lj = lk - 1; lj >= 0; --lj) {
+        const int j = 1 << lj;
+        if (j >= 256) {                                              // across warps
+#pragma unroll
+          for (int r = 0; r < 8; ++r) key[sort_pad(8 * t + r)] = v[r];
+          __syncthreads();
+#pragma unroll
+          for (int r = 0; r < 8; ++r) {
+            const int a = 8 * t + r;
+            const uint32_t p = key[sort_pad(a ^ j)];
+            v[r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[r], p) : max(v[r], p);
+          }
+          __syncthreads();
+        } else if (j >= 8) {                                         // lanes t and t ^ (j / 8)
+#pragma unroll
+          for (int r = 0; r < 8; ++r) {
+            const int a = 8 * t + r;
+            const uint32_t p = __shfl_xor_sync(0xffffffffu, v[r], j >> 3);
+            v[r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[r], p) : max(v[r], p);
+          }
+        } else {                                                     // registers r and r + j
+#pragma unroll
+          for (int r = 0; r < 8; ++r) {
+            if (r & j) continue;
+            const bool asc = ((8 * t + r) & k) == 0;
+            const uint32_t lo = v[r], hi = v[r + j];
+            v[r] = asc ? min(lo, hi) : max(lo, hi);
+            v[r + j] = asc ? max(lo, hi) : min(lo, hi);
           }
         }
-        __syncthreads();
       }
     }
-    uint32_t* dst = y + seg * kSortSeg;
-    for (int i = threadIdx.x; i < kSortSeg; i += kThreads) dst[i] = key[i];
-    __syncthreads();
+    uint32_t* dst = y + seg * kSortSeg + 8 * t;
+    if (vec) {
+      reinterpret_cast<uint4*>(dst)[0] = make_uint4(v[0], v[1], v[2], v[3]);
+      reinterpret_cast<uint4*>(dst)[1] = make_uint4(v[4], v[5], v[6], v[7]);
+    } else {
+#pragma unroll
+      for (int r = 0; r < 8; ++r) dst[r] = v[r];
+    }
   }
 }
 
