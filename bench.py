@@ -237,6 +237,30 @@ def kernel_rooflines(torch, S, peaks) -> list:
     ref = (a.float() @ b.float())
     assert torch.equal(c, ref), "GEMM roofline run produced a wrong result"
     del a, b, c, ref
+    # NEXT-2 tenant kernels (pairwise mix): algorithmic bytes vs the HBM peak
+    n = 1 << 30
+    xb = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda")
+    hb = torch.zeros(256, dtype=torch.int32, device="cuda")
+    t = time_launch(S.make_desc(S.HIST, n=n), [xb], [hb])
+    gbs = (n + 1024) / t / 1e9
+    out.append({"kernel": "HIST", "bound": "hbm", "size": "n=2^30 bytes -> 256 bins", "achieved": round(gbs, 1),
+                "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": round(gbs / peaks["hbm_gbs"], 4),
+                "ms": round(t * 1e3, 4), "note": "shared-memory atomics bound (per-warp sub-histograms)"})
+    del xb, hb
+    n = 1 << 28
+    xs = torch.randint(0, 1 << 20, (n,), dtype=torch.int32, device="cuda")
+    ys = torch.empty_like(xs)
+    for cls, name, bound in ((S.SCAN, "SCAN", "hbm"), (S.SORT, "SORT", "alu")):
+        t = time_launch(S.make_desc(cls, n=n), [xs], [ys])
+        gbs = 8 * n / t / 1e9
+        out.append({"kernel": name, "bound": bound, "size": "n=2^28 u32" + (", 2048-key segments" if name == "SORT"
+                                                                              else ""),
+                    "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                    "frac": round(gbs / peaks["hbm_gbs"], 4), "ms": round(t * 1e3, 4),
+                    **({"note": "bitonic network, 66 compare-exchange stages per segment: ALU/shuffle bound; "
+                                "frac is of the HBM peak, for context"} if name == "SORT" else
+                       {"note": "reduce-then-scan: reads the input twice (12n bytes moved for 8n algorithmic)"})})
+    del xs, ys
     torch.cuda.empty_cache()
     return out
 

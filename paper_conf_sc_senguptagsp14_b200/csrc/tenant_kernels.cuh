@@ -568,21 +568,29 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
   __syncthreads();
   uint32_t carry = wsum[8];
   __syncthreads();
-  // 3. tiles
+  // 3. tiles; the next tile's 32 elements are loaded while this one is scanned
+  auto load_tile = [&](uint64_t base, uint32_t* w) {
+    const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
+    if (vec && e0 + kScanPT <= b1) {
+#pragma unroll
+      for (int u = 0; u < kScanPT / 4; ++u) {
+        const uint4 q = reinterpret_cast<const uint4*>(x + e0)[u];
+        w[4 * u] = q.x; w[4 * u + 1] = q.y; w[4 * u + 2] = q.z; w[4 * u + 3] = q.w;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < kScanPT; ++i) w[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
+    }
+  };
+  uint32_t nxt[kScanPT];
+  if (b0 < b1) load_tile(b0, nxt);
   for (uint64_t base = b0; base < b1; base += kTile) {
     const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
     const bool full = vec && e0 + kScanPT <= b1;
     uint32_t v[kScanPT];
-    if (full) {
 #pragma unroll
-      for (int u = 0; u < kScanPT / 4; ++u) {
-        const uint4 q = reinterpret_cast<const uint4*>(x + e0)[u];
-        v[4 * u] = q.x; v[4 * u + 1] = q.y; v[4 * u + 2] = q.z; v[4 * u + 3] = q.w;
-      }
-    } else {
-#pragma unroll
-      for (int i = 0; i < kScanPT; ++i) v[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
-    }
+    for (int i = 0; i < kScanPT; ++i) v[i] = nxt[i];
+    if (base + kTile < b1) load_tile(base + kTile, nxt);
     uint32_t run = 0;
 #pragma unroll
     for (int i = 0; i < kScanPT; ++i) {
@@ -633,18 +641,25 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
   const uint64_t nseg = n / kSortSeg;
   const int t = threadIdx.x;
   const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
-  for (uint64_t seg = rank; seg < nseg; seg += S) {
+  auto load8 = [&](uint64_t seg, uint32_t* w) {
     const uint32_t* src = x + seg * kSortSeg + 8 * t;
-    uint32_t v[8];
     if (vec) {
       const uint4 q0 = ld_stream(reinterpret_cast<const uint4*>(src));
       const uint4 q1 = ld_stream(reinterpret_cast<const uint4*>(src) + 1);
-      v[0] = q0.x; v[1] = q0.y; v[2] = q0.z; v[3] = q0.w;
-      v[4] = q1.x; v[5] = q1.y; v[6] = q1.z; v[7] = q1.w;
+      w[0] = q0.x; w[1] = q0.y; w[2] = q0.z; w[3] = q0.w;
+      w[4] = q1.x; w[5] = q1.y; w[6] = q1.z; w[7] = q1.w;
     } else {
 #pragma unroll
-      for (int r = 0; r < 8; ++r) v[r] = src[r];
+      for (int r = 0; r < 8; ++r) w[r] = src[r];
     }
+  };
+  uint32_t nxt[8];
+  if ((uint64_t)rank < nseg) load8(rank, nxt);
+  for (uint64_t seg = rank; seg < nseg; seg += S) {
+    uint32_t v[8];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) v[r] = nxt[r];
+    if (seg + S < nseg) load8(seg + S, nxt);                       // next segment's loads fly during this sort
 #pragma unroll
     for (int lk = 1; lk <= 11; ++lk) {
       const int k = 1 << lk;
