@@ -121,6 +121,17 @@ def test_hist_single_bin_contention():
     assert h[7] == x.size and h.sum() == x.size
 
 
+@pytest.mark.parametrize("ctas", [1, 3])
+def test_hist_counter_flush_one_bin(ctas):
+    # one CTA sees > 65535 copies of one byte per lane: the 16-bit lane counters
+    # must be flushed before they wrap (every 4095 16-B loads)
+    n = (1 << 24) * 2 // ctas + 77
+    x = np.full(n, 200, np.uint8)
+    x[::4097] = 3
+    (h,) = _launch(S.make_desc(S.HIST, n=n), [x], [np.zeros(256, np.uint32)], ctas)
+    assert np.array_equal(h, K.hist(x))
+
+
 @pytest.mark.parametrize("n", [0, 1, 7, 8, 2047, 2049, 100_003, (1 << 22) + 5])
 @pytest.mark.parametrize("ctas", [0, 1, 5, 148])
 def test_scan_bit_exact(n, ctas):
