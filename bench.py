@@ -257,7 +257,8 @@ def kernel_rooflines(torch, S, peaks) -> list:
                                                                               else ""),
                     "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                     "frac": round(gbs / peaks["hbm_gbs"], 4), "ms": round(t * 1e3, 4),
-                    **({"note": "bitonic network, 66 compare-exchange stages per segment: ALU/shuffle bound; "
+                    **({"note": "bitonic network, 66 compare-exchange stages per segment, 2 segments per CTA at once: "
+                                "ALU/shuffle bound; "
                                 "frac is of the HBM peak, for context"} if name == "SORT" else
                        {"note": "reduce-then-scan: reads the input twice (12n bytes moved for 8n algorithmic)"})})
     del xs, ys

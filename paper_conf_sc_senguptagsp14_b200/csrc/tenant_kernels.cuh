@@ -632,16 +632,19 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
 // at index a with partner a ^ j keeps min(v, p) when it is the lower index of
 // an ascending block ((a & k) == 0) or the higher index of a descending one.
 constexpr int kSortSeg = 2048;
+constexpr int kSortPar = 2;                                       // segments sorted at once per CTA (ILP)
 __device__ __forceinline__ int sort_pad(int a) { return a + (a >> 5); }
 
 __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
                                  int S, uint8_t* stage) {
   static_assert(kSortSeg == 8 * kThreads, "8 keys per thread");
-  uint32_t* key = reinterpret_cast<uint32_t*>(stage);            // [2048 + 64] padded
+  constexpr int kPadSeg = kSortSeg + kSortSeg / 32;
+  uint32_t* key = reinterpret_cast<uint32_t*>(stage);            // [kSortPar][2048 + 64] padded
   const uint64_t nseg = n / kSortSeg;
   const int t = threadIdx.x;
   const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   auto load8 = [&](uint64_t seg, uint32_t* w) {
+    if (seg >= nseg) return;                                      // idle lane of the pair: garbage, never stored
     const uint32_t* src = x + seg * kSortSeg + 8 * t;
     if (vec) {
       const uint4 q0 = ld_stream(reinterpret_cast<const uint4*>(src));
@@ -653,13 +656,18 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
       for (int r = 0; r < 8; ++r) w[r] = src[r];
     }
   };
-  uint32_t nxt[8];
-  if ((uint64_t)rank < nseg) load8(rank, nxt);
-  for (uint64_t seg = rank; seg < nseg; seg += S) {
-    uint32_t v[8];
+  // segment pairs (rank + 2iS, rank + (2i+1)S)
+  uint32_t nxt[kSortPar][8];
 #pragma unroll
-    for (int r = 0; r < 8; ++r) v[r] = nxt[r];
-    if (seg + S < nseg) load8(seg + S, nxt);                       // next segment's loads fly during this sort
+  for (int h = 0; h < kSortPar; ++h) load8((uint64_t)rank + (uint64_t)h * S, nxt[h]);
+  for (uint64_t seg = rank; seg < nseg; seg += (uint64_t)kSortPar * S) {
+    uint32_t v[kSortPar][8];
+#pragma unroll
+    for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+      for (int r = 0; r < 8; ++r) v[h][r] = nxt[h][r];
+#pragma unroll
+    for (int h = 0; h < kSortPar; ++h) load8(seg + (uint64_t)(kSortPar + h) * S, nxt[h]);   // next pair in flight
 #pragma unroll
     for (int lk = 1; lk <= 11; ++lk) {
       const int k = 1 << lk;
@@ -668,41 +676,53 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
         const int j = 1 << lj;
         if (j >= 256) {                                              // across warps
 #pragma unroll
-          for (int r = 0; r < 8; ++r) key[sort_pad(8 * t + r)] = v[r];
+          for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+            for (int r = 0; r < 8; ++r) key[h * kPadSeg + sort_pad(8 * t + r)] = v[h][r];
           __syncthreads();
 #pragma unroll
-          for (int r = 0; r < 8; ++r) {
-            const int a = 8 * t + r;
-            const uint32_t p = key[sort_pad(a ^ j)];
-            v[r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[r], p) : max(v[r], p);
-          }
+          for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+              const int a = 8 * t + r;
+              const uint32_t p = key[h * kPadSeg + sort_pad(a ^ j)];
+              v[h][r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[h][r], p) : max(v[h][r], p);
+            }
           __syncthreads();
         } else if (j >= 8) {                                         // lanes t and t ^ (j / 8)
 #pragma unroll
-          for (int r = 0; r < 8; ++r) {
-            const int a = 8 * t + r;
-            const uint32_t p = __shfl_xor_sync(0xffffffffu, v[r], j >> 3);
-            v[r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[r], p) : max(v[r], p);
-          }
+          for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+              const int a = 8 * t + r;
+              const uint32_t p = __shfl_xor_sync(0xffffffffu, v[h][r], j >> 3);
+              v[h][r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[h][r], p) : max(v[h][r], p);
+            }
         } else {                                                     // registers r and r + j
 #pragma unroll
-          for (int r = 0; r < 8; ++r) {
-            if (r & j) continue;
-            const bool asc = ((8 * t + r) & k) == 0;
-            const uint32_t lo = v[r], hi = v[r + j];
-            v[r] = asc ? min(lo, hi) : max(lo, hi);
-            v[r + j] = asc ? max(lo, hi) : min(lo, hi);
-          }
+          for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+              if (r & j) continue;
+              const bool asc = ((8 * t + r) & k) == 0;
+              const uint32_t lo = v[h][r], hi = v[h][r + j];
+              v[h][r] = asc ? min(lo, hi) : max(lo, hi);
+              v[h][r + j] = asc ? max(lo, hi) : min(lo, hi);
+            }
         }
       }
     }
-    uint32_t* dst = y + seg * kSortSeg + 8 * t;
-    if (vec) {
-      reinterpret_cast<uint4*>(dst)[0] = make_uint4(v[0], v[1], v[2], v[3]);
-      reinterpret_cast<uint4*>(dst)[1] = make_uint4(v[4], v[5], v[6], v[7]);
-    } else {
 #pragma unroll
-      for (int r = 0; r < 8; ++r) dst[r] = v[r];
+    for (int h = 0; h < kSortPar; ++h) {
+      if (seg + (uint64_t)h * S >= nseg) continue;
+      uint32_t* dst = y + (seg + (uint64_t)h * S) * kSortSeg + 8 * t;
+      if (vec) {
+        reinterpret_cast<uint4*>(dst)[0] = make_uint4(v[h][0], v[h][1], v[h][2], v[h][3]);
+        reinterpret_cast<uint4*>(dst)[1] = make_uint4(v[h][4], v[h][5], v[h][6], v[h][7]);
+      } else {
+#pragma unroll
+        for (int r = 0; r < 8; ++r) dst[r] = v[h][r];
+      }
     }
   }
 }
