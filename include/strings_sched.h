@@ -29,6 +29,8 @@
  *   STRINGS_SM_COPY_MAX=b    largest op (bytes, all buffers) sent to those SMs
  *                            (default 1 MiB); host buffers must be mapped pinned
  *                            memory, 16-B aligned, sizes multiples of 16
+ *   STRINGS_SM_COPY_WHEN=always  send every eligible op there (default: only
+ *                            while that direction's copy engine has queued work)
  *   STRINGS_ITEM_VIA_COPY=1  also send KL work items of copy-engine jobs there
  *   STRINGS_COPY_STREAMS=physical  one H2D and one D2H stream per GPU instead of
  *                            per logical device

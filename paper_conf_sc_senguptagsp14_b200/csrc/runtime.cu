@@ -498,6 +498,12 @@ class Runtime : public strings::Hooks {
     return (uint64_t)((e ? atof(e) : 20.0) * 1e9);
   }();
   const uint64_t sm_copy_max = sm_copy_max_env();
+  // STRINGS_SM_COPY_WHEN=always: every eligible op on the copy partition; default
+  // "busy": only while that direction's copy engine has queued work
+  const bool sm_copy_always = [] {
+    const char* e = getenv("STRINGS_SM_COPY_WHEN");
+    return e && strcmp(e, "always") == 0;
+  }();
   // STRINGS_ITEM_VIA_COPY=1: the KL work item of a copy-engine job goes through the
   // copy partition too.  Off by default: C3 6% slower (the KL issue must wait for
   // the item behind the ring's 256 KiB copies), C1/C2/C4 within noise
@@ -937,7 +943,7 @@ class Runtime : public strings::Hooks {
         }
         jc->dev_out = reinterpret_cast<uint64_t>(base + off);
       }
-      if (sm_copy_eligible(jc->in, ph)) {
+      if (sm_copy_eligible(jc->in, ph, engine)) {
         // small inputs (+ the KL work item) as one zero-copy item on the copy partition
         CopyItem ci;
         memset(&ci, 0, sizeof ci);
@@ -987,7 +993,7 @@ class Runtime : public strings::Hooks {
                                        cudaMemcpyHostToDevice, ph->dbstream));
         }
       }
-    } else if (engine == strings::ENG_D2H && sm_copy_eligible(jc->out, ph)) {
+    } else if (engine == strings::ENG_D2H && sm_copy_eligible(jc->out, ph, engine)) {
       CopyItem ci;
       memset(&ci, 0, sizeof ci);
       ci.job = j.id;
@@ -1120,8 +1126,17 @@ class Runtime : public strings::Hooks {
   // An H2D/D2H op goes to the copy partition when it is small, every host buffer
   // is mapped pinned memory, every address and size is 16-B aligned, there is a
   // segment left for the KL work item, and the copy ring has room.
-  bool sm_copy_eligible(const std::vector<HostBuf>& bufs, const Phys* ph) const {
+  bool sm_copy_eligible(const std::vector<HostBuf>& bufs, const Phys* ph, int engine) const {
     if (!ph->copy_ctas || kl_mode != 0) return false;
+    if (!sm_copy_always) {
+      // only when that direction's copy engine has queued work: an idle engine starts
+      // a small copy sooner than the memop publish + item read of the SM path
+      // (4 KB job: 11.7 vs 16.6 us), the penalty is for queueing behind big copies
+      bool busy = false;
+      for (const auto& lg : logical)
+        if (lg.phys == ph && lg.ctr && (int32_t)(lg.issued[engine] - lg.ctr->done[engine]) > 0) busy = true;
+      if (!busy) return false;
+    }
     uint64_t total = 0;
     int nseg = 0;
     for (const auto& b : bufs) {

@@ -210,6 +210,7 @@ def test_small_copies_on_the_copy_partition(copy_ctas, monkeypatch):
     # 4 MiB copies stay on the copy engines.  Outputs exact either way, measured
     # invariants hold, and the stats say which path ran.
     monkeypatch.setenv("STRINGS_COPY_CTAS", copy_ctas)
+    monkeypatch.setenv("STRINGS_SM_COPY_WHEN", "always")
     wl = W.config_c1(reps=2)
     r = run_workload(wl, timing_mode=S.MEASURED)
     assert r.status == S.OK
@@ -222,10 +223,36 @@ def test_small_copies_on_the_copy_partition(copy_ctas, monkeypatch):
         assert r.stats.sm_copy_ops == 2 * n_gemm        # H2D and D2H of every GEMM job
 
 
+def test_small_copies_only_while_the_engine_is_busy():
+    # default policy: a small op goes to the copy partition only while its
+    # direction's copy engine has queued work (C1: GEMM copies among VSCALE's 4 MiB
+    # copies); an isolated small job uses the idle engine
+    wl = W.config_c1(reps=2)
+    r = run_workload(wl, timing_mode=S.MEASURED)
+    assert r.status == S.OK
+    check_outputs(wl, r)
+    n_gemm = sum(1 for j in wl.jobs if j.kclass == W.GEMM)
+    assert 0 <= r.stats.sm_copy_ops <= 2 * n_gemm
+    S.init(num_gpus=1, physical_gpus=1)
+    try:
+        t = S.register_tenant()
+        x = S.pinned_array((4096,), np.uint32)
+        y = S.pinned_array((4096,), np.uint32)
+        x[...] = np.arange(4096, dtype=np.uint32)
+        for _ in range(3):
+            S.submit(t, S.make_desc(S.XFER, n=4096, seed=1), [x], [y])
+            assert S.sync(t) == S.OK
+        assert np.array_equal(y, K.xfer(x, 1))
+        assert S.stats().sm_copy_ops == 0
+    finally:
+        S.shutdown()
+
+
 def test_small_copies_injected_parity_and_threshold(monkeypatch):
     # the physical copy path never changes decisions: INJECTED traces stay
     # byte-identical to the oracle with every op small enough for the partition
     monkeypatch.setenv("STRINGS_SM_COPY_MAX", str(64 << 20))
+    monkeypatch.setenv("STRINGS_SM_COPY_WHEN", "always")
     wl = W.config_c3(scale=4)
     r = run_workload(wl, timing_mode=S.INJECTED)
     assert r.status == S.OK
