@@ -257,7 +257,8 @@ constexpr uint32_t kSmemB = kTileN * kMaxK * 2;          // 128 KB
 // 128-B tail of mbarriers / TMEM slot sits after the larger of the two.
 constexpr uint32_t kSmemMain = (kStreamStages * kStreamChunk > kSmemA + kSmemB) ? kStreamStages * kStreamChunk
                                                                                  : kSmemA + kSmemB;
-constexpr uint32_t kSmemGemm = kSmemMain + 128;          // dynamic smem of the dispatcher / one-shot kernels
+constexpr uint32_t kSmemGemm = kSmemMain + 256;          // dynamic smem of the dispatcher / one-shot kernels
+                                                         // (tail: 128 B mbarriers / TMEM slot + 128 B scratch)
 static_assert(kSmemGemm + 2048 <= 227 * 1024, "dynamic + static smem must fit one CTA per SM");
 constexpr uint32_t kTmemCols = 256;                      // fp32 accumulator 128 x 256
 constexpr uint32_t kSlabA = 128 * 128;                   // 16 KB
@@ -345,6 +346,7 @@ struct GemmSmem {
   uint32_t* tmem_slot; // TMEM base written by tcgen05.alloc
   uint8_t* stage;      // streaming stages (aliases a/b: a CTA runs one item at a time)
   uint64_t* sbar;      // streaming stage mbarriers / GEMM fill mbarriers [4]
+  uint32_t* scratch;   // 32 words outside the stages (SCAN warp totals)
 };
 
 // Units u = tile * R + rep, tile = (mt, nt); this CTA takes the contiguous
@@ -520,9 +522,40 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
 // and the warp / CTA totals give its offset; chunks are whole tiles, so every
 // CTA's loads stay 16-B aligned when the buffers are.
 constexpr int kScanPT = 32;
+// One 32 KB chunk (8192 u32) scanned in place in shared memory: warp w owns
+// elements [1024w, 1024w + 1024) and walks them in 32 rounds of 32 consecutive
+// words (lane l reads word 32r + l: conflict-free), carrying its running sum;
+// the warps' offsets come from their chunk totals (phase A).  Returns the
+// chunk total; `carry` is the sum of everything before the chunk.
+__device__ __forceinline__ uint32_t scan_chunk_smem(uint32_t* c, uint32_t carry, uint32_t* wtot) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t* mine = c + warp * 1024;
+  uint32_t s = 0;
+#pragma unroll 8
+  for (int r = 0; r < 32; ++r) s += mine[r * 32 + lane];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) wtot[warp] = s;
+  __syncthreads();
+  uint32_t run = carry, total = 0;
+  for (int w = 0; w < 8; ++w) {
+    const uint32_t t = wtot[w];
+    if (w < warp) run += t;
+    total += t;
+  }
+#pragma unroll 4
+  for (int r = 0; r < 32; ++r) {
+    const uint32_t v = mine[r * 32 + lane];
+    const uint32_t incl = warp_incl_scan(v);
+    mine[r * 32 + lane] = run + incl;
+    run += __shfl_sync(0xffffffffu, incl, 31);
+  }
+  return total;
+}
+
 __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
-                                 int S, GroupSync* gs, uint8_t* stage) {
-  uint32_t* wsum = reinterpret_cast<uint32_t*>(stage);           // [8] warp totals + [1] broadcast
+                                 int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* wsum) {
+  // wsum: 16 words outside the stages ([8] warp totals + [8] broadcast / second buffer)
   constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;
   const uint64_t chunk = ((n + S - 1) / S + kTile - 1) / kTile * kTile;
   const uint64_t b0 = min(n, (uint64_t)rank * chunk), b1 = min(n, b0 + chunk);
@@ -568,7 +601,49 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
   __syncthreads();
   uint32_t carry = wsum[8];
   __syncthreads();
-  // 3. tiles; the next tile's 32 elements are loaded while this one is scanned
+  // 3a. whole 32 KB chunks through the TMA bulk pipeline (as stream_body), each
+  //     scanned in shared memory and bulk-stored back
+  static_assert(kStreamChunk == kTile * 4, "a scan tile is one pipeline chunk");
+  const uint64_t nch = vec ? (b1 - b0) / kTile : 0;
+  if (nch) {
+    const uint8_t* xb = reinterpret_cast<const uint8_t*>(x + b0);
+    uint8_t* yb = reinterpret_cast<uint8_t*>(y + b0);
+    if (threadIdx.x == 0) {
+      for (int q = 0; q < kStreamStages; ++q) mbar_init(&sbar[q], 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0)
+      for (int q = 0; q < kStreamLead && (uint64_t)q < nch; ++q) {
+        mbar_expect_tx(&sbar[q], kStreamChunk);
+        bulk_g2s(stage + q * kStreamChunk, xb + (uint64_t)q * kStreamChunk, kStreamChunk, &sbar[q]);
+      }
+    for (uint64_t i = 0; i < nch; ++i) {
+      const int q = (int)(i % kStreamStages);
+      const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
+      if (threadIdx.x == 0 && i + kStreamLead < nch) {
+        const int q2 = (int)((i + kStreamLead) % kStreamStages);
+        if (i + kStreamLead >= (uint64_t)kStreamStages)
+          asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStoreSlack) : "memory");
+        mbar_expect_tx(&sbar[q2], kStreamChunk);
+        bulk_g2s(stage + q2 * kStreamChunk, xb + (i + kStreamLead) * kStreamChunk, kStreamChunk, &sbar[q2]);
+      }
+      mbar_wait(&sbar[q], ph);
+      carry += scan_chunk_smem(reinterpret_cast<uint32_t*>(stage + q * kStreamChunk), carry,
+                               wsum + 8 * (int)(i & 1));       // alternate totals: no trailing barrier
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncthreads();
+      if (threadIdx.x == 0) bulk_s2g(yb + i * kStreamChunk, stage + q * kStreamChunk, kStreamChunk);
+    }
+    if (threadIdx.x == 0) {
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+    }
+    __syncthreads();
+  }
+  // 3b. the rest (unaligned buffers, the ragged last chunk): tiles in registers;
+  //     the next tile's 32 elements are loaded while this one is scanned
+  const uint64_t r0 = b0 + nch * kTile;
   auto load_tile = [&](uint64_t base, uint32_t* w) {
     const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
     if (vec && e0 + kScanPT <= b1) {
@@ -583,8 +658,8 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
     }
   };
   uint32_t nxt[kScanPT];
-  if (b0 < b1) load_tile(b0, nxt);
-  for (uint64_t base = b0; base < b1; base += kTile) {
+  if (r0 < b1) load_tile(r0, nxt);
+  for (uint64_t base = r0; base < b1; base += kTile) {
     const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
     const bool full = vec && e0 + kScanPT <= b1;
     uint32_t v[kScanPT];
@@ -739,7 +814,7 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
       break;
     case 4:
       scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
-                gs, sm.stage);
+                gs, sm.stage, sm.sbar, sm.scratch);
       break;
     case 5:
       sort_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
@@ -760,7 +835,8 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
   }
 }
 
-// smem: [A 64 KB][B 128 KB][tail 128 B: GEMM mbarrier @0, TMEM slot @8, <= 14 stream/fill mbarriers @16..]
+// smem: [A 64 KB][B 128 KB] (or the streaming stages if larger) [tail 256 B: GEMM mbarrier @0, TMEM slot @8,
+//        <= 14 stream/fill mbarriers @16.., scratch words @128]
 __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   GemmSmem s;
   s.a = base;
@@ -770,6 +846,7 @@ __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   s.tmem_slot = reinterpret_cast<uint32_t*>(tail + 8);
   s.stage = base;
   s.sbar = reinterpret_cast<uint64_t*>(tail + 16);
+  s.scratch = reinterpret_cast<uint32_t*>(tail + 128);
   return s;
 }
 
