@@ -4,7 +4,8 @@
         -o gpurun_out/prof python tools/kernel_probe.py
 
 Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2);
-`xfer_item`: XFER n=2^24 on 74 CTAs (x2), the C2 work item on one P=2 partition.
+`xfer_item`: XFER n=2^24 on 74 CTAs (x2), the C2 work item on one P=2 partition;
+`hist` (2^30 bytes), `scan`, `sort` (2^28 u32): the NEXT-2 bodies.
 The persistent dispatcher runs exactly these device bodies on its SM partitions.
 """
 import os
@@ -51,6 +52,23 @@ def main():
                             [c.data_ptr()], stream=st)
         torch.cuda.synchronize()
         assert torch.equal(c, a.float() @ b.float())
+    if "hist" in which:
+        nb = 1 << 30
+        xb = torch.randint(0, 256, (nb,), dtype=torch.uint8, device="cuda")
+        hb = torch.zeros(256, dtype=torch.int32, device="cuda")
+        for _ in range(2):
+            S.kernel_launch(0, S.make_desc(S.HIST, n=nb), [xb.data_ptr()], [hb.data_ptr()], stream=st)
+        torch.cuda.synchronize()
+        del xb, hb
+    for name, cls in (("scan", S.SCAN), ("sort", S.SORT)):
+        if name in which:
+            n28 = 1 << 28
+            xs = torch.randint(0, 1 << 20, (n28,), dtype=torch.int32, device="cuda")
+            ys = torch.empty_like(xs)
+            for _ in range(2):
+                S.kernel_launch(0, S.make_desc(cls, n=n28), [xs.data_ptr()], [ys.data_ptr()], stream=st)
+            torch.cuda.synchronize()
+            del xs, ys
     print("probe done")
 
 
