@@ -37,6 +37,8 @@
  *   STRINGS_COPY_THREADS=n   host threads of the pageable-buffer staging pool
  *   STRINGS_NT_COPY=0|1|2|3  staging copy loop: memcpy | SSE2 (default) | AVX2 |
  *                            AVX-512 non-temporal stores
+ *   STRINGS_KL_HELP=0        an idle KL slot does not lend its SMs to its sibling
+ *                            slot's VSCALE/XFER item (default: it does)
  *   STRINGS_SM_LIMIT=n       run the persistent kernel on n SMs (tests)
  *   STRINGS_POLL_MAX_NS=ns   idle-poll back-off cap of partition leaders (1024)
  *   STRINGS_STALL_DUMP_S=s   print in-flight ops to stderr if none completes

@@ -38,8 +38,14 @@ struct __align__(128) PartState {
   uint32_t seq;                       // claim number of the current item (ring entry)
   uint64_t t_start;
   uint64_t t_exec;
+  // Lending an idle KL partition to its sibling's streaming item (DispatchParams::help):
+  uint32_t lock;                      // 0 free, kLockOwn = running its own item, q+1 = lent to partition q
+  uint32_t total;                     // CTAs working on this partition's current item (own + lent)
+  uint64_t help;                      // (kHelpGen | owner << 16 | slot) << 32 when lent, published by the owner
   GroupSync sync;                     // barrier + partials for group-wide bodies (SCAN, HIST)
 };
+constexpr uint32_t kLockOwn = 0xFFFFFFFEu;
+constexpr uint32_t kHelpGen = 0x80000000u;     // generation slot word: this is a lent share of another item
 
 // The KL request queue lives in DEVICE memory: the host never makes the GPU
 // read host memory on the dispatch path (16 leaders polling host memory cut the
@@ -126,6 +132,7 @@ struct DispatchParams {
   uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
   uint32_t poll_max_ns;               // idle-poll back-off cap (STRINGS_POLL_MAX_NS)
   uint64_t fault_job;                 // fault injection (STRINGS_FAULT_JOB): trap on this job id
+  uint32_t help;                      // 1: an idle sibling KL partition joins VSCALE/XFER items
   // copy partition (partition index L*P, CTAs [part_start[L*P], part_start[L*P+1])) when copy_ctas > 0;
   // its claim counter is heads[L] and its PartState parts[L*P]
   int copy_ctas;

@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ KlItem s_item;
   __shared__ CopyItem s_citem;
-  __shared__ uint32_t s_gen, s_slot;
+  __shared__ uint32_t s_gen, s_slot, s_total, s_owner;
   GemmSmem sm = carve_smem(smem);
   if ((smem_u32(smem) & 1023u) != 0) __trap();   // SWIZZLE_128B tiles need a 1 KB-aligned base
   const int NK = p.L * p.P;                       // KL partitions; the copy partition (if any) is NK
@@ -82,6 +82,10 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   PartState* ps = p.parts + q;
   const KlItem* table = p.items + (size_t)(cpart ? 0 : ld) * p.M;
   const uint64_t* ring = cpart ? p.cring : p.ring + (size_t)ld * kRing;
+  // the sibling KL slot of the same logical device that may lend its CTAs (P >= 2)
+  const int sib = (!cpart && p.help && (q ^ 1) < NK && (q ^ 1) / p.P == ld) ? (q ^ 1) : -1;
+  PartState* sps = sib >= 0 ? p.parts + sib : nullptr;
+  const int S_sib = sib >= 0 ? p.part_start[sib + 1] - p.part_start[sib] : 0;
   const uint32_t tmem = cta_setup(sm);
   uint32_t mma_phase = 0;
   uint32_t seen = 0;
@@ -93,17 +97,38 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         uint32_t backoff = 32;
         uint64_t pub;
         for (;;) {
+          if (sib >= 0) {                         // lent to the sibling's item?
+            const uint64_t hw = ld_acquire_gpu_u64(&ps->help);
+            if (hw) {
+              pub = (hw & 0xFFFFFFFF00000000ull) | (seen + 1);
+              break;
+            }
+          }
           const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&p.heads[ld]);
           const uint64_t e = ld_acquire_gpu_u64(&ring[h % kRing]);
           if ((uint32_t)(e >> 32) == h + 1) {     // entry h published
+            if (sib >= 0 && atomicCAS(&ps->lock, 0u, kLockOwn) != 0u) continue;   // being lent: help first
             const uint64_t t_seen = globaltimer();
             if (atomicCAS(&p.heads[ld], h, h + 1) == h) {
               ps->ring_idx = h % kRing;
               ps->seq = h + 1;
               ps->t_start = t_seen;
+              uint32_t total = (uint32_t)S;
+              if (sib >= 0) {
+                // a streaming item borrows the sibling slot's CTAs if that slot is idle
+                const uint32_t slot = (uint32_t)e;
+                uint32_t kc;
+                asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(kc) : "l"(&table[slot].kclass) : "memory");
+                if ((kc == 0 || kc == 2) && atomicCAS(&sps->lock, 0u, (uint32_t)q + 1) == 0u) {
+                  total += (uint32_t)S_sib;
+                  st_release_gpu_u64(&sps->help, (uint64_t)(kHelpGen | ((uint32_t)q << 16) | slot) << 32);
+                }
+              }
+              ps->total = total;
               pub = ((uint64_t)(uint32_t)e << 32) | (seen + 1);
               break;
             }
+            if (sib >= 0) st_release_gpu(&ps->lock, 0u);
             continue;                             // the other KL slot took it
           }
           if (ld_acquire_gpu(p.stop)) {
@@ -121,7 +146,9 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         while ((uint32_t)(gw = ld_acquire_gpu_u64(&ps->gen)) == seen) __nanosleep(32);
       __syncwarp();                               // orders lane 0's acquire before the item loads
       gw = __shfl_sync(0xffffffffu, gw, 0);
-      const uint32_t g = (uint32_t)gw, slot = (uint32_t)(gw >> 32);
+      const uint32_t g = (uint32_t)gw, slot_word = (uint32_t)(gw >> 32);
+      const bool lent = !cpart && g != kStop && (slot_word & kHelpGen);
+      const uint32_t slot = lent ? (slot_word & 0xFFFFu) : slot_word;
       if (g != kStop && cpart) {
         // the 128-B copy item from the host-mapped table: one PCIe read by 8 lanes
         if (lane < sizeof(CopyItem) / 16)
@@ -138,19 +165,29 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
       if (lane == 0) {
         s_gen = g;
         s_slot = slot;
+        s_owner = lent ? ((slot_word >> 16) & 0x7FFFu) : (uint32_t)q;
+        // CTAs on this item: own partition + lent sibling (the owner wrote total before its gen)
+        s_total = (g == kStop || cpart) ? (uint32_t)S
+                  : lent ? (uint32_t)(p.part_start[((slot_word >> 16) & 0x7FFFu) + 1] -
+                                      p.part_start[(slot_word >> 16) & 0x7FFFu]) + (uint32_t)S
+                         : *reinterpret_cast<volatile uint32_t*>(&ps->total);
       }
     }
     __syncthreads();
     const uint32_t g = s_gen;
     if (g == kStop) break;
     seen = g;
-    if (rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
+    const bool lent = s_owner != (uint32_t)q;
+    PartState* ops = p.parts + s_owner;          // the partition whose item this is
+    const int total = (int)s_total;
+    if (!lent && rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
     if (cpart) {
       copy_body(s_citem, rank, S);
     } else {
       const KlItem it = s_item;
       if (it.job == p.fault_job) __trap();        // fault injection (tests the watchdog)
-      run_item(it, table + s_slot, true, rank, S, sm, tmem, mma_phase, &ps->sync);
+      // a lent CTA takes rank S_owner + rank among total (the owner's CTAs come first)
+      run_item(it, table + s_slot, true, lent ? total - S + rank : rank, total, sm, tmem, mma_phase, &ps->sync);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -160,21 +197,32 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         __threadfence_system();
       else
         __threadfence();
-      const uint32_t old = atomicAdd(&ps->done_cnt, 1u);
-      if (old == (uint32_t)S - 1) {
-        ps->done_cnt = 0;
-        KlDone* d = cpart ? &p.cdone[ps->ring_idx] : &p.done[ld * kRing + ps->ring_idx];
-        d->partition = (uint32_t)q;
-        d->t_start = ps->t_start;
-        d->t_exec = ps->t_exec;
+      const uint32_t old = atomicAdd(&ops->done_cnt, 1u);
+      if (old == (uint32_t)total - 1) {           // last CTA of the item (own or lent)
+        ops->done_cnt = 0;
+        KlDone* d = cpart ? &p.cdone[ops->ring_idx] : &p.done[ld * kRing + ops->ring_idx];
+        d->partition = s_owner;
+        d->t_start = ops->t_start;
+        d->t_exec = ops->t_exec;
         d->t_end = globaltimer();
         // Every CTA fenced its output writes at gpu scope before counting in, so the
         // outputs are in L2/HBM; the host reacts to this word only by issuing a D2H
         // DMA from device memory, so a gpu-scope fence + plain store is sufficient
         // (a sys-scope release costs ~3 us more per item, PCIe-fence round trip).
         __threadfence();
-        d->seq = ps->seq;
-        st_release_gpu(&ps->done_gen, seen);
+        d->seq = ops->seq;
+        const uint32_t og = (uint32_t)*reinterpret_cast<volatile uint64_t*>(&ops->gen);
+        if (sib >= 0 || lent) st_release_gpu(&ops->lock, 0u);   // the owner may claim / lend again
+        st_release_gpu(&ops->done_gen, og);
+      }
+      if (lent) {                                  // this partition's own bookkeeping for the lent share
+        const uint32_t o2 = atomicAdd(&ps->done_cnt, 1u);
+        if (o2 == (uint32_t)S - 1) {
+          ps->done_cnt = 0;
+          st_release_gpu_u64(&ps->help, 0ull);     // before done_gen: the leader must not help twice
+          st_release_gpu(&ps->lock, 0u);
+          st_release_gpu(&ps->done_gen, seen);
+        }
       }
     }
   }

@@ -793,6 +793,11 @@ class Runtime : public strings::Hooks {
         dp.poll_max_ns = pm ? (uint32_t)strtoul(pm, nullptr, 0) : 1024u;
         dp.stop = reinterpret_cast<const uint32_t*>(ph->doorbells);
         dp.copy_ctas = ph->copy_ctas;
+        {
+          // an idle KL slot lends its CTAs to its sibling's VSCALE/XFER item (STRINGS_KL_HELP=0: off)
+          const char* kh = getenv("STRINGS_KL_HELP");
+          dp.help = (kh && kh[0] == '0') ? 0u : 1u;
+        }
         dp.cring = reinterpret_cast<const uint64_t*>(ph->cring_dev);
         dp.citems = reinterpret_cast<const CopyItem*>(dbase + (reinterpret_cast<uint8_t*>(ph->citems) -
                                                                reinterpret_cast<uint8_t*>(ph->ctrl)));
