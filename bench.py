@@ -554,9 +554,10 @@ def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
            "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": _XFER_ITEM_NCU["dram_bytes"],
            "traffic_source": _XFER_ITEM_NCU["source"],
-           "bytes_per_launch": 8 * n, "note": "per work item on a half-GPU partition (72 of 148 SMs); the other "
-           "partition often runs an item concurrently and shares HBM; device time includes the partition "
-           "broadcast and completion publish (stand-alone full-GPU runs: kernel_rooflines)"}
+           "bytes_per_launch": 8 * n, "note": "per work item on its KL slot's 72 SMs plus the sibling slot's 72 "
+           "when that one is idle (lent CTAs, STRINGS_KL_HELP); otherwise the other slot runs its own item and "
+           "shares HBM; device time includes the claim, broadcast and completion publish (stand-alone full-GPU "
+           "runs: kernel_rooflines)"}
     if x.get("kl_body_us_p50"):
         # the body alone (leader's body start -> last CTA done): without the claim and
         # the partition broadcast, which are dispatch cost, not kernel work
