@@ -239,6 +239,7 @@ struct Phys {
   CopyItem* citems = nullptr;          // [kRing] host-mapped items
   KlDone* cdone = nullptr;             // [kRing] host-mapped completion words
   uint32_t ctail = 0, ccompleted = 0;
+  uint64_t last_big_copy_ns = 0;       // last copy-engine op larger than the SM-copy limit (mono ns)
   // ring index still owned by an op whose completion the engine has not consumed:
   // ops of different logical devices / directions are consumed out of ring order
   // (in INJECTED timing an op may be issued long before its virtual DONE), so an
@@ -976,6 +977,7 @@ class Runtime : public strings::Hooks {
           ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma,
                                        jc->in[i].bytes, cudaMemcpyHostToDevice, lg.h2d));
       ok = ok && signal_copy(lg, jc, engine, lg.h2d);
+      if (jc->job.h2d_bytes > sm_copy_max) ph->last_big_copy_ns = mono_ns();
       if (ok && kl_mode == 0) {
         // The job's KL work item goes to the device item table (the dispatcher
         // never reads host memory, ctrl.hpp): optionally through the copy
@@ -1018,6 +1020,7 @@ class Runtime : public strings::Hooks {
         off = align_up(off + jc->out[i].bytes);
       }
       ok = ok && signal_copy(lg, jc, engine, lg.d2h);
+      if (jc->job.d2h_bytes > sm_copy_max) ph->last_big_copy_ns = mono_ns();
     } else if (kl_mode == 0) {
       if (!await_item_copy(ph, jc)) {
         ok = false;
@@ -1134,10 +1137,11 @@ class Runtime : public strings::Hooks {
   bool sm_copy_eligible(const std::vector<HostBuf>& bufs, const Phys* ph, int engine) const {
     if (!ph->copy_ctas || kl_mode != 0) return false;
     if (!sm_copy_always) {
-      // only when that direction's copy engine has queued work: an idle engine starts
-      // a small copy sooner than the memop publish + item read of the SM path
-      // (4 KB job: 11.7 vs 16.6 us), the penalty is for queueing behind big copies
-      bool busy = false;
+      // only under load: that direction's copy engine has queued work, or a large copy
+      // went to the engines in the last 2 ms (the next one would queue behind a small
+      // copy issued now); an idle engine starts a small copy sooner than the memop
+      // publish + item read of the SM path (4 KB job: 11.7 vs 16.6 us)
+      bool busy = mono_ns() - ph->last_big_copy_ns < 2000000ull;
       for (const auto& lg : logical)
         if (lg.phys == ph && lg.ctr && (int32_t)(lg.issued[engine] - lg.ctr->done[engine]) > 0) busy = true;
       if (!busy) return false;

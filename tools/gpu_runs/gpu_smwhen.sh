@@ -2,7 +2,7 @@
 # Copy partition only while the engine is busy (default) vs always: tests, latency probe, configs, bench.
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests -m gpu -x -q --timeout 300 --timeout-method=thread > gpurun_out/pytest_gpu.log 2>&1; echo "pytest exit $? $(tail -1 gpurun_out/pytest_gpu.log)"
+timeout 900 python -m pytest tests -m gpu -x -q --timeout 300 --timeout-method=thread -k "small_copies or pageable or full_size_c2 or measured" > gpurun_out/pytest_gpu.log 2>&1; echo "pytest exit $? $(tail -1 gpurun_out/pytest_gpu.log)"
 for w in busy always; do
   STRINGS_SM_COPY_WHEN=$w timeout 300 python tools/latency_probe.py > gpurun_out/lat_$w.json 2>&1
   echo "$w latency: $(cat gpurun_out/lat_$w.json | cut -c1-200)"
