@@ -547,8 +547,8 @@ def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
     import strings_workload as W
     x = kl_lat.get("XFER")
     n = [j for j in wl.jobs if j.kclass == W.XFER][0].n
-    if not x:
-        return None
+    if not x or not x["kl_device_us_p50"]:
+        return None                                  # kl_mode 1: no dispatcher stamps
     gbs = 8 * n / (x["kl_device_us_p50"] * 1e3)
     out = {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline)", "bound": "hbm",
            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
