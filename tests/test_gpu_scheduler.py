@@ -392,3 +392,31 @@ def test_node_mode_on_several_physical_gpus(timing):
     assert invariants.check(r.trace, wl) == []
     check_outputs(wl, r)
     assert r.stats.physical_gpus == min(4, n)
+
+
+@pytest.mark.parametrize("help_on", ["1", "0"])
+def test_lent_kl_slot_streaming_items_exact(help_on, monkeypatch):
+    # one tenant, jobs one at a time: the sibling KL slot is always idle, so with
+    # lending on every VSCALE/XFER item runs on both halves (owner ranks first, lent
+    # ranks after); ragged sizes put the bulk pipeline and the LDG tail across
+    # the combined CTA set.  Outputs must be exact either way.
+    monkeypatch.setenv("STRINGS_KL_HELP", help_on)
+    S.init(num_gpus=1, physical_gpus=1)
+    try:
+        t = S.register_tenant()
+        rng = np.random.default_rng(11)
+        for n in (1, 4099, (1 << 20) + 37, (1 << 22) + 12345):
+            x = S.pinned_array((n,), np.uint32)
+            y = S.pinned_array((n,), np.uint32)
+            x[...] = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+            S.submit(t, S.make_desc(S.XFER, n=n, seed=n & 0xFFFF), [x], [y])
+            assert S.sync(t) == S.OK
+            assert np.array_equal(y, K.xfer(x, n & 0xFFFF)), n
+            xf = S.pinned_array((n,), np.float32)           # no NaN inputs (R-23)
+            xf[...] = rng.uniform(-1, 1, n).astype(np.float32)
+            yf = S.pinned_array((n,), np.float32)
+            S.submit(t, S.make_desc(S.VSCALE, n=n, alpha=1.0009765625), [xf], [yf])
+            assert S.sync(t) == S.OK
+            assert np.array_equal(yf.view(np.uint32), K.vscale(xf, 1.0009765625).view(np.uint32)), n
+    finally:
+        S.shutdown()
