@@ -3,13 +3,13 @@ INJECTED timing through the library (copy partition, busy policy, KL partitions)
 each checked against the oracle (INJECTED trace byte-identical, MEASURED
 invariants) and every output against the oracle's CPU kernels.
 
-    python tools/fuzz_gpu.py [first_seed] [count]
+    python tests/fuzz_gpu.py [first_seed] [count]   (test infrastructure: it runs the oracle)
 """
 import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 
 import strings_workload as W  # noqa: E402
 from oracle import invariants  # noqa: E402
