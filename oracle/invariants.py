@@ -8,7 +8,9 @@ Checks the invariants of SURVEY.md §8(c) on a canonical trace
   I2  LAS ordering: every LAS admission (when LAS admission is on and joint
       selection is off) places a job of minimal weighted key among the
       eligible ones; every LAS-policy wake takes a minimal-key candidate of its
-      device at that moment (reading R-7).
+      device at that moment (reading R-7); every PS wake takes a
+      minimal-key candidate among the device's candidates of the same phase
+      (reading R-11).
   I3  resource exclusivity: <= 1 op per copy engine, <= P KL ops per device,
       <= A woken-unfinished ops, <= M resident jobs, <= c_t in-flight per tenant.
   I4  per-tenant order: a tenant's jobs are admitted in
@@ -191,6 +193,13 @@ def check(lines: List[str], wl: W.Workload) -> List[str]:
                 for u in candidates(g):
                     if u != j and las_cmp(u, j) < 0:
                         errs.append(f"I2 t={r.t} gid={g} LAS woke job {j} before lower-key job {u}")
+            if cfg.device_policy == W.PS:
+                # PS (R-11) chooses *which phases* to wake, but
+                # within a phase it always takes the minimal-key candidate
+                # (diversity step and fill step alike)
+                for u in candidates(g):
+                    if u != j and phase[u] == x and las_cmp(u, j) < 0:
+                        errs.append(f"I2 t={r.t} gid={g} PS woke job {j} before lower-key job {u} of its phase")
             if cfg.device_policy == W.TFS:
                 others = {ten_of[i] for i in resident[g] if woken[i]} - {ten_of[j]}
                 if others:

@@ -244,18 +244,20 @@ def test_eq1_constant_service_converges_geometrically():
     g = 1000
     cfg = W.SystemConfig(num_gpus=1, device_policy=W.FIFO, quantum_ns=g)
     o = run_oracle(W.Workload("c", cfg, [W.TenantSpec()], [kl_only_job(0, 12 * g)]))
-    cg = [int(f[9]) for f in (ln.split() for ln in o.trace) if f[1] == "EPOCH"][:12]
+    cg = [int(f[9]) for f in (ln.split() for ln in o.trace) if f[1] == "EPOCH"]
+    assert len(cg) == 12                     # one per epoch the 12g op spans (in-progress service)
     for n, c in enumerate(cg, start=1):
         exact = g * (1 - 0.2 ** n) * 65536
         assert exact - n <= c <= exact + 1e-6
 
 
 # ------------------------------------------------------------------- M/M/1
+@pytest.mark.slow
 @pytest.mark.parametrize("policy", [W.FIFO, W.LAS, W.PS])
 def test_mm1_mean_response_time(policy):
     # G=P=A=1, zero-byte copies, Poisson arrivals (Eq. 4), exponential KL
     # sizes, size-blind work-conserving order => E[T] = 1/(mu - lambda).
-    mean_s, rho, T, per = 10_000.0, 0.5, 8, 5000
+    mean_s, rho, T, per = 10_000.0, 0.5, 8, 25_000          # 2*10^5 jobs
     rng = W.SplitMix64(2024 + policy)
     jobs = []
     for t in range(T):
@@ -272,7 +274,7 @@ def test_mm1_mean_response_time(policy):
     mu = 1.0 / svc.mean()
     lam = len(jobs) / max(j.arrival for j in o.jobs)
     want = 1.0 / (mu - lam)
-    assert abs(resp.mean() / want - 1.0) < 0.08
+    assert abs(resp.mean() / want - 1.0) < 0.03
 
 
 # ---------------------------------------------------------- roofline (I6)
@@ -411,6 +413,21 @@ def test_gwtmin_places_in_proportion_to_device_weights(weights, jobs):
     cfg.balancer = W.GMIN
     pl = placements(run_oracle(wl))
     assert max(pl.count(g) for g in range(len(weights))) - min(pl.count(g) for g in range(len(weights))) <= 1
+
+
+def test_invariant_checker_catches_ps_within_phase_wake_order():
+    # two same-phase WAKEs of one PS pass swapped must be flagged (I2, R-11)
+    wl = W.config_c3()
+    tr = run_oracle(wl).trace
+    assert invariants.check(tr, wl) == []
+    for i in range(len(tr) - 1):
+        a, b = tr[i].split(), tr[i + 1].split()
+        if (a[1] == b[1] == "WAKE" and a[0] == b[0] and a[2] == b[2] and a[3] == b[3]
+                and a[5] != b[5]):
+            m = tr[:i] + [tr[i + 1], tr[i]] + tr[i + 2:]
+            if any(e.startswith("I2") for e in invariants.check(m, wl)):
+                return
+    pytest.fail("no PS wake-order mutation detected")
 
 
 def test_invariant_checker_catches_las_wake_order():

@@ -1,0 +1,129 @@
+"""Mutation check of the oracle's pins -- no GPU.
+
+Each entry below is a plausible slip in ``oracle/`` (a sum where the paper's
+rule needs a max, a dropped term, a wrong EWMA weight, a tie broken the wrong
+way, ...).  The test copies the oracle, the input generator and the oracle's
+pin tests into a scratch directory, applies ONE slip, and runs the pins there:
+at least one pin must fail.  A slip that survives means the oracle's arithmetic
+at that spot is checked only against itself -- exactly what the pins exist to
+prevent (the GPU path is compared with the oracle, so a misreading shared by
+both would otherwise go unseen).
+
+The snippets are matched literally and must occur exactly once, so a refactor
+of the oracle breaks this test loudly instead of silently skipping a mutation.
+"""
+import os
+import shutil
+import subprocess
+import sys
+from concurrent.futures import ThreadPoolExecutor
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+# (name, file, original snippet, mutated snippet)
+MUTATIONS = [
+    ("guf_sum_to_max", "oracle/des.py",
+     "return sum(self.pred(i)[3] for i in res) + self.pred(j)[3]",
+     "return max([self.pred(i)[3] for i in res] + [self.pred(j)[3]])"),
+    ("guf_drops_new_job", "oracle/des.py",
+     "return sum(self.pred(i)[3] for i in res) + self.pred(j)[3]",
+     "return sum(self.pred(i)[3] for i in res)"),
+    ("prior_flop_rate", "oracle/des.py",
+     "PRIOR_KL_FLOP_PER_NS = 700_000", "PRIOR_KL_FLOP_PER_NS = 70_000"),
+    ("prior_util_copy_share", "oracle/des.py",
+     "return h, k, d, (k * 65536 // tot) if tot else 0",
+     "return h, k, d, ((h + d) * 65536 // tot) if tot else 0"),
+    ("sft_ewma_weight", "oracle/des.py",
+     "e.kl = (4 * smp[1] + e.kl) // 5", "e.kl = (smp[1] + 4 * e.kl) // 5"),
+    ("ps_fill_not_merged", "oracle/des.py",
+     "for j in self.las_sorted(by[H2D] + by[D2H]):", "for j in by[H2D] + by[D2H]:"),
+    ("ps_diversity_tie_to_d2h", "oracle/des.py",
+     "if len(copies) == 2 and self.las_key_less(by[D2H][0], by[H2D][0]):",
+     "if len(copies) == 2 and not self.las_key_less(by[H2D][0], by[D2H][0]):"),
+    ("dtf_max_to_sum", "oracle/des.py",
+     "return max(copy + h + dd, kern + k)", "return copy + h + dd + kern + k"),
+    ("rtf_total_not_remaining", "oracle/des.py",
+     "s += (h if i.phase <= H2D else 0) + (k if i.phase <= KL else 0) + (dd if i.phase <= D2H else 0)",
+     "s += h + k + dd"),
+    ("mbf_total_not_remaining", "oracle/des.py",
+     "if fresh or i.phase <= H2D:", "if True:"),
+    ("epoch_drops_in_progress", "oracle/des.py",
+     "inprog[j.tenant] += t - max(j.start[x], self.epoch_start)", "inprog[j.tenant] += 0"),
+    ("eq1_k_0_6", "oracle/des.py",
+     "tn.cgs = (4 * (gs << 16) + old) // 5", "tn.cgs = (3 * (gs << 16) + 2 * old) // 5"),
+    ("joint_tie_last", "oracle/des.py",
+     "if best is None or s_ < best[0]:", "if best is None or s_ <= best[0]:"),
+    ("score_tie_highest_gid", "oracle/des.py",
+     "if bs is None or s < bs:", "if bs is None or s <= bs:"),
+    ("util_span_from_arrival", "oracle/des.py",
+     "span = t - j.t_place", "span = t - j.arrival"),
+    ("tfs_no_service_history", "oracle/des.py",
+     "d.svc[j.tenant] = d.svc.get(j.tenant, 0) + (t - j.start[x])", "d.svc[j.tenant] = 0"),
+    ("las_admission_to_arrival", "oracle/des.py",
+     "if self.cfg.las_admission:", "if False:"),
+    ("las_weight_ignored", "oracle/des.py",
+     "lhs, rhs = ca * b.prio, cb * a.prio", "lhs, rhs = ca, cb"),
+    ("gwtmin_ignores_weight", "oracle/des.py",
+     "if best is None or len(d.resident) * best.weight < len(best.resident) * d.weight:",
+     "if best is None or len(d.resident) < len(best.resident):"),
+    ("fmix32_shift", "oracle/kernels.py",
+     "h ^= h >> np.uint32(13)", "h ^= h >> np.uint32(15)"),
+    ("gemm_rounds_operands_to_f32", "oracle/kernels.py",
+     "return (a @ b).astype(np.float32)",
+     "return (a.astype(np.float32) @ b.astype(np.float32)).astype(np.float32)"),
+    ("jain_unsquared_sum", "oracle/metrics.py",
+     "return sum(xs) ** 2 / (n * s2)", "return sum(xs) / (n * s2)"),
+]
+
+PIN_FILES = ["test_oracle_pins.py", "test_oracle_des.py", "test_golden.py",
+             "test_oracle_metrics.py", "test_oracle_kernels.py"]
+
+
+def _stage(dst):
+    for d in ("oracle", "strings_workload"):
+        shutil.copytree(os.path.join(ROOT, d), os.path.join(dst, d),
+                        ignore=shutil.ignore_patterns("__pycache__"))
+    os.makedirs(os.path.join(dst, "tests"))
+    for f in ["conftest.py"] + PIN_FILES:
+        shutil.copy(os.path.join(ROOT, "tests", f), os.path.join(dst, "tests", f))
+    shutil.copytree(os.path.join(ROOT, "tests", "golden"), os.path.join(dst, "tests", "golden"))
+    shutil.copy(os.path.join(ROOT, "pytest.ini"), os.path.join(dst, "pytest.ini"))
+
+
+def _run_pins(dst):
+    env = dict(os.environ, PYTHONPATH=dst, PYTHONDONTWRITEBYTECODE="1")
+    cmd = [sys.executable, "-m", "pytest", "-x", "-q", "-m", "not slow and not gpu",
+           "-p", "no:cacheprovider"] + [os.path.join("tests", f) for f in PIN_FILES]
+    return subprocess.run(cmd, cwd=dst, env=env, capture_output=True, text=True, timeout=900)
+
+
+def test_every_mutation_is_caught_by_a_pin(tmp_path):
+    base = tmp_path / "base"
+    _stage(str(base))
+    # the unmutated copy must pass its pins (so a failure below is the mutation's)
+    r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
+                        os.path.join("tests", "test_oracle_pins.py")],
+                       cwd=str(base), env=dict(os.environ, PYTHONPATH=str(base)),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:]
+
+    def one(m):
+        name, path, old, new = m
+        dst = tmp_path / name
+        _stage(str(dst))
+        fp = dst / path
+        src = fp.read_text()
+        assert src.count(old) == 1, f"{name}: snippet not found exactly once in {path}"
+        fp.write_text(src.replace(old, new))
+        r = _run_pins(str(dst))
+        return name, r.returncode, r.stdout[-1500:]
+
+    muts = MUTATIONS
+    assert len(muts) >= 20
+    with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:
+        results = list(ex.map(one, muts))
+    survivors = [(n, rc, out) for n, rc, out in results if rc != 1]
+    # rc 1 = some test failed; 0 = the mutation survived; anything else = harness error
+    assert not survivors, "\n".join(f"{n}: rc={rc}\n{out}" for n, rc, out in survivors)
