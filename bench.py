@@ -59,13 +59,16 @@ def parse_args():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--kl-mode", type=int, default=0, help="0 persistent dispatcher, 1 per-job launches (ncu)")
     p.add_argument("--trace-out", default=None)
-    p.add_argument("--static-repeats", type=int, default=3)
+    p.add_argument("--static-repeats", type=int, default=5)
     p.add_argument("--awake-budget", type=int, default=0, help="A (0 = config default)")
     p.add_argument("--admit-cap", type=int, default=0, help="M (0 = config default)")
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
     p.add_argument("--config-repeats", type=int, default=3, help="timed runs per config in --configs")
+    p.add_argument("--config-static", action="store_true", help="--configs: add static baselines")
+    p.add_argument("--no-baseline-config", action="store_true",
+                   help="N > 1: skip the BASELINE config whose G equals N (C1/C3/C5)")
     p.add_argument("--configs", action="store_true",
                    help="run BASELINE configs C1-C5 at full size (node mode, logical devices if G > GPUs)")
     p.add_argument("--fig2", action="store_true",
@@ -89,7 +92,8 @@ class ClockSampler:
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
     def __init__(self, index):
-        self.index = index                 # nvidia-smi --id (index, bus id or UUID)
+        # nvidia-smi --id: an index, bus id or UUID, or a list of them (node mode: every GPU used)
+        self.index = ",".join(str(i) for i in index) if isinstance(index, (list, tuple)) else index
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         self.p = None
 
@@ -170,6 +174,38 @@ def host_link_peaks(torch, nbytes=256 << 20, iters=5) -> dict:
     r["bidir_gbs"] = 2 * nbytes / timed(both) / 1e9
     del h_in, h_out, d_a, d_b
     return r
+
+
+def host_link_concurrent(torch, ngpu: int, nbytes=256 << 20, iters=3) -> dict:
+    """H2D + D2H copies on every one of `ngpu` GPUs at once (the
+    host's DRAM and PCIe root complexes are shared): aggregate GB/s and the
+    per-GPU share, the link peak each device's T*_d uses in node mode."""
+    res = []
+    for g in range(ngpu):
+        with torch.cuda.device(g):
+            res.append((torch.empty(nbytes, dtype=torch.uint8).pin_memory(),
+                        torch.empty(nbytes, dtype=torch.uint8).pin_memory(),
+                        torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{g}"),
+                        torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{g}"),
+                        torch.cuda.Stream(device=g), torch.cuda.Stream(device=g)))
+    best = None
+    for _ in range(iters + 1):
+        for g in range(ngpu):
+            torch.cuda.synchronize(g)
+        t = time.perf_counter()
+        for g, (hi, ho, da, db, s1, s2) in enumerate(res):
+            with torch.cuda.device(g):
+                with torch.cuda.stream(s1):
+                    da.copy_(hi, non_blocking=True)
+                with torch.cuda.stream(s2):
+                    ho.copy_(db, non_blocking=True)
+        for g in range(ngpu):
+            torch.cuda.synchronize(g)
+        dt = time.perf_counter() - t
+        best = dt if best is None else min(best, dt)
+    agg = 2 * nbytes * ngpu / best / 1e9
+    del res
+    return {"gpus": ngpu, "aggregate_bidir_gbs": agg, "per_gpu_bidir_gbs": agg / ngpu}
 
 
 def kernel_rooflines(torch, S, peaks) -> list:
@@ -427,9 +463,9 @@ def run_strings(args, rank, world, torch, gloo):
     tstar, terms = tstar_device(wl, link, peaks["hbm_gbs"], peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"])
     moved = sum(sum(j.h2d_sizes()) + sum(j.d2h_sizes()) for j in wl.jobs)
     link_gbs = moved / span_step / 1e9
-    # Jain fairness (Eq. 3, reading R-2) over tenants of the last timed step:
-    # x_i = (service tenant i received = its busy time on the engines) /
-    #       (its elapsed time first arrival -> last completion) / w_i
+    # Jain fairness (Eq. 3, reading R-2) over tenants of the last timed step,
+    # secondary form: x_i = (service tenant i received = its busy time on the
+    # engines) / (its elapsed time first arrival -> last completion) / w_i
     last = infos[-jobs_step:]
     busy, first, lastd = {}, {}, {}
     for inf in last:
@@ -447,6 +483,10 @@ def run_strings(args, rank, world, torch, gloo):
     for inf in last:
         mlat.setdefault(inf.tenant, []).append((inf.t_done[2] - step_t0) / 1e9)
     mlat = {t: sum(v) / len(v) for t, v in mlat.items()}
+    # the primary form of R-2: x_i = (T_alone_i / T_shared_i) / w_i, T_alone from
+    # each tenant's jobs run alone through the library on this GPU
+    alone = alone_mean_latency(S, wl, lambda sp: per_tenant[sp.tenant][0], lambda sp: per_tenant[sp.tenant][1])
+    jain_primary, _ = jain_r2(wl, mlat, alone)
     # KL phase: device execution (%globaltimer claim -> last CTA done) vs the
     # host-observed START -> DONE (adds ring pickup + completion notification)
     timed = infos[-jobs_step * args.steps:]
@@ -493,9 +533,14 @@ def run_strings(args, rank, world, torch, gloo):
         "host_link": {k: round(v, 2) for k, v in link.items()},
         "kernel_rooflines": krl,
         "_mean_latency_s_by_tenant": mlat,
-        "jain": round(jain, 4),
-        "jain_definition": "Jain over x_i = engine-busy service of tenant i / its elapsed time (last timed step), "
-                           "all tenants of all ranks",
+        "jain": round(jain_primary, 4),
+        "jain_definition": "Eq. (3) over x_i = (T_alone_i / T_shared_i) / w_i (reading R-2): mean completion "
+                           "latency of tenant i's jobs in the last timed step vs the same jobs run alone through "
+                           "the library on this GPU",
+        "jain_service": round(jain, 4),
+        "jain_service_definition": "secondary (R-2): x_i = engine-busy service of tenant i / its elapsed time",
+        "alone_mean_latency_ms": {W.CLASS_NAMES[k]: round(alone[t] * 1e3, 3) for k, t in
+                                  {sp.kclass: sp.tenant for sp in wl.jobs}.items()},
         "phase_latency": kl_lat,
         "gpu_launches": kl_items,
         "gpu_launches_note": "work items executed by the persistent dispatcher kernel (launched once at init): "
@@ -519,6 +564,263 @@ def run_strings(args, rank, world, torch, gloo):
     if args.trace_out and rank == 0:
         with open(args.trace_out, "w") as f:
             f.write("\n".join(trace) + "\n")
+    return res, wl
+
+
+
+# ------------------------------------------------ shared measurement helpers
+def tenant_buffers(torch, wl):
+    """Pinned host buffers, one input and one output set per (tenant, job shape):
+    c_t = 1, so a tenant's jobs never overlap, and every job still moves its own
+    bytes each way.  Returns (ins_of(spec), outs_of(spec))."""
+    import numpy as np
+
+    import strings_workload as W
+    bufs = {}
+    for spec in wl.jobs:
+        key = (spec.tenant, spec.kclass, spec.n, spec.m, spec.k)
+        if key not in bufs:
+            bufs[key] = ([torch.from_numpy(a.view(np.uint8).reshape(-1)).pin_memory() for a in W.job_inputs(spec)],
+                         [torch.empty(sz, dtype=torch.uint8).pin_memory() for sz in spec.d2h_sizes()])
+    key = lambda s: (s.tenant, s.kclass, s.n, s.m, s.k)  # noqa: E731
+    return (lambda s: bufs[key(s)][0]), (lambda s: bufs[key(s)][1]), bufs
+
+
+def mean_latency_by_tenant(infos) -> dict:
+    """Mean completion latency (s) per tenant of one batch whose jobs were all
+    submitted together: JOB_DONE - the batch's first arrival (reading R-1)."""
+    t0 = min(i.t_arrival for i in infos)
+    lat = {}
+    for i in infos:
+        lat.setdefault(i.tenant, []).append((i.t_done[2] - t0) / 1e9)
+    return {t: sum(v) / len(v) for t, v in lat.items()}
+
+
+def job_signature(sp) -> tuple:
+    return (sp.kclass, sp.n, sp.m, sp.k, sp.reps)
+
+
+def alone_mean_latency(S, wl, ins_of, outs_of) -> dict:
+    """T-bar_alone of reading R-2: each tenant's job sequence run
+    ALONE on one GPU through the library (same config, G = 1), its jobs
+    submitted together as in the shared run.  Tenants whose job sequences have
+    the same shapes (class and sizes, job by job) share one alone run: their
+    data differs, which changes no phase's time.  Returns {tenant: mean s}."""
+    cfg = dataclasses.replace(wl.config, num_gpus=1, device_weights=None).resolved()
+    seqs = {}
+    for sp in wl.jobs:
+        seqs.setdefault(sp.tenant, []).append(sp)
+    groups = {}
+    for t, specs in seqs.items():
+        groups.setdefault((wl.tenants[t].max_inflight, tuple(job_signature(s) for s in specs)), []).append(t)
+    S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=1, trace_in_memory=False)
+    out = {}
+    try:
+        for members in groups.values():
+            t = members[0]
+            tid = S.register_tenant(wl.tenants[t].weight, wl.tenants[t].max_inflight)
+            for _warm in (True, False):
+                ids = [S.submit_spec(tid, sp, ins_of(sp), outs_of(sp)) for sp in seqs[t]]
+                assert S.drain() == S.OK
+            lat = sum(mean_latency_by_tenant([S.job_info(i) for i in ids]).values())
+            for m in members:
+                out[m] = lat
+    finally:
+        S.shutdown()
+    return out
+
+
+def jain_r2(wl, shared_lat: dict, alone: dict):
+    """Jain's index (Eq. 3) over x_i = (T-bar_alone_i / T-bar_shared_i) / w_i
+    (reading R-2, the primary definition: weighted normalised progress)."""
+    xs = [alone[t] / shared_lat[t] / wl.tenants[t].weight for t in sorted(shared_lat)]
+    return sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs)), xs
+
+
+def per_gpu_roofline(wl, infos, phys: int, link, peaks, partitions: int, lpg: int) -> list:
+    """Overlapped roofline T*_d / span for every physical GPU,
+    over the jobs the balancer placed there (logical g -> physical g mod phys)."""
+    import strings_workload as W
+    by = {}
+    for sp, inf in zip(wl.jobs, infos):
+        by.setdefault(inf.gid % phys, []).append((sp, inf))
+    out = []
+    for g in sorted(by):
+        rows = by[g]
+        sub = W.Workload(f"gpu{g}", wl.config, wl.tenants, [dataclasses.replace(sp, arrival_ns=0) for sp, _ in rows])
+        tstar, terms = tstar_device(sub, link, peaks["hbm_gbs"], peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"],
+                                    kl_slots=lpg * partitions)
+        span = (max(i.t_done[2] for _, i in rows) - min(i.t_start[0] for _, i in rows)) / 1e9
+        out.append({"gpu": g, "jobs": len(rows), "tstar_ms": round(tstar * 1e3, 3), "span_ms": round(span * 1e3, 3),
+                    "frac": round(tstar / span, 4) if span > 0 else None,
+                    "bound_by": max(terms, key=terms.get)})
+    return out
+
+
+def scaled_link(link1: dict, conc: dict) -> dict:
+    """Per-GPU link peaks while every GPU copies at once: the alone peaks scaled
+    by the concurrent per-GPU bidirectional share (never above the alone peak)."""
+    f = min(1.0, conc["per_gpu_bidir_gbs"] / link1["bidir_gbs"])
+    return {k: v * f for k, v in link1.items()}
+
+
+def run_node(args, torch, gloo, world):
+    """N > 1 GPUs in NODE MODE: one process owns all N GPUs and the
+    library's level-1 balancer places every job on one of them (the
+    runtime overrides the application's GPU choice).  Workload: C2 weak-scaled,
+    16 tenants per GPU (16N tenants, 128N jobs per step), DTF joint placement,
+    PS dispatch, MEASURED timing.  Beside it, at the same N: static provisioning
+    both ways (tenant mod N, and every tenant on device 0), Jain per R-2 from
+    alone runs, the overlapped roofline per GPU, and the BASELINE config whose
+    G equals N (C1 at 2, C3 at 4, C5 at 8)."""
+    import strings_workload as W
+    from paper_conf_sc_senguptagsp14_b200 import strings as S
+
+    N = args.gpus
+    ngpu = torch.cuda.device_count()
+    phys = min(N, ngpu)
+    lpg = -(-N // phys)
+    peaks = measured_peaks()
+    link1 = host_link_peaks(torch)
+    conc = host_link_concurrent(torch, phys)
+    link = scaled_link(link1, conc)
+    wl = W.config_c2(jobs_per_tenant=args.jobs_per_tenant, num_gpus=N)
+    for name in ("awake_budget", "admit_cap", "partitions"):
+        if getattr(args, name) > 0:
+            setattr(wl.config, name, getattr(args, name))
+    if args.device_policy >= 0:
+        wl.config.device_policy = args.device_policy
+    if args.balancer >= 0:
+        wl.config.balancer = args.balancer
+    cfg = wl.config.resolved()
+    ins_of, outs_of, bufs = tenant_buffers(torch, wl)
+    arenas = S.torch_arenas(N, phys, cfg.admit_cap)
+    torch.cuda.synchronize()
+    S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=phys, kl_mode=args.kl_mode,
+                       trace_in_memory=False, arenas=arenas)
+    tenants = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+    stream = torch.cuda.Stream(device=0)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ids = []
+
+    def one_step():
+        ids.clear()
+        for spec in wl.jobs:
+            ids.append(S.submit_spec(tenants[spec.tenant], spec, ins_of(spec), outs_of(spec)))
+        st = S.drain()
+        assert st == S.OK, S.strerror(st)
+
+    for _ in range(args.warmup):
+        one_step()
+    stream.synchronize()
+    with ClockSampler(list(range(phys))) as clk:
+        ev0.record(stream)
+        t_wall = time.perf_counter()
+        for _ in range(args.steps):
+            one_step()
+        ev1.record(stream)
+        ev1.synchronize()
+        t_wall = time.perf_counter() - t_wall
+    dt = max_over(gloo, ev0.elapsed_time(ev1) / 1e3)
+    infos = [S.job_info(i) for i in ids]            # the last timed step
+    stats = S.stats()
+    jobs_step = len(wl.jobs)
+    e2e = None
+    if not args.no_e2e:
+        import numpy as np
+        np_bufs = {k: ([a.numpy().copy() for a in i], [np.empty(o.numel(), dtype=np.uint8) for o in o_])
+                   for k, (i, o_) in bufs.items()}
+        key = lambda s: (s.tenant, s.kclass, s.n, s.m, s.k)  # noqa: E731
+        for spec in wl.jobs:                         # warm the staging pool once
+            S.submit_spec(tenants[spec.tenant], spec, np_bufs[key(spec)][0], np_bufs[key(spec)][1])
+        assert S.drain() == S.OK
+        e2e_steps = max(1, min(args.steps, 5))
+        t = time.perf_counter()
+        for _ in range(e2e_steps):
+            for spec in wl.jobs:
+                S.submit_spec(tenants[spec.tenant], spec, np_bufs[key(spec)][0], np_bufs[key(spec)][1])
+            assert S.drain() == S.OK
+        e2e_dt = time.perf_counter() - t
+        e2e = {"value": round(jobs_step * e2e_steps / e2e_dt, 3), "unit": "jobs/s", "steps": e2e_steps,
+               "h2d_bytes_per_step": int(sum(sum(j.h2d_sizes()) for j in wl.jobs)),
+               "d2h_bytes_per_step": int(sum(sum(j.d2h_sizes()) for j in wl.jobs)),
+               "host_buffers": "the caller's own (pageable) numpy arrays, staged by the library (PMT/MOT, "
+                               "P:L327-329) inside the timed region",
+               "timer": "wall clock, first strings_submit to strings_drain() return"}
+        del np_bufs
+    S.shutdown()
+    del arenas
+    torch.cuda.synchronize()
+    value = jobs_step * args.steps / dt
+    moved = sum(sum(j.h2d_sizes()) + sum(j.d2h_sizes()) for j in wl.jobs)
+    span_step = dt / args.steps
+    link_gbs = moved / span_step / 1e9
+    agg_peak = link["bidir_gbs"] * phys
+    shared = mean_latency_by_tenant(infos)
+    alone = alone_mean_latency(S, wl, ins_of, outs_of)
+    jain, xs = jain_r2(wl, shared, alone)
+    per_gpu = per_gpu_roofline(wl, infos, phys, link, peaks, cfg.partitions, lpg)
+    placed = {}
+    for inf in infos:
+        placed[inf.gid] = placed.get(inf.gid, 0) + 1
+    res = {
+        "metric": METRIC, "value": round(value, 3), "unit": "jobs/s", "n_gpus": N,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16/f32/u32",
+        "data": "synthetic (seeded; strings_workload)",
+        "config": {"workload": f"C2 weak-scaled to {N} GPUs: {len(wl.tenants)} tenants (GEMM 256^3 R=64 / XFER "
+                               f"2^24 u32 alternating) x {args.jobs_per_tenant} jobs, DTF joint placement over "
+                               f"{N} devices, PS dispatch, measured timing",
+                   "jobs_per_step": jobs_step, "partitions": cfg.partitions, "awake_budget": cfg.awake_budget,
+                   "admit_cap": cfg.admit_cap, "l2": "inputs larger than L2 (4 GiB each way per GPU per step)",
+                   "parallelism": f"node mode, {W.BALANCER_NAMES[cfg.balancer]} balancer: one process places "
+                                  f"every job on one of {N} devices ({phys} physical GPU(s))"
+                                  + ("" if phys == N else "; LOGICAL devices share GPUs: not an N-GPU number"),
+                   "ranks": f"{world} (rank 0 drives the node; other ranks idle: no data-path collective)",
+                   "kl_mode": "persistent dispatcher" if stats.kl_mode == 0 else "per-op launches"},
+        "placement": {str(g): placed.get(g, 0) for g in range(N)},
+        "roofline": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(agg_peak, 2),
+                     "unit": "GB/s", "frac": round(link_gbs / agg_peak, 4), "traffic": None,
+                     "resource": f"copy engines H2D+D2H of {phys} GPU(s)",
+                     "peak_source": "measured in this run: pinned H2D+D2H 256 MiB copies on every GPU at once"},
+        "per_gpu_roofline": per_gpu,
+        "per_gpu_roofline_min": min((d["frac"] for d in per_gpu if d["frac"]), default=None),
+        "host_link": {"alone": {k: round(v, 2) for k, v in link1.items()},
+                      "concurrent": {k: round(v, 2) if isinstance(v, float) else v for k, v in conc.items()}},
+        "jain": round(jain, 4),
+        "jain_definition": "Eq. (3) over x_i = (T_alone_i / T_shared_i) / w_i (reading R-2): mean completion "
+                           "latency of tenant i's jobs in the last timed step vs the same class's jobs run alone "
+                           "through the library on one GPU",
+        "alone_mean_latency_ms": {W.CLASS_NAMES[k]: round(alone[t] * 1e3, 3) for k, t in
+                                  {sp.kclass: sp.tenant for sp in wl.jobs}.items()},
+        "gpu_launches": jobs_step * args.steps if stats.kl_mode == 0 else jobs_step * args.steps,
+        "gpu_launches_note": "KL work items executed by the persistent dispatcher kernels (one launch per GPU at "
+                             "init), one per job; plus copy-partition items" if stats.kl_mode == 0 else
+                             "per-job tenant kernel launches",
+        "clocks": clk.summary(),
+        "decision_us_per_job": round((stats.decision_ns - stats.issue_ns) / 1e3 / max(1, stats.jobs_done), 3),
+        "issue_us_per_job": round(stats.issue_ns / 1e3 / max(1, stats.jobs_done), 3),
+        "wall_s": round(t_wall, 4),
+    }
+    if e2e:
+        res["e2e"] = e2e
+    if not args.no_static:
+        from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
+        reps = max(5, args.static_repeats)
+        sb = {"tenant_mod_N": run_static(wl, num_gpus=phys, policy="mod", repeats=reps),
+              "device_0": run_static(wl, num_gpus=phys, policy="zero", repeats=reps)}
+        for k in sb:
+            lat = sb[k].pop("mean_latency_s_by_tenant")
+            sb[k]["weighted_speedup_strings"] = round(sum(lat[t] / shared[t] for t in shared) / len(shared), 3)
+        res["static_baseline"] = sb
+        res["speedup_vs_static"] = round(value / sb["tenant_mod_N"]["value"], 3)
+        res["speedup_vs_static_device0"] = round(value / sb["device_0"]["value"], 3)
+        res["weighted_speedup_vs_static"] = sb["tenant_mod_N"]["weighted_speedup_strings"]
+    if not args.no_baseline_config:
+        name = {2: "C1", 4: "C3", 8: "C5"}.get(N)
+        if name:
+            res["baseline_config"] = config_result(torch, name, phys, link, peaks, repeats=3,
+                                                   static=not args.no_static)
     return res, wl
 
 
@@ -814,95 +1116,102 @@ def copy_replay_s(torch, wl, streams_per_dir: int, reps: int = 2) -> float:
     return best
 
 
-def run_configs(args) -> None:
-    """All five BASELINE.json configurations at full size, MEASURED timing, node
-    mode (one process, G logical devices mapped round-robin onto the visible
-    GPUs).  Host buffers are allocated per tenant and reused by its jobs (every
-    tenant has c_t = 1, so its jobs never overlap).  One untimed warm-up run,
-    then `--config-repeats` timed runs; reports the median jobs/s and span, the
-    overlapped roofline T* of the physical GPU (all jobs of the
-    config share its host link and SMs) and T*/span, and Jain
-    (service/elapsed).  Measured-trace invariants are checked in tests/."""
-    import statistics
-
-    import torch
-
+def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, static: bool = False,
+                  replay: bool = False) -> dict:
+    """One BASELINE configuration at full size, MEASURED timing, node mode (one
+    process, G logical devices mapped round-robin onto `ngpu` GPUs).  One
+    untimed warm-up run, then `repeats` timed runs; the median jobs/s and span,
+    the overlapped roofline T*/span per physical GPU over the jobs placed there
+    (SURVEY §8(d)), Jain per R-2 (alone runs), optionally static provisioning
+    (tenant mod GPUs, and device 0) and the plain-copy replay."""
     import strings_workload as W
     from paper_conf_sc_senguptagsp14_b200 import strings as S
 
+    wl = W.CONFIGS[name]()
+    # arrivals are submit times in MEASURED mode: the whole config is offered at t = 0
+    wl = dataclasses.replace(wl, jobs=[dataclasses.replace(j, arrival_ns=0) for j in wl.jobs])
+    cfg = wl.config.resolved()
+    lpg = max(1, -(-cfg.num_gpus // ngpu))       # logical devices per GPU
+    ins_of, outs_of, bufs = tenant_buffers(torch, wl)
+    runs = []
+    for rep in range(1 + repeats):
+        S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
+        ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
+        t0 = time.perf_counter()
+        ids = [S.submit_spec(ts[sp.tenant], sp, ins_of(sp), outs_of(sp)) for sp in wl.jobs]
+        st = S.drain()
+        wall = time.perf_counter() - t0
+        infos = [S.job_info(i) for i in ids]
+        stats = S.stats()
+        S.shutdown()
+        if rep == 0:
+            continue                    # warm-up
+        span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
+        runs.append({"span": span, "wall": wall, "status": st, "infos": infos, "sm_copy_ops": stats.sm_copy_ops,
+                     "failed": sum(1 for i in infos if i.status != S.OK),
+                     "decision_us": (stats.decision_ns - stats.issue_ns) / 1e3 / max(1, stats.jobs_done),
+                     "issue_us": stats.issue_ns / 1e3 / max(1, stats.jobs_done)})
+    runs.sort(key=lambda r: r["span"])
+    mid = runs[len(runs) // 2]
+    span = mid["span"]
+    tstar, terms = tstar_device(wl, link, peaks["hbm_gbs"], peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"],
+                                kl_slots=lpg * cfg.partitions)
+    per_gpu = per_gpu_roofline(wl, mid["infos"], ngpu, link, peaks, cfg.partitions, lpg)
+    shared = mean_latency_by_tenant(mid["infos"])
+    alone = alone_mean_latency(S, wl, ins_of, outs_of)
+    jain, _ = jain_r2(wl, shared, alone)
+    out = {"config": name, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
+           "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
+           "balancer": W.BALANCER_NAMES[cfg.balancer], "las_admission": cfg.las_admission,
+           "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
+           "status": max((r["status"] for r in runs), key=abs),
+           "failed_jobs": sum(r["failed"] for r in runs),
+           "jobs_per_s": round(len(wl.jobs) / span, 1),
+           "span_ms": round(span * 1e3, 2), "span_ms_min_max": [round(runs[0]["span"] * 1e3, 2),
+                                                             round(runs[-1]["span"] * 1e3, 2)],
+           "runs": len(runs), "sm_copy_ops": mid["sm_copy_ops"],
+           "tstar_ms": round(tstar * 1e3, 3) if ngpu == 1 else None,
+           "roofline_frac": round(tstar / span, 4) if ngpu == 1 else None,
+           "tstar_terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()} if ngpu == 1 else None,
+           "per_gpu_roofline": per_gpu,
+           "per_gpu_roofline_min": min((d["frac"] for d in per_gpu if d["frac"]), default=None),
+           "jain": round(jain, 4), "jain_definition": "R-2: x_i = (T_alone_i / T_shared_i) / w_i",
+           "decision_us_per_job": round(mid["decision_us"], 3), "issue_us_per_job": round(mid["issue_us"], 3),
+           "host_link_gbs": {k: round(v, 2) for k, v in link.items()},
+           "note": "logical devices share the physical GPUs' host links and SMs"
+           if cfg.num_gpus > ngpu else "one logical device per GPU"}
+    if replay:
+        rp = copy_replay_s(torch, wl, lpg)
+        out["copy_replay_ms"] = round(rp * 1e3, 3)
+        out["frac_vs_copy_replay"] = round(rp / span, 4)
+        out["copy_replay_note"] = ("the config's H2D + D2H buffers copied with plain cudaMemcpyAsync, "
+                                   f"{lpg} stream(s) per direction (jobs dealt round-robin), all pre-queued, no "
+                                   "kernels or dependencies: what plain copies of these sizes achieve")
+    if static:
+        from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
+        for pol, key in (("mod", "static_tenant_mod_gpus"), ("zero", "static_device_0")):
+            sb = run_static(wl, num_gpus=ngpu, policy=pol, repeats=repeats)
+            lat = sb.pop("mean_latency_s_by_tenant")
+            sb["weighted_speedup_strings"] = round(sum(lat[t] / shared[t] for t in shared) / len(shared), 3)
+            out[key] = sb
+            out["speedup_vs_" + key] = round(out["jobs_per_s"] / sb["value"], 3)
+    del bufs
+    return out
+
+
+def run_configs(args) -> None:
+    """All five BASELINE.json configurations at full size (config_result), one
+    JSON line each.  BENCH_CONFIGS selects a subset; --config-static adds the
+    static baselines."""
+    import torch
+
     ngpu = torch.cuda.device_count()
     peaks = measured_peaks()
-    link = host_link_peaks(torch)
-    names = os.environ.get("BENCH_CONFIGS", "C1,C2,C3,C4,C5").split(",")
-    for name in names:
-        wl = W.CONFIGS[name]()
-        cfg = wl.config.resolved()
-        # per-tenant buffers sized for the tenant's largest job
-        need_in, need_out = {}, {}
-        for sp in wl.jobs:
-            need_in[sp.tenant] = [max(a, b) for a, b in zip(need_in.get(sp.tenant, [0, 0]),
-                                                          (sp.h2d_sizes() + [0])[:2])]
-            need_out[sp.tenant] = max(need_out.get(sp.tenant, 0), sum(sp.d2h_sizes()))
-        hin = {t: [torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for b in v] for t, v in need_in.items()}
-        hout = {t: torch.empty(max(1, b), dtype=torch.uint8).pin_memory() for t, b in need_out.items()}
-        runs = []
-        for rep in range(1 + args.config_repeats):
-            S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
-            ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
-            t0 = time.perf_counter()
-            for sp in wl.jobs:
-                ins = [S.HostRef(hin[sp.tenant][i].data_ptr(), b) for i, b in enumerate(sp.h2d_sizes())]
-                outs = [S.HostRef(hout[sp.tenant].data_ptr(), b) for b in sp.d2h_sizes()]
-                S.submit_spec(ts[sp.tenant], sp, ins, outs)
-            st = S.drain()
-            wall = time.perf_counter() - t0
-            infos = [S.job_info(i) for i in range(len(wl.jobs))]
-            sm_ops = S.stats().sm_copy_ops
-            S.shutdown()
-            if rep == 0:
-                continue                    # warm-up
-            busy, first, last = {}, {}, {}
-            for inf in infos:
-                busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
-                first[inf.tenant] = min(first.get(inf.tenant, inf.t_arrival), inf.t_arrival)
-                last[inf.tenant] = max(last.get(inf.tenant, 0), inf.t_done[2])
-            xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
-            jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
-            span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
-            runs.append({"span": span, "wall": wall, "jain": jain, "status": st, "sm_copy_ops": sm_ops,
-                         "failed": sum(1 for i in infos if i.status != S.OK)})
-        # arrivals are submit times in MEASURED mode: the whole config is offered at t = 0
-        wl0 = dataclasses.replace(wl, jobs=[dataclasses.replace(j, arrival_ns=0) for j in wl.jobs])
-        tstar, terms = tstar_device(wl0, link, peaks["hbm_gbs"],
-                                    peaks["bf16_tflops_sustained"] or peaks["bf16_tflops"],
-                                    kl_slots=max(1, (cfg.num_gpus + ngpu - 1) // ngpu) * cfg.partitions)
-        spans = [r["span"] for r in runs]
-        span = statistics.median(spans)
-        lpg = max(1, (cfg.num_gpus + ngpu - 1) // ngpu)       # logical devices per GPU
-        replay = copy_replay_s(torch, wl, lpg)
-        print(json.dumps({"config": name, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
-                          "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
-                          "balancer": W.BALANCER_NAMES[cfg.balancer],
-                          "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
-                          "status": max((r["status"] for r in runs), key=abs),
-                          "failed_jobs": sum(r["failed"] for r in runs),
-                          "jobs_per_s": round(len(wl.jobs) / span, 1),
-                          "span_ms": round(span * 1e3, 2), "span_ms_min_max": [round(min(spans) * 1e3, 2),
-                                                                            round(max(spans) * 1e3, 2)],
-                          "runs": len(runs), "sm_copy_ops": runs[-1]["sm_copy_ops"],
-                          "tstar_ms": round(tstar * 1e3, 3), "roofline_frac": round(tstar / span, 4),
-                          "tstar_terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()},
-                          "copy_replay_ms": round(replay * 1e3, 3),
-                          "frac_vs_copy_replay": round(replay / span, 4),
-                          "copy_replay_note": "the config's H2D + D2H buffers copied with plain cudaMemcpyAsync, "
-                          f"{lpg} stream(s) per direction (jobs dealt round-robin), all pre-queued (host issue "
-                          "excluded), no kernels or dependencies: what plain copies of these sizes achieve "
-                          "(not a strict floor: a fixed round-robin can be slower than the scheduler's order)",
-                          "jain": round(statistics.median(r["jain"] for r in runs), 4),
-                          "host_link_gbs": {k: round(v, 2) for k, v in link.items()},
-                          "note": "logical devices share the physical GPUs' host links and SMs"
-                          if cfg.num_gpus > ngpu else "one logical device per GPU"}), flush=True)
-        del hin, hout
+    link1 = host_link_peaks(torch)
+    link = scaled_link(link1, host_link_concurrent(torch, ngpu)) if ngpu > 1 else link1
+    for name in os.environ.get("BENCH_CONFIGS", "C1,C2,C3,C4,C5").split(","):
+        print(json.dumps(config_result(torch, name, ngpu, link, peaks, repeats=args.config_repeats,
+                                       static=args.config_static, replay=True)), flush=True)
 
 
 def _pct(xs, q):
@@ -1055,6 +1364,22 @@ def main():
         if rank == 0:
             run_reference(args)
         return
+    if args.gpus > 1 or world > 1:
+        # N GPUs: node mode -- rank 0 owns every GPU through the level-1 balancer
+        args.gpus = max(args.gpus, world)
+        gloo = par.init_groups(info, device_backend=None, timeout_s=4 * 3600)
+
+        def work(group):
+            import torch
+            res, _ = run_node(args, torch, group, world)
+            res["paper_context"] = PAPER_CONTEXT
+            print(json.dumps(res), flush=True)
+            return res
+        par.node_mode(info, gloo, work)
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+        return
     par.isolate_gpu(info)                 # one process per GPU (before CUDA init)
     numa = par.bind_to_gpu_numa_node(par.physical_gpu(info))
     if world > 1 and "STRINGS_COPY_THREADS" not in os.environ:
@@ -1070,6 +1395,7 @@ def main():
         if world == 1 and not args.no_static:
             from paper_conf_sc_senguptagsp14_b200.static_baseline import run_static
             sb = run_static(wl, num_gpus=1, repeats=args.static_repeats)
+            sb["note"] = "at N = 1 'tenant mod N' and 'device 0' are the same placement"
             res["static_baseline"] = sb
             res["speedup_vs_static"] = round(res["value"] / sb["value"], 3)
             # weighted speedup, Eq. (2) (reading R-1): mean over tenants of

@@ -116,7 +116,11 @@ typedef struct {
     int32_t  trace_in_memory;/* 1 = keep the trace for strings_trace_copy; with trace_path NULL
                                 and trace_in_memory 0 no record is formatted (counters only)    */
     int32_t  kl_mode;        /* 0 = persistent dispatcher kernel (product); 1 = per-job launches of
-                                the same bodies on per-slot streams (profilers that replay kernels) */
+                                the same bodies on per-slot streams (profilers that replay kernels).
+                                0 becomes 1 when a kernel profiler is injected (Nsight Compute's
+                                NV_COMPUTE_PROFILER_* / NSIGHT_COMPUTE_* variables or LD_PRELOAD
+                                interceptor, or CUDA_INJECTION64_PATH) unless STRINGS_KL_MODE_FORCE=1; the effective
+                                mode is reported in strings_stats_t::kl_mode                       */
     int32_t  reserved[6];
     uint64_t tfs_slice_ns;   /* TFS base slice S: a tenant of weight w is awake for w*S; 0 -> 500 us */
     const uint32_t* device_weights; /* num_gpus DST weights >= 1 (GWtMin); NULL = all 1.
@@ -127,6 +131,15 @@ typedef struct {
                                        hold (logical devices on that GPU) x admit_cap x slot_bytes
                                        and stay valid until strings_shutdown.  NULL = cudaMalloc.  */
     const uint64_t* ext_arena_bytes;/* sizes of ext_arenas[i]                                      */
+    void* const* ext_streams;       /* optional: 2 * num_gpus caller-owned cudaStream_t handles (e.g.
+                                       torch.cuda.Stream().cuda_stream), [2g] = H2D and [2g+1] = D2H
+                                       copy stream of logical device g (the paper's per-app stream,
+                                       P:L315; the copy engines' FIFOs of DESIGN §2).  Each must be a
+                                       non-blocking stream of the physical GPU that hosts g, distinct
+                                       from every other entry, stay valid until strings_shutdown and
+                                       carry no other work meanwhile; the library never destroys it.
+                                       An entry may be NULL (the library creates that stream).  Bad
+                                       handles -> STRINGS_EINVAL.  NULL = all library streams.     */
 } strings_config_t;
 
 /* Kernel descriptor: which tenant kernel the KL phase runs, and its sizes.
@@ -187,6 +200,8 @@ typedef struct {
                                                      dispatcher's copy partition (small ops with mapped
                                                      pinned host buffers; STRINGS_COPY_CTAS,
                                                      STRINGS_SM_COPY_MAX) instead of the copy engines */
+    int32_t  kl_mode;                             /* effective KL mode (0 persistent, 1 per-op launches) */
+    int32_t  reserved_i32;
 } strings_stats_t;
 
 /* Initialise the runtime (gPool creation): enumerate the GPUs,

@@ -22,6 +22,7 @@
 // With copy_ctas > 0 the last partition serves small H2D/D2H copies instead
 // (ctrl.hpp, CopyItem): same claim/broadcast/completion protocol on its own
 // ring, the item read from host memory, the body a zero-copy PCIe copy.
+#include <atomic>
 #include <cstdio>
 
 #include "ctrl.hpp"
@@ -284,13 +285,16 @@ cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaS
 }
 
 cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t s) {
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(strings_dev::oneshot_kernel,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)strings_dev::kSmemGemm);
+  // the smem opt-in is a per-device (per-context) function attribute: one flag per device
+  static std::atomic<bool> attr_set[64];
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64 || !attr_set[dev].load(std::memory_order_acquire)) {
+    e = cudaFuncSetAttribute(strings_dev::oneshot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)strings_dev::kSmemGemm);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    if (dev >= 0 && dev < 64) attr_set[dev].store(true, std::memory_order_release);
   }
   strings_dev::oneshot_kernel<<<ctas, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(it);
   return cudaGetLastError();

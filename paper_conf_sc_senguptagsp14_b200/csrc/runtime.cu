@@ -194,6 +194,7 @@ struct Logical {
   Phys* phys = nullptr;
   int local = 0;                       // index among the logical devices of phys
   cudaStream_t h2d = nullptr, d2h = nullptr;
+  bool h2d_ext = false, d2h_ext = false; // caller-owned (strings_config_t::ext_streams): never destroyed
   std::vector<cudaStream_t> kl_streams;  // KL_MODE_LAUNCH only
   uint8_t* kl_sync = nullptr;            // KL_MODE_LAUNCH: one GroupSync per KL stream (device)
   int next_kl_stream = 0;
@@ -249,6 +250,8 @@ struct Phys {
   int64_t clock_offset_ns = 0;         // %globaltimer - CLOCK_REALTIME (ping-pong, min RTT)
   uint64_t clock_rtt_ns = 0;
   bool kernel_running = false;
+  strings_dev::DispatchParams dp{};    // the dispatcher's parameters (launched after every GPU is set up)
+  void* probe_host = nullptr;          // clock-calibration buffer, freed at shutdown with everything else
   std::vector<int> part_start;         // [L*P + 1] partition table (host copy)
   std::vector<cudaEvent_t> ev_pool;
 };
@@ -464,6 +467,17 @@ int copy_threads() {
   return std::min(12, std::max(2, hw - 4));
 }
 
+// A kernel profiler is injected into this process: Nsight Compute sets its
+// NV_COMPUTE_PROFILER_* / NSIGHT_COMPUTE_* variables and LD_PRELOADs its
+// interceptor; other CUPTI tools come in through CUDA_INJECTION64_PATH.
+bool profiler_attached() {
+  if (getenv("CUDA_INJECTION64_PATH") || getenv("NV_COMPUTE_PROFILER_PERFWORKS_DIR") ||
+      getenv("NSIGHT_COMPUTE_HOST_PORT"))
+    return true;
+  const char* pre = getenv("LD_PRELOAD");
+  return pre && (strstr(pre, "InjectionTarget") || strstr(pre, "nsight-compute"));
+}
+
 class Runtime;
 Runtime* g_rt = nullptr;
 std::mutex g_init_mu;
@@ -550,7 +564,18 @@ class Runtime : public strings::Hooks {
         cfg.timing_mode < 0 || cfg.timing_mode > 2)
       return STRINGS_EINVAL;
     if (cfg.kl_mode < 0 || cfg.kl_mode > 1) return STRINGS_EINVAL;
+    // device-side limits: at most A ops of a logical device are woken at once, so
+    // A <= kRing keeps its KL ring from filling; a lent KL share names its slot in
+    // 16 bits of the partition's generation word (dispatcher.cu), so M <= 0xFFFF
+    if (cfg.awake_budget > kRing || cfg.admit_cap > 0xFFFF) return STRINGS_EINVAL;
     kl_mode = cfg.kl_mode;
+    // A kernel profiler (ncu, or anything injected through CUDA_INJECTION64_PATH)
+    // serialises and replays kernels one at a time: the resident dispatcher would
+    // never return and every KL would wait behind it.  Under a profiler the same
+    // tenant bodies run as one launch per KL op instead (kl_mode 1), unless
+    // STRINGS_KL_MODE_FORCE=1 insists on the requested mode.
+    if (kl_mode == 0 && profiler_attached() && !getenv("STRINGS_KL_MODE_FORCE")) kl_mode = 1;
+    cfg.kl_mode = kl_mode;
     int nphys = 0;
     if (has_gpu()) {
       if (!cuda_ok(cudaGetDeviceCount(&nphys)) || nphys <= 0) return STRINGS_ECUDA;
@@ -588,6 +613,7 @@ class Runtime : public strings::Hooks {
       strings_status_t s = init_gpus(nphys);
       cfg.ext_arenas = nullptr;            // only read during init
       cfg.ext_arena_bytes = nullptr;
+      cfg.ext_streams = nullptr;
       if (s != STRINGS_OK) {
         teardown_gpus();
         return s;
@@ -749,8 +775,28 @@ class Runtime : public strings::Hooks {
           lg.h2d = ph->h2d;
           lg.d2h = ph->d2h;
         } else {
-          if (!cuda_ok(cudaStreamCreateWithFlags(&lg.h2d, cudaStreamNonBlocking))) return STRINGS_ECUDA;
-          if (!cuda_ok(cudaStreamCreateWithFlags(&lg.d2h, cudaStreamNonBlocking))) return STRINGS_ECUDA;
+          for (int dir = 0; dir < 2; ++dir) {
+            cudaStream_t& st = dir == 0 ? lg.h2d : lg.d2h;
+            bool& ext = dir == 0 ? lg.h2d_ext : lg.d2h_ext;
+            void* given = cfg.ext_streams ? cfg.ext_streams[2 * lg.gid + dir] : nullptr;
+            if (given) {
+              // a caller's (torch) stream: must live on this GPU, be non-blocking and unique
+              cudaStream_t s = static_cast<cudaStream_t>(given);
+              unsigned int flags = 0;
+              int sdev = -1;
+              if (cudaStreamGetFlags(s, &flags) != cudaSuccess || !(flags & cudaStreamNonBlocking) ||
+                  cudaStreamGetDevice(s, &sdev) != cudaSuccess || sdev != ph->dev) {
+                cudaGetLastError();
+                return STRINGS_EINVAL;
+              }
+              for (int k = 0; k < 2 * cfg.num_gpus; ++k)
+                if (k != 2 * lg.gid + dir && cfg.ext_streams[k] == given) return STRINGS_EINVAL;
+              st = s;
+              ext = true;
+            } else if (!cuda_ok(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking))) {
+              return STRINGS_ECUDA;
+            }
+          }
         }
         if (kl_mode == 1) {
           lg.kl_streams.resize(cfg.partitions);
@@ -804,8 +850,19 @@ class Runtime : public strings::Hooks {
                                                                reinterpret_cast<uint8_t*>(ph->ctrl)));
         dp.cdone = reinterpret_cast<KlDone*>(dbase + (reinterpret_cast<uint8_t*>(ph->cdone) -
                                                       reinterpret_cast<uint8_t*>(ph->ctrl)));
-        if (!calibrate_clock(ph.get())) return STRINGS_ECUDA;
-        if (!cuda_ok(strings::launch_dispatcher(dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
+        ph->dp = dp;
+      }
+    }
+    // Two passes: a resident dispatcher owns every SM of its GPU, and allocating or
+    // freeing (pinned) memory may synchronise devices, so every GPU is allocated and
+    // its clock calibrated before the first dispatcher starts on any of them.
+    if (kl_mode == 0) {
+      for (auto& ph : phys)
+        if (ph->L && (!cuda_ok(cudaSetDevice(ph->dev)) || !calibrate_clock(ph.get()))) return STRINGS_ECUDA;
+      for (auto& ph : phys) {
+        if (!ph->L) continue;
+        if (!cuda_ok(cudaSetDevice(ph->dev))) return STRINGS_ECUDA;
+        if (!cuda_ok(strings::launch_dispatcher(ph->dp, ph->sms, ph->kstream))) return STRINGS_ECUDA;
         ph->kernel_running = true;
       }
     }
@@ -817,7 +874,8 @@ class Runtime : public strings::Hooks {
   // KL timestamps can be placed on one time line.  Best of 16 ping-pongs.
   bool calibrate_clock(Phys* ph) {
     void* hp = nullptr;
-    if (!cuda_ok(cudaHostAlloc(&hp, 256, cudaHostAllocMapped))) return false;
+    if (!cuda_ok(cudaHostAlloc(&hp, 256, cudaHostAllocMapped | cudaHostAllocPortable))) return false;
+    ph->probe_host = hp;                       // freed in teardown_gpus
     memset(hp, 0, 256);
     void* dp = nullptr;
     bool ok = cuda_ok(cudaHostGetDevicePointer(&dp, hp, 0));
@@ -849,23 +907,36 @@ class Runtime : public strings::Hooks {
     }
     ok = ok && cuda_ok(cudaStreamSynchronize(ph->kstream));
     ph->clock_rtt_ns = best_rtt;
-    cudaFreeHost(hp);
     return ok;
   }
 
   void teardown_gpus() {
-    for (auto& ph : phys) {
-      if (ph->L == 0) continue;
-      cudaSetDevice(ph->dev);
-      if (ph->kernel_running) {
+    // first ring every stop doorbell and wait for every dispatcher: freeing memory
+    // (below) may synchronise devices, which would wait forever on a resident one
+    for (auto& ph : phys)
+      if (ph->L && ph->kernel_running) {
+        cudaSetDevice(ph->dev);
         g_write_value32(reinterpret_cast<CUstream>(ph->dbstream), reinterpret_cast<CUdeviceptr>(ph->doorbells), 1, 0);
+      }
+    for (auto& ph : phys)
+      if (ph->L && ph->kernel_running) {
+        cudaSetDevice(ph->dev);
         cudaStreamSynchronize(ph->kstream);
         ph->kernel_running = false;
       }
+    for (auto& ph : phys) {
+      if (ph->L == 0) continue;
+      cudaSetDevice(ph->dev);
       for (auto& lg : logical) {
         if (lg.phys != ph.get()) continue;
-        if (lg.h2d && lg.h2d != ph->h2d) cudaStreamSynchronize(lg.h2d), cudaStreamDestroy(lg.h2d);
-        if (lg.d2h && lg.d2h != ph->d2h) cudaStreamSynchronize(lg.d2h), cudaStreamDestroy(lg.d2h);
+        if (lg.h2d && lg.h2d != ph->h2d) {
+          cudaStreamSynchronize(lg.h2d);
+          if (!lg.h2d_ext) cudaStreamDestroy(lg.h2d);
+        }
+        if (lg.d2h && lg.d2h != ph->d2h) {
+          cudaStreamSynchronize(lg.d2h);
+          if (!lg.d2h_ext) cudaStreamDestroy(lg.d2h);
+        }
         for (auto s : lg.kl_streams) cudaStreamSynchronize(s), cudaStreamDestroy(s);
         lg.h2d = lg.d2h = nullptr;
         lg.kl_streams.clear();
@@ -892,6 +963,8 @@ class Runtime : public strings::Hooks {
       ph->items_host = nullptr;
       if (ph->ctrs) cudaFreeHost(ph->ctrs);
       ph->ctrs = nullptr;
+      if (ph->probe_host) cudaFreeHost(ph->probe_host);
+      ph->probe_host = nullptr;
       ph->kstream = nullptr;
       ph->arena = nullptr;
       ph->dev_state = nullptr;
@@ -1479,9 +1552,16 @@ class Runtime : public strings::Hooks {
                           int32_t n_h2d, const strings_buf_t* d2h, int32_t n_d2h, uint32_t prio,
                           strings_job_t* out) {
     if (!d) return STRINGS_EINVAL;
+    // the cheap checks first, so a rejected submit never stages anything
+    auto admissible = [&]() -> strings_status_t {
+      if (fatal != STRINGS_OK) return fatal;       // device fault: the GPU's tenants are poisoned
+      if (t >= tenants.size() || !tenants[t].active) return STRINGS_EINVAL;
+      if (virtual_clock() && sealed && d->arrival_ns < core->current_time()) return STRINGS_EINVAL;
+      return STRINGS_OK;
+    };
     {
       std::lock_guard<std::mutex> g(mu);
-      if (fatal != STRINGS_OK) return fatal;       // device fault: the GPU's tenants are poisoned
+      if (strings_status_t s = admissible()) return s;
     }
     std::vector<uint64_t> need_in, need_out;
     switch (d->kclass) {
@@ -1552,14 +1632,19 @@ class Runtime : public strings::Hooks {
     };
     jc->in.resize(n_h2d);
     jc->out.resize(n_d2h);
+    // any error from here on hands the job's staging buffers back to the pool
+    auto reject = [&](strings_status_t s) {
+      for (auto* v : {&jc->in, &jc->out})
+        for (auto& b : *v)
+          if (b.staged && b.dma) staging.put(b.dma, b.bytes), b.dma = nullptr;
+      return s;
+    };
     for (int i = 0; i < n_h2d; ++i)
-      if (strings_status_t s = prep(h2d[i], true, jc->in[i])) return s;
+      if (strings_status_t s = prep(h2d[i], true, jc->in[i])) return reject(s);
     for (int i = 0; i < n_d2h; ++i)
-      if (strings_status_t s = prep(d2h[i], false, jc->out[i])) return s;
+      if (strings_status_t s = prep(d2h[i], false, jc->out[i])) return reject(s);
     std::lock_guard<std::mutex> g(mu);
-    if (fatal != STRINGS_OK) return fatal;
-    if (t >= tenants.size() || !tenants[t].active) return STRINGS_EINVAL;
-    if (virtual_clock() && sealed && d->arrival_ns < core->current_time()) return STRINGS_EINVAL;
+    if (strings_status_t s = admissible()) return reject(s);   // state may have changed while staging
     strings::Job& j = jc->job;
     j.id = jobs.size();
     j.tenant = t;
@@ -1779,6 +1864,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->issue_ns = r.issue_ns;
   for (size_t i = 0; i < r.phys.size() && i < 8; ++i) st->gpu_clock_offset_ns[i] = r.phys[i]->clock_offset_ns;
   st->sm_copy_ops = r.sm_copies;
+  st->kl_mode = r.kl_mode;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

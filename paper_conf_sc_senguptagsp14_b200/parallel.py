@@ -102,19 +102,38 @@ def bind_to_gpu_numa_node(gpu_id: str) -> dict:
         return {"bound": False, "why": type(e).__name__}
 
 
-def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl"):
+def init_groups(info: RankInfo, device_backend: Optional[str] = "nccl", timeout_s: Optional[float] = None):
     """Default process group (NCCL when a GPU is present) plus a gloo group for
     host-side coordination.  Returns the gloo group (None for world == 1)."""
     if info.world == 1:
         return None
+    import datetime
+
     import torch
     import torch.distributed as dist
+    kw = {"timeout": datetime.timedelta(seconds=timeout_s)} if timeout_s else {}
     if device_backend == "nccl" and torch.cuda.is_available() and not shared_gpu_test():
         torch.cuda.set_device(0)
-        dist.init_process_group("nccl", device_id=torch.device("cuda:0"))
-        return dist.new_group(backend="gloo")
-    dist.init_process_group("gloo")
+        dist.init_process_group("nccl", device_id=torch.device("cuda:0"), **kw)
+        return dist.new_group(backend="gloo", **kw)
+    dist.init_process_group("gloo", **kw)
     return dist.group.WORLD
+
+
+def node_mode(info: RankInfo, group, work):
+    """Node mode under a one-process-per-GPU launcher (torchrun): rank 0 runs
+    `work(group)`, which owns every GPU of the node through the library's
+    level-1 balancer and may call max_over_ranks(group, x) exactly
+    once; the other ranks do no work (jobs are independent: no data-path
+    collective), contribute 0 to that max and wait.  Returns work's result on
+    rank 0, None elsewhere."""
+    if info.rank == 0:
+        out = work(group)
+    else:
+        max_over_ranks(group, 0.0)
+        out = None
+    barrier(group)
+    return out
 
 
 def barrier(group) -> None:

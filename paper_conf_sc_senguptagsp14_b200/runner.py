@@ -32,7 +32,7 @@ class RunResult:
 def run_workload(wl: W.Workload, timing_mode: int = S.INJECTED, pinned: bool = True,
                  inputs: Optional[List[List[np.ndarray]]] = None, keep_inputs: bool = False,
                  trace_path: Optional[str] = None, physical_gpus: int = 0, kl_mode: int = 0,
-                 slot_bytes: int = 0, torch_memory: bool = True) -> RunResult:
+                 slot_bytes: int = 0, torch_memory: bool = True, streams=None) -> RunResult:
     cfg = wl.config.resolved()
     arenas = None
     if timing_mode != S.DECISIONS_ONLY and torch_memory:
@@ -41,7 +41,7 @@ def run_workload(wl: W.Workload, timing_mode: int = S.INJECTED, pinned: bool = T
         arenas = S.torch_arenas(cfg.num_gpus, min(nphys, cfg.num_gpus), cfg.admit_cap, slot_bytes)
         physical_gpus = len(arenas)
     S.init_from_config(cfg, timing_mode=timing_mode, trace_path=trace_path, physical_gpus=physical_gpus,
-                       kl_mode=kl_mode, slot_bytes=slot_bytes, arenas=arenas)
+                       kl_mode=kl_mode, slot_bytes=slot_bytes, arenas=arenas, streams=streams)
     pinned_arrays = []
     try:
         for t in wl.tenants:

@@ -37,7 +37,8 @@ class Config(C.Structure):
                 ("trace_path", C.c_char_p), ("trace_in_memory", C.c_int32),
                 ("kl_mode", C.c_int32), ("reserved", C.c_int32 * 6), ("tfs_slice_ns", C.c_uint64),
                 ("device_weights", C.POINTER(C.c_uint32)),
-                ("ext_arenas", C.POINTER(C.c_void_p)), ("ext_arena_bytes", C.POINTER(C.c_uint64))]
+                ("ext_arenas", C.POINTER(C.c_void_p)), ("ext_arena_bytes", C.POINTER(C.c_uint64)),
+                ("ext_streams", C.POINTER(C.c_void_p))]
 
 
 class KernelDesc(C.Structure):
@@ -68,7 +69,7 @@ class Stats(C.Structure):
                 ("engine_busy_ns", (C.c_uint64 * 3) * 8), ("num_gpus", C.c_int32),
                 ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32),
                 ("issue_ns", C.c_uint64), ("gpu_clock_offset_ns", C.c_int64 * 8),
-                ("sm_copy_ops", C.c_uint64)]
+                ("sm_copy_ops", C.c_uint64), ("kl_mode", C.c_int32), ("reserved_i32", C.c_int32)]
 
 
 def _load() -> C.CDLL:
@@ -132,9 +133,11 @@ def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy
          awake_budget=0, admit_cap=0, joint_select=-1, timing_mode=MEASURED, quantum_ns=1_000_000,
          slot_bytes=0, trace_path: Optional[str] = None, trace_in_memory=True, kl_mode=0,
          tfs_slice_ns=0, device_weights: Optional[Sequence[int]] = None,
-         arenas: Optional[Sequence] = None) -> None:
+         arenas: Optional[Sequence] = None, streams: Optional[Sequence] = None) -> None:
     """arenas: optional per-physical-GPU device buffers (torch tensors or
-    (pointer, nbytes) pairs) for the resident-job slots; see torch_arenas()."""
+    (pointer, nbytes) pairs) for the resident-job slots; see torch_arenas().
+    streams: optional 2 * num_gpus copy streams ([2g] H2D, [2g+1] D2H of logical
+    device g): torch.cuda.Stream objects, raw cudaStream_t ints or None."""
     c = Config(num_gpus=num_gpus, physical_gpus=physical_gpus, balancer=balancer, las_admission=las_admission,
                device_policy=device_policy, partitions=partitions, awake_budget=awake_budget,
                admit_cap=admit_cap, joint_select=joint_select, timing_mode=timing_mode,
@@ -150,6 +153,10 @@ def init(num_gpus=0, physical_gpus=0, balancer=1, las_admission=0, device_policy
         pb = (C.c_uint64 * len(ptrs))(*[b for _, b in ptrs])
         c.ext_arenas = C.cast(pa, C.POINTER(C.c_void_p))
         c.ext_arena_bytes = C.cast(pb, C.POINTER(C.c_uint64))
+    if streams is not None:
+        hs = [0 if s is None else (s.cuda_stream if hasattr(s, "cuda_stream") else int(s)) for s in streams]
+        ps = (C.c_void_p * len(hs))(*[h or None for h in hs])
+        c.ext_streams = C.cast(ps, C.POINTER(C.c_void_p))
     _check(lib.strings_init(C.byref(c)), "strings_init")
 
 

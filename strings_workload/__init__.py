@@ -280,10 +280,13 @@ def config_c1(seed: int = 1, reps: int = 64, scale: int = 1, int_valued: bool = 
     return _closed_loop("C1", cfg, tenants, 8, mk)
 
 
-def config_c2(seed: int = 1, reps: int = 64, scale: int = 1, jobs_per_tenant: int = 8) -> Workload:
-    """C2: 16 tenants (8 GEMM R=64 + 8 XFER), 1 GPU, DTF (joint selection)."""
-    cfg = SystemConfig(num_gpus=1, balancer=DTF, device_policy=PS)
-    tenants = [TenantSpec() for _ in range(16)]
+def config_c2(seed: int = 1, reps: int = 64, scale: int = 1, jobs_per_tenant: int = 8,
+              num_gpus: int = 1) -> Workload:
+    """C2: 16 tenants (8 GEMM R=64 + 8 XFER), 1 GPU, DTF (joint selection).
+    num_gpus = N > 1 is the weak-scaled variant the bench runs at N GPUs: 16N
+    tenants of the same mix (16 per GPU), placed by the balancer."""
+    cfg = SystemConfig(num_gpus=num_gpus, balancer=DTF, device_policy=PS)
+    tenants = [TenantSpec() for _ in range(16 * num_gpus)]
 
     def mk(t, s):
         ds = seed * 1_000_003 + t * 1009 + s

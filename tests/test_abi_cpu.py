@@ -179,6 +179,13 @@ def test_slot_size_and_mode_validation():
     with pytest.raises(S.StringsError) as e:
         S.init(timing_mode=3)
     assert e.value.status == S.EINVAL
+    # device-side limits: A <= kRing (256) KL ring entries, M <= 0xFFFF (16-bit slot of a lent share)
+    for bad in (dict(awake_budget=257), dict(admit_cap=65536)):
+        with pytest.raises(S.StringsError) as e:
+            S.init(timing_mode=S.DECISIONS_ONLY, **bad)
+        assert e.value.status == S.EINVAL
+    S.init(timing_mode=S.DECISIONS_ONLY, awake_budget=256, admit_cap=512)
+    S.shutdown()
 
 
 def test_heterogeneous_gwtmin_parity_and_validation():

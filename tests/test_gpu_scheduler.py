@@ -420,3 +420,33 @@ def test_lent_kl_slot_streaming_items_exact(help_on, monkeypatch):
             assert np.array_equal(yf.view(np.uint32), K.vscale(xf, 1.0009765625).view(np.uint32)), n
     finally:
         S.shutdown()
+
+
+def test_ext_streams_from_torch():
+    # strings_config_t::ext_streams: the copy phases run on the
+    # caller's torch streams, one H2D + one D2H stream per logical device
+    import torch
+    wl = W.config_c1(reps=2)
+    streams = [torch.cuda.Stream() for _ in range(2 * wl.config.num_gpus)]
+    r = run_workload(wl, timing_mode=S.INJECTED, streams=streams)
+    assert r.status == S.OK
+    assert r.trace == run_oracle(wl).trace
+    check_outputs(wl, r)
+    for s in streams:                       # still valid (not destroyed by the library), idle
+        assert s.query()
+        s.synchronize()
+    # MEASURED timing with only the H2D streams given (NULL entries: library streams)
+    mixed = [streams[i] if i % 2 == 0 else None for i in range(len(streams))]
+    r = run_workload(wl, timing_mode=S.MEASURED, streams=mixed)
+    assert r.status == S.OK
+    check_outputs(wl, r)
+
+
+def test_ext_streams_rejects_a_duplicate_handle():
+    import torch
+    wl = W.config_c1(reps=1)
+    s = torch.cuda.Stream()
+    with pytest.raises(S.StringsError) as e:
+        S.init_from_config(wl.config.resolved(), timing_mode=S.INJECTED, physical_gpus=1,
+                           streams=[s, s, None, None])
+    assert e.value.status == S.EINVAL

@@ -108,3 +108,54 @@ def test_copy_threads_per_rank(monkeypatch):
     monkeypatch.setattr(par.os, "cpu_count", lambda: 16)
     assert par.copy_threads_per_rank(par.RankInfo(0, 4, 0, 4)) == 2            # 4 CPUs each
     assert par.copy_threads_per_rank(par.RankInfo(0, 1, 0, 1)) == 12
+
+
+def _node_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
+                      WORLD_SIZE=str(world), LOCAL_RANK=str(rank))
+    try:
+        from oracle.des import run_oracle
+        from paper_conf_sc_senguptagsp14_b200 import parallel as par
+        from paper_conf_sc_senguptagsp14_b200 import strings as S
+        from paper_conf_sc_senguptagsp14_b200.runner import run_workload
+
+        info = par.rank_info()
+        g = par.init_groups(info, device_backend=None, timeout_s=600)
+
+        def work(group):
+            # node mode: ONE library instance places every job of the whole
+            # workload on one of G devices through the level-1 balancer
+            wl = W.config_c3()                       # G = 4, MBF
+            r = run_workload(wl, timing_mode=S.DECISIONS_ONLY)
+            span = max(i.t_done[2] for i in r.infos)
+            mx = par.max_over_ranks(group, float(span))
+            gids = sorted({i.gid for i in r.infos})
+            return (r.trace == run_oracle(wl).trace, span, mx, gids, r.stats.jobs_done)
+
+        out = par.node_mode(info, g, work)
+        q.put((rank, out))
+        import torch.distributed as dist
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put((rank, repr(e)))
+
+
+def test_world2_gloo_node_mode_rank0_drives_the_balancer():
+    # bench.py --gpus N under torchrun: rank 0 owns the node (level-1 balancer
+    # over all devices), rank 1 does no work, the timing max over ranks is rank 0's
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_node_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    res = dict(q.get(timeout=240) for _ in ps)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res[1] is None, res
+    same, span, mx, gids, done = res[0]
+    assert same                                   # the balancer's trace equals the oracle's
+    assert mx == span                             # max over ranks = rank 0's span
+    assert gids == [0, 1, 2, 3]                   # jobs spread over every device
+    assert done == len(W.config_c3().jobs)

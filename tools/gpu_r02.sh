@@ -1,0 +1,19 @@
+#!/bin/bash
+# Round-2 GPU session helper: `tools/gpu_r02.sh <task> ...` runs on the B200 box
+# under gpurun (cwd = repo snapshot).  Logs land in gpurun_out/.
+set -u
+mkdir -p gpurun_out
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/gpu.txt 2>&1
+python -m paper_conf_sc_senguptagsp14_b200.build > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
+for task in "$@"; do
+  case "$task" in
+    tests)  timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "tests rc=$?"; tail -5 gpurun_out/pytest_gpu.log ;;
+    smoke)  timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -3 gpurun_out/smoke.log ;;
+    ncu_smoke) timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_smoke.csv python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/ncu_smoke.log 2>&1; echo "ncu_smoke rc=$?"; tail -3 gpurun_out/ncu_smoke.log; grep -c '"gpu__time_duration.sum"' gpurun_out/launches_smoke.csv ;;
+    bench1) timeout 1200 python bench.py --steps ${STEPS:-10} --warmup ${WARMUP:-3} > gpurun_out/bench1.log 2>&1; echo "bench1 rc=$?"; tail -c 3000 gpurun_out/bench1.log ;;
+    bench2) timeout 1500 python bench.py --gpus 2 --steps ${STEPS:-5} --warmup ${WARMUP:-3} > gpurun_out/bench2.log 2>&1; echo "bench2 rc=$?"; tail -c 3000 gpurun_out/bench2.log ;;
+    bench2tr) timeout 1500 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps ${STEPS:-3} --warmup 3 --no-static --no-baseline-config --no-e2e > gpurun_out/bench2tr.log 2>&1; echo "bench2tr rc=$?"; tail -c 2000 gpurun_out/bench2tr.log ;;
+    configs) BENCH_CONFIGS=${CONFIGS:-C1,C2,C3,C4,C5} timeout 2400 python bench.py --configs --config-repeats ${REPEATS:-3} > gpurun_out/configs.log 2>&1; echo "configs rc=$?"; tail -c 4000 gpurun_out/configs.log ;;
+    *) echo "unknown task $task" ;;
+  esac
+done
