@@ -244,7 +244,7 @@ def kernel_rooflines(torch, S, peaks) -> list:
     xs = [torch.randint(0, 1 << 30, (n24,), dtype=torch.int32, device="cuda") for _ in range(4)]
     ys = [torch.empty_like(x) for x in xs]         # 4 rotating pairs: 512 MiB > L2
     d24 = S.make_desc(S.XFER, n=n24, seed=7)
-    for ctas in (sms // 2, sms):
+    for ctas in ((sms - 4) // 2, sms - 4):          # one KL partition beside the copy partition; two
         for i in range(4):
             S.kernel_launch(0, d24, [xs[i].data_ptr()], [ys[i].data_ptr()], ctas=ctas, stream=st.cuda_stream)
         torch.cuda.synchronize()
@@ -507,6 +507,8 @@ def run_strings(args, rank, world, torch, gloo):
                                             "half_bidir_peak": round(link["bidir_gbs"] / 2, 2)}
         if dev:
             kl_lat[name] = {"kl_device_us_p50": round(dev[len(dev) // 2], 1),
+                            "kl_device_us_mean": round(sum(dev) / len(dev), 2), "items": len(dev),
+                            "kl_body_us_mean": round(sum(body) / len(body), 2) if body else None,
                             "kl_body_us_p50": round(body[len(body) // 2], 1) if body else None,
                             "kl_host_us_p50": round(host[len(host) // 2], 1),
                             "h2d_host_us_p50": round(h2d[len(h2d) // 2], 1)}
@@ -522,11 +524,13 @@ def run_strings(args, rank, world, torch, gloo):
         "continuous": {"value": round(jobs_step * args.steps * world / dt_cont, 3), "unit": "jobs/s",
                        "frac_host_link": round(moved * args.steps / dt_cont / 1e9 / link["bidir_gbs"], 4),
                        "note": "same K batches submitted back to back, one drain (no per-step fill/drain)"},
-        "roofline": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(link["bidir_gbs"], 2),
-                     "unit": "GB/s", "frac": round(link_gbs / link["bidir_gbs"], 4), "traffic": None,
-                     "resource": "copy engines H2D+D2H (the step's dominant resource)",
-                     "peak_source": "measured in this run: concurrent pinned H2D+D2H cudaMemcpyAsync 256 MiB"},
-        "roofline_kernel": _kernel_roofline(kl_lat, wl, peaks, krl),
+        # the dominant kernel (the contract's `roofline`): the XFER work item
+        "roofline": _kernel_roofline(kl_lat, wl, peaks, krl),
+        # the step's dominant resource: the host link
+        "roofline_step": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(link["bidir_gbs"], 2),
+                          "unit": "GB/s", "frac": round(link_gbs / link["bidir_gbs"], 4), "traffic": None,
+                          "resource": "copy engines H2D+D2H (the step's dominant resource)",
+                          "peak_source": "measured in this run: concurrent pinned H2D+D2H cudaMemcpyAsync 256 MiB"},
         "overlapped_roofline": {"tstar_ms": round(tstar * 1e3, 3), "span_ms": round(span_step * 1e3, 3),
                                 "frac": round(tstar / span_step, 4),
                                 "terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()}},
@@ -840,32 +844,38 @@ def arm_config(cfg, jobs_step: int, world: int, kl_mode: int) -> dict:
 def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
     """The dominant kernel work inside the timed step: XFER items run by the
     persistent dispatcher on one P=2 SM partition (72 SMs beside the 4-CTA copy
-    partition), HBM-bound.
-    achieved = algorithmic bytes per item (read + write) / median device time
-    of the item (%globaltimer claim -> last CTA done).  Beside it: the same body
-    launched stand-alone on the same CTA count at the same size (measured in
-    this run, kernel_rooflines) -- a 128 MiB pass on 74 SMs does not reach the
-    2 GiB full-GPU rate -- and the ncu DRAM traffic of that launch."""
+    partition, plus the sibling slot's 72 when it is idle), HBM-bound.
+    achieved = algorithmic bytes per item (read + write) / MEAN device
+    time of the timed region's items (%globaltimer: leader claim -> last CTA
+    done; a launch of the persistent kernel is one work item, and CUDA events
+    cannot bracket an item inside a resident kernel).  Beside it: the median,
+    the body alone, the same body launched stand-alone on the same CTA count
+    (measured in this run, kernel_rooflines) and the ncu DRAM traffic of that
+    launch."""
     import strings_workload as W
     x = kl_lat.get("XFER")
     n = [j for j in wl.jobs if j.kclass == W.XFER][0].n
     if not x or not x["kl_device_us_p50"]:
         return None                                  # kl_mode 1: no dispatcher stamps
-    gbs = 8 * n / (x["kl_device_us_p50"] * 1e3)
-    out = {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline)", "bound": "hbm",
+    gbs = 8 * n / (x["kl_device_us_mean"] * 1e3)
+    gbs50 = 8 * n / (x["kl_device_us_p50"] * 1e3)
+    out = {"kernel": "dispatcher XFER item (fmix32, TMA bulk pipeline, dynamic chunk claiming)", "bound": "hbm",
            "achieved": round(gbs, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
            "frac": round(gbs / peaks["hbm_gbs"], 4), "traffic": _XFER_ITEM_NCU["dram_bytes"],
-           "traffic_source": _XFER_ITEM_NCU["source"],
+           "traffic_source": _XFER_ITEM_NCU["source"], "items_timed": x["items"],
+           "duration_us_mean": x["kl_device_us_mean"], "duration_us_p50": x["kl_device_us_p50"],
+           "frac_p50": round(gbs50 / peaks["hbm_gbs"], 4),
+           "peak_source": peaks["source"] + " hbm_gbs",
            "bytes_per_launch": 8 * n, "note": "per work item on its KL slot's 72 SMs plus the sibling slot's 72 "
            "when that one is idle (lent CTAs, STRINGS_KL_HELP); otherwise the other slot runs its own item and "
            "shares HBM; device time includes the claim, broadcast and completion publish (stand-alone full-GPU "
            "runs: kernel_rooflines)"}
-    if x.get("kl_body_us_p50"):
+    if x.get("kl_body_us_mean"):
         # the body alone (leader's body start -> last CTA done): without the claim and
         # the partition broadcast, which are dispatch cost, not kernel work
-        bg = 8 * n / (x["kl_body_us_p50"] * 1e3)
+        bg = 8 * n / (x["kl_body_us_mean"] * 1e3)
         out["body_only"] = {"achieved": round(bg, 1), "frac": round(bg / peaks["hbm_gbs"], 4),
-                            "us": x["kl_body_us_p50"]}
+                            "us_mean": x["kl_body_us_mean"], "us_p50": x["kl_body_us_p50"]}
     same = sorted((k for k in (krl or []) if k.get("ctas") and k["kernel"] == "XFER"), key=lambda k: k["ctas"])
     if same:
         out["same_work_standalone"] = {"ctas": same[0]["ctas"], "GBps": same[0]["achieved"],

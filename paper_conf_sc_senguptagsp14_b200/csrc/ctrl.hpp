@@ -40,7 +40,9 @@ struct __align__(128) PartState {
   uint64_t t_exec;
   // Lending an idle KL partition to its sibling's streaming item (DispatchParams::help):
   uint32_t lock;                      // 0 free, kLockOwn = running its own item, q+1 = lent to partition q
-  uint32_t total;                     // CTAs working on this partition's current item (own + lent)
+  uint32_t total;                     // CTAs working on this partition's current item (own + lent);
+                                      // 0 until the leader has decided on lending, which it does only
+                                      // after releasing its own CTAs (they read it when they finish)
   uint64_t help;                      // (kHelpGen | owner << 16 | slot) << 32 when lent, published by the owner
   GroupSync sync;                     // barrier + partials for group-wide bodies (SCAN, HIST)
 };
@@ -53,8 +55,9 @@ constexpr uint32_t kHelpGen = 0x80000000u;     // generation slot word: this is 
 // read of a work item took ~20 us; profiles/r01_doorbell.md):
 //   items[ld][slot]  work item of the job holding resident slot `slot`, DMA'd at
 //                    the job's H2D issue on the queue stream;
-//   ring[ld][i]      (seq << 32) | slot, one 64-bit stream memory op per KL on
-//                    the same stream (so after the item copy).  Entry i is
+//   ring[ld][i]      (seq << 32) | (kclass << 16) | slot, one 64-bit stream
+//                    memory op per KL on the same stream (so after the item
+//                    copy; slot < 2^16 since M <= 0xFFFF).  Entry i is
 //                    published when its seq == i + 1 (mod kRing reuse: seq is
 //                    monotone and the host never overwrites an unclaimed entry);
 //   stop             shutdown word, stream memory op at teardown.

@@ -70,7 +70,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ KlItem s_item;
   __shared__ CopyItem s_citem;
-  __shared__ uint32_t s_gen, s_slot, s_total, s_owner;
+  __shared__ uint32_t s_gen, s_slot, s_owner;
   GemmSmem sm = carve_smem(smem);
   if ((smem_u32(smem) & 1023u) != 0) __trap();   // SWIZZLE_128B tiles need a 1 KB-aligned base
   const int NK = p.L * p.P;                       // KL partitions; the copy partition (if any) is NK
@@ -97,6 +97,8 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         while (ld_acquire_gpu(&ps->done_gen) != seen) __nanosleep(32);
         uint32_t backoff = 32;
         uint64_t pub;
+        uint32_t kc = 0xFFu, slot = 0;            // class and slot of an item claimed by this partition
+        bool claimed = false;
         for (;;) {
           if (sib >= 0) {                         // lent to the sibling's item?
             const uint64_t hw = ld_acquire_gpu_u64(&ps->help);
@@ -114,19 +116,11 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
               ps->ring_idx = h % kRing;
               ps->seq = h + 1;
               ps->t_start = t_seen;
-              uint32_t total = (uint32_t)S;
-              if (sib >= 0) {
-                // a streaming item borrows the sibling slot's CTAs if that slot is idle
-                const uint32_t slot = (uint32_t)e;
-                uint32_t kc;
-                asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(kc) : "l"(&table[slot].kclass) : "memory");
-                if ((kc == 0 || kc == 2) && atomicCAS(&sps->lock, 0u, (uint32_t)q + 1) == 0u) {
-                  total += (uint32_t)S_sib;
-                  st_release_gpu_u64(&sps->help, (uint64_t)(kHelpGen | ((uint32_t)q << 16) | slot) << 32);
-                }
-              }
-              ps->total = total;
-              pub = ((uint64_t)(uint32_t)e << 32) | (seen + 1);
+              ps->total = 0;                      // decided below, after the CTAs are released
+              slot = cpart ? (uint32_t)e : ((uint32_t)e & 0xFFFFu);
+              kc = cpart ? 0xFFu : (((uint32_t)e >> 16) & 0xFFu);
+              claimed = true;
+              pub = ((uint64_t)slot << 32) | (seen + 1);
               break;
             }
             if (sib >= 0) st_release_gpu(&ps->lock, 0u);
@@ -140,7 +134,18 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
           __nanosleep(backoff);
           if (backoff < p.poll_max_ns) backoff <<= 1;
         }
-        st_release_gpu_u64(&ps->gen, pub);
+        st_release_gpu_u64(&ps->gen, pub);        // the partition's CTAs start now
+        if (claimed) {
+          // an item of this partition (own claim): a streaming item borrows the
+          // sibling slot's CTAs if that slot is idle.  Decided after the release:
+          // the own CTAs claim chunks dynamically, so lent CTAs may join late
+          uint32_t total = (uint32_t)S;
+          if (sib >= 0 && (kc == 0 || kc == 2) && atomicCAS(&sps->lock, 0u, (uint32_t)q + 1) == 0u) {
+            total += (uint32_t)S_sib;
+            st_release_gpu_u64(&sps->help, (uint64_t)(kHelpGen | ((uint32_t)q << 16) | slot) << 32);
+          }
+          st_release_gpu(&ps->total, total);
+        }
       }
       uint64_t gw = 0;
       if (lane == 0)                              // one poller per CTA
@@ -167,11 +172,6 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         s_gen = g;
         s_slot = slot;
         s_owner = lent ? ((slot_word >> 16) & 0x7FFFu) : (uint32_t)q;
-        // CTAs on this item: own partition + lent sibling (the owner wrote total before its gen)
-        s_total = (g == kStop || cpart) ? (uint32_t)S
-                  : lent ? (uint32_t)(p.part_start[((slot_word >> 16) & 0x7FFFu) + 1] -
-                                      p.part_start[(slot_word >> 16) & 0x7FFFu]) + (uint32_t)S
-                         : *reinterpret_cast<volatile uint32_t*>(&ps->total);
       }
     }
     __syncthreads();
@@ -180,27 +180,38 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     seen = g;
     const bool lent = s_owner != (uint32_t)q;
     PartState* ops = p.parts + s_owner;          // the partition whose item this is
-    const int total = (int)s_total;
+    // the owner partition's CTAs come first in the item's rank order
+    const int S_owner = lent ? p.part_start[s_owner + 1] - p.part_start[s_owner] : S;
     if (!lent && rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
     if (cpart) {
       copy_body(s_citem, rank, S);
     } else {
       const KlItem it = s_item;
       if (it.job == p.fault_job) __trap();        // fault injection (tests the watchdog)
-      // a lent CTA takes rank S_owner + rank among total (the owner's CTAs come first)
-      run_item(it, table + s_slot, true, lent ? total - S + rank : rank, total, sm, tmem, mma_phase, &ps->sync);
+      // a lent CTA takes rank S_owner + rank; it claims the owner's streaming chunks
+      // (the owner's GroupSync) and leaves a ragged tail to the owner's CTAs
+      run_item(it, table + s_slot, true, lent ? S_owner + rank : rank, S_owner, sm, tmem, mma_phase, &ops->sync,
+               &ops->total);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
+      // CTAs on this item (own + lent), published by the owner's leader after it
+      // released its CTAs (long ago by now: the load overlaps the fence below)
+      uint32_t total = ld_acquire_gpu(&ops->total);
       // D2H copy items wrote host memory: their stores must be visible system-wide
       // before the completion word; everything else only needs gpu scope
       if (cpart && s_citem.to_host)
         __threadfence_system();
       else
         __threadfence();
+      while (total == 0u) {
+        __nanosleep(32);
+        total = ld_acquire_gpu(&ops->total);
+      }
       const uint32_t old = atomicAdd(&ops->done_cnt, 1u);
-      if (old == (uint32_t)total - 1) {           // last CTA of the item (own or lent)
+      if (old == total - 1) {                     // last CTA of the item (own or lent)
         ops->done_cnt = 0;
+        ops->sync.chunk_next = 0;                 // streaming chunk counter for the next item
         KlDone* d = cpart ? &p.cdone[ops->ring_idx] : &p.done[ld * kRing + ops->ring_idx];
         d->partition = s_owner;
         d->t_start = ops->t_start;
@@ -235,16 +246,38 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
 __device__ GroupSync g_oneshot_sync;
 
 // Stand-alone launch of one tenant body on `gridDim.x` CTAs (kernel-level
-// checks outside the scheduler, and KL_MODE_LAUNCH).
+// checks outside the scheduler, and KL_MODE_LAUNCH).  One instantiation per
+// kernel class, so each contains only its own body: the register allocation of
+// one body no longer depends on the others (with every body in one kernel the
+// SORT network ran 29% slower after an unrelated streaming-body change).
+template <int KC>
 __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_constant__ KlItem it) {
   extern __shared__ __align__(1024) uint8_t smem[];
   GemmSmem sm = carve_smem(smem);
   uint32_t tmem = 0, mma_phase = 0;
-  const bool gemm = it.kclass == 1;
-  if (gemm) tmem = cta_setup(sm);
   GroupSync* gs = it.sync ? reinterpret_cast<GroupSync*>(it.sync) : &g_oneshot_sync;
-  run_item(it, &it, false, blockIdx.x, gridDim.x, sm, tmem, mma_phase, gs);
-  if (gemm) cta_teardown(tmem);
+  const int rank = blockIdx.x, S = gridDim.x;
+  if constexpr (KC == 0) {
+    stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n,
+                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, nullptr);
+  } else if constexpr (KC == 1) {
+    tmem = cta_setup(sm);
+    gemm_body(it.tmap_a, it.tmap_b, it.tmap_c, false, reinterpret_cast<float*>(it.out0), it.m, it.n, it.k, it.reps,
+              rank, S, sm, tmem, mma_phase);
+    cta_teardown(tmem);
+  } else if constexpr (KC == 2) {
+    stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n,
+                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, nullptr);
+  } else if constexpr (KC == 3) {
+    hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
+              sm.stage);
+  } else if constexpr (KC == 4) {
+    scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
+              sm.stage, sm.sbar, sm.scratch);
+  } else {
+    sort_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
+              sm.stage);
+  }
 }
 
 // Clock calibration ping-pong: sample i is taken when the host raises flag to
@@ -286,17 +319,22 @@ cudaError_t launch_clock_probe(const uint32_t* flag, uint64_t* out, int n, cudaS
 
 cudaError_t launch_oneshot(const strings_dev::KlItem& it, int ctas, cudaStream_t s) {
   // the smem opt-in is a per-device (per-context) function attribute: one flag per device
-  static std::atomic<bool> attr_set[64];
+  if (it.kclass > 5) return cudaErrorInvalidValue;
+  using K = void (*)(strings_dev::KlItem);
+  static const K kernels[6] = {strings_dev::oneshot_kernel<0>, strings_dev::oneshot_kernel<1>,
+                               strings_dev::oneshot_kernel<2>, strings_dev::oneshot_kernel<3>,
+                               strings_dev::oneshot_kernel<4>, strings_dev::oneshot_kernel<5>};
+  const K k = kernels[it.kclass];
+  static std::atomic<bool> attr_set[64][6];
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  if (dev < 0 || dev >= 64 || !attr_set[dev].load(std::memory_order_acquire)) {
-    e = cudaFuncSetAttribute(strings_dev::oneshot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)strings_dev::kSmemGemm);
+  if (dev < 0 || dev >= 64 || !attr_set[dev][it.kclass].load(std::memory_order_acquire)) {
+    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)strings_dev::kSmemGemm);
     if (e != cudaSuccess) return e;
-    if (dev >= 0 && dev < 64) attr_set[dev].store(true, std::memory_order_release);
+    if (dev >= 0 && dev < 64) attr_set[dev][it.kclass].store(true, std::memory_order_release);
   }
-  strings_dev::oneshot_kernel<<<ctas, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(it);
+  k<<<ctas, strings_dev::kThreads, strings_dev::kSmemGemm, s>>>(it);
   return cudaGetLastError();
 }
 

@@ -1100,15 +1100,18 @@ class Runtime : public strings::Hooks {
       } else if (!jc->item_ok || lg.tail - lg.completed >= (uint32_t)kRing) {
         ok = false;   // bad item (fault localised to this job); a full ring cannot happen with A <= kRing
       } else {
-        // one 64-bit stream memory op publishes ring entry (seq, slot); it is ordered
-        // after the item copy issued on the same stream at H2D time
+        // one 64-bit stream memory op publishes ring entry (seq, kclass, slot); it is
+        // ordered after the item copy issued on the same stream at H2D time.  The
+        // class rides along so the claiming leader decides on lending its sibling
+        // slot without first reading the item (ctrl.hpp)
         const uint32_t idx = lg.tail % kRing;
         const uint32_t seq = lg.tail + 1;
         jc->kl_issue = real_ns();
         jc->kl_seq = seq;
         jc->kl_idx = (int)idx;
         CUresult r = g_write_value64(reinterpret_cast<CUstream>(ph->dbstream), lg.ring_dev + sizeof(uint64_t) * idx,
-                                     ((uint64_t)seq << 32) | (uint32_t)jc->slot, 0);
+                                     ((uint64_t)seq << 32) | ((uint32_t)jc->desc.kclass << 16) | (uint32_t)jc->slot,
+                                     0);
         if (r != CUDA_SUCCESS) {
           g_last_cuda_error.store(10000 + (int32_t)r);
           ok = false;

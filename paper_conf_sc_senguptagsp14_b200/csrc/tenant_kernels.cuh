@@ -57,6 +57,18 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       :: "r"(a), "r"(parity) : "memory");
 }
 
+// A "group" is the S CTAs running one item (an SM partition of the dispatcher,
+// or a stand-alone grid).  All of them are co-resident (one CTA per SM), so a
+// counter/generation barrier in global memory is safe.
+struct __align__(128) GroupSync {
+  uint32_t bar_cnt;
+  uint32_t bar_gen;
+  uint32_t chunk_next;                 // streaming items: next unclaimed 32 KB chunk (dynamic claiming)
+  uint32_t chunk_done;                 // streaming items: CTAs finished claiming (the last one resets both)
+  uint32_t pad[28];
+  uint32_t partial[256];               // per-CTA partial results (S <= 256)
+};
+
 // ---------------------------------------------------------------- streaming
 __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
   h ^= h >> 16;
@@ -171,15 +183,31 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
-// Streaming body: the buffer is cut into 32 KB chunks; chunk c belongs to CTA
-// (c mod S).  Each CTA runs a 6-stage TMA bulk-copy pipeline through shared
-// memory (cp.async.bulk global->smem with mbarrier completion, the element op
-// in smem, cp.async.bulk smem->global), keeping 4 chunks (128 KB) of loads in
-// flight per SM while the previous chunk's store drains.  Unaligned buffers
-// and the tail use the LDG path.
+// Streaming body: the buffer is cut into 32 KB chunks.  The first kStreamLead
+// rounds go statically to the group's own CTAs (no atomic before the first
+// loads); the rest are CLAIMED dynamically from a per-item counter
+// (GroupSync::chunk_next): CTAs that
+// start late (an idle sibling partition lending its SMs joins a microsecond or
+// two after the owner's) or run slower simply take fewer chunks, so the item
+// ends when the bytes are done rather than when the slowest CTA's static share
+// is.  Each CTA runs a 6-stage TMA bulk-copy pipeline through shared memory
+// (cp.async.bulk global->smem with mbarrier completion, the element op in smem,
+// cp.async.bulk smem->global), keeping 4 chunks (128 KB) of loads in flight per
+// SM while the previous chunk's store drains; thread 0 claims the chunk of a
+// load one iteration before it issues it (so the atomic's round trip is off the
+// pipeline's critical path) and records it for the stage in smem (`cid`).
+// A stage whose claim came back empty gets an arrive without bytes and the id
+// kNoChunk, which ends the CTA's loop.  The last CTA to finish claiming resets
+// the counter for the group's next item (inside the dispatcher, total_word set,
+// the item's last CTA does, in its completion step).  Unaligned buffers and the tail (the last
+// partial chunk) use the LDG path with a static split over ranks < S (a lent
+// CTA has rank >= S and skips it).
+constexpr uint32_t kNoChunk = 0xFFFFFFFFu;
+
 template <int KCLASS>
 __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
-                            float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar) {
+                            float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar,
+                            uint32_t* cid, GroupSync* gs, const uint32_t* total_word) {
   const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   const uint64_t bytes = n * 4;
   // items too small to fill the pipeline (fewer than kStreamMinChunks chunks per CTA)
@@ -187,34 +215,59 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
   const uint64_t nchunks =
       aligned && bytes / kStreamChunk >= (uint64_t)S * kStreamMinChunks ? bytes / kStreamChunk : 0;
   if (nchunks) {
-    const uint64_t my = (uint64_t)rank < nchunks ? (nchunks - 1 - rank) / S + 1 : 0;
-    if (threadIdx.x == 0) {
-      for (int s = 0; s < kStreamStages; ++s) mbar_init(&sbar[s], 1);
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
     const uint8_t* xb = reinterpret_cast<const uint8_t*>(x);
     uint8_t* yb = reinterpret_cast<uint8_t*>(y);
-    if (threadIdx.x == 0)
-      for (int s = 0; s < kStreamLead && (uint64_t)s < my; ++s) {
-        mbar_expect_tx(&sbar[s], kStreamChunk);
-        bulk_g2s(stage + s * kStreamChunk, xb + (rank + (uint64_t)s * S) * kStreamChunk, kStreamChunk, &sbar[s]);
+    uint32_t next = kNoChunk;                     // thread 0: the claim for the next load
+    bool claiming = true;                         // thread 0: the counter may still hold chunks
+    // The first kStreamLead rounds are dealt statically to the group's own CTAs
+    // (chunk rank + j*S): their loads go out at once, with no atomic round trip
+    // on the item's start-up path; the counter hands out the chunks after them.
+    const uint64_t dealt = nchunks < (uint64_t)kStreamLead * S ? nchunks : (uint64_t)kStreamLead * S;
+    int pre = 0;                                  // thread 0: statically dealt chunks used so far
+    auto claim = [&]() -> uint32_t {
+      if (rank < S && pre < kStreamLead) {
+        const uint64_t c = (uint64_t)rank + (uint64_t)(pre++) * S;
+        if (c < dealt) return (uint32_t)c;
+        pre = kStreamLead;                        // this CTA's static share is used up
       }
-    for (uint64_t i = 0; i < my; ++i) {
-      const int s = (int)(i % kStreamStages);
+      const uint64_t c = dealt + atomicAdd(&gs->chunk_next, 1u);
+      return c < nchunks ? (uint32_t)c : kNoChunk;
+    };
+    // thread 0: fill stage st with the chunk claimed earlier (or end the CTA's loop there)
+    auto issue = [&](int st) {
+      const uint32_t c = claiming ? next : kNoChunk;
+      cid[st] = c;
+      if (c == kNoChunk) {
+        claiming = false;
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(&sbar[st])) : "memory");
+        return;
+      }
+      mbar_expect_tx(&sbar[st], kStreamChunk);
+      bulk_g2s(stage + st * kStreamChunk, xb + (uint64_t)c * kStreamChunk, kStreamChunk, &sbar[st]);
+      next = claim();                             // consumed at the next issue
+    };
+    if (threadIdx.x == 0) {
+      for (int st = 0; st < kStreamStages; ++st) mbar_init(&sbar[st], 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      next = claim();
+      for (int st = 0; st < kStreamLead && claiming; ++st) issue(st);
+    }
+    __syncthreads();
+    for (uint64_t i = 0;; ++i) {
+      const int st = (int)(i % kStreamStages);
       const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
-      if (threadIdx.x == 0 && i + kStreamLead < my) {
+      if (threadIdx.x == 0 && claiming) {
         const int s2 = (int)((i + kStreamLead) % kStreamStages);
         // stage s2 was last stored at iteration i + kStreamLead - kStreamStages: that
         // store must have finished reading smem before the load overwrites it
         if (i + kStreamLead >= (uint64_t)kStreamStages)
           asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStoreSlack) : "memory");
-        mbar_expect_tx(&sbar[s2], kStreamChunk);
-        bulk_g2s(stage + s2 * kStreamChunk, xb + (rank + (i + kStreamLead) * S) * kStreamChunk,
-                 kStreamChunk, &sbar[s2]);
+        issue(s2);
       }
-      mbar_wait(&sbar[s], ph);
-      uint4* buf = reinterpret_cast<uint4*>(stage + s * kStreamChunk);
+      mbar_wait(&sbar[st], ph);
+      const uint32_t c = *reinterpret_cast<volatile uint32_t*>(&cid[st]);
+      if (c == kNoChunk) break;                   // every thread sees the same end stage
+      uint4* buf = reinterpret_cast<uint4*>(stage + st * kStreamChunk);
 #pragma unroll 4
       for (int j = threadIdx.x; j < (int)(kStreamChunk / 16); j += kThreads) {
         uint4 v = buf[j];
@@ -226,15 +279,27 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // smem writes -> async proxy
       __syncthreads();
-      if (threadIdx.x == 0) bulk_s2g(yb + (rank + i * S) * kStreamChunk, stage + s * kStreamChunk, kStreamChunk);
+      if (threadIdx.x == 0) bulk_s2g(yb + (uint64_t)c * kStreamChunk, stage + st * kStreamChunk, kStreamChunk);
     }
     if (threadIdx.x == 0) {
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");                   // writes done
       asm volatile("fence.proxy.async.global;" ::: "memory");                     // async -> generic
+      // every claim of this CTA has returned (the last one came back empty and was
+      // consumed): count out; the last CTA of a stand-alone group resets the
+      // counter.  Inside the dispatcher (total_word set) the item's last CTA
+      // resets it instead, in the completion step it runs anyway.
+      if (!total_word) {
+        __threadfence();
+        if (atomicAdd(&gs->chunk_done, 1u) == (uint32_t)S - 1) {
+          atomicExch(&gs->chunk_next, 0u);
+          atomicExch(&gs->chunk_done, 0u);
+          __threadfence();
+        }
+      }
     }
-    __syncthreads();
+    __syncthreads();                              // cid / stages free for the next item
   }
-  stream_ldg<KCLASS>(x, y, nchunks * (kStreamChunk / 4), n, alpha, seed, rank, S);
+  if (rank < S) stream_ldg<KCLASS>(x, y, nchunks * (kStreamChunk / 4), n, alpha, seed, rank, S);
 }
 
 // --------------------------------------------------------------------- GEMM
@@ -447,12 +512,6 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, const v
 // A "group" is the S CTAs running one item (an SM partition of the dispatcher,
 // or a stand-alone grid).  All of them are co-resident (one CTA per SM), so a
 // counter/generation barrier in global memory is safe.
-struct __align__(128) GroupSync {
-  uint32_t bar_cnt;
-  uint32_t bar_gen;
-  uint32_t pad[30];
-  uint32_t partial[256];               // per-CTA partial results (S <= 256)
-};
 
 __device__ __forceinline__ void group_barrier(GroupSync* gs, int S) {
   __syncthreads();
@@ -805,8 +864,12 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
 // Run one work item on this CTA (rank of S).
 // `tmaps` is the item as it sits in global memory (dispatcher mailbox,
 // tmap_global = true) or in kernel-parameter space (stand-alone launches).
+// rank / S: this CTA's rank and the group's own CTA count (a lent CTA of a
+// streaming item has rank >= S); total_word: the dispatcher's word holding the
+// item's CTA count with lent ones (nullptr = S).
 __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, bool tmap_global, int rank, int S,
-                                         const GemmSmem& sm, uint32_t tmem_base, uint32_t& mma_phase, GroupSync* gs) {
+                                         const GemmSmem& sm, uint32_t tmem_base, uint32_t& mma_phase, GroupSync* gs,
+                                         const uint32_t* total_word) {
   switch (it.kclass) {
     case 3:
       hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
@@ -822,11 +885,11 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
       break;
     case 0:
       stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, total_word);
       break;
     case 2:
       stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, total_word);
       break;
     case 1:
       gemm_body(tmaps->tmap_a, tmaps->tmap_b, tmaps->tmap_c, tmap_global, reinterpret_cast<float*>(it.out0), it.m,

@@ -4,7 +4,7 @@
         -o gpurun_out/prof python tools/kernel_probe.py
 
 Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2);
-`xfer_item`: XFER n=2^24 on 74 CTAs (x2), the C2 work item on one P=2 partition;
+`xfer_item`: XFER n=2^24 on 72 then 144 CTAs (x2 each), the C2 work item on one P=2 partition;
 `hist` (2^30 bytes), `scan`, `sort` (2^28 u32): the NEXT-2 bodies.
 The persistent dispatcher runs exactly these device bodies on its SM partitions.
 """
@@ -33,15 +33,18 @@ def main():
         torch.cuda.synchronize()
         del x, y
     if "xfer_item" in which:
-        # the C2 work item as the dispatcher runs it: XFER 2^24 u32 on a 74-SM partition
+        # the C2 work item as the dispatcher runs it: XFER 2^24 u32 on one 72-SM KL
+        # partition (148 SMs - 4 copy-partition CTAs, P = 2), and on 144 SMs (an idle
+        # sibling slot lending its CTAs); 4 rotating buffer pairs (512 MiB > L2)
         n24 = 1 << 24
-        x = torch.randint(0, 1 << 30, (n24,), dtype=torch.int32, device="cuda")
-        y = torch.empty_like(x)
-        for _ in range(2):
-            S.kernel_launch(0, S.make_desc(S.XFER, n=n24, seed=7), [x.data_ptr()], [y.data_ptr()], ctas=74,
-                            stream=st)
+        xs = [torch.randint(0, 1 << 30, (n24,), dtype=torch.int32, device="cuda") for _ in range(4)]
+        ys = [torch.empty_like(x) for x in xs]
+        for ctas in (72, 144):
+            for i in range(2):
+                S.kernel_launch(0, S.make_desc(S.XFER, n=n24, seed=7), [xs[i].data_ptr()], [ys[i].data_ptr()],
+                                ctas=ctas, stream=st)
         torch.cuda.synchronize()
-        del x, y
+        del xs, ys
     if "gemm" in which:
         m, nn, k, reps = 128 * 148, 256, 256, 64
         a = torch.randint(-2, 3, (m, k), device="cuda").to(torch.bfloat16)
