@@ -76,6 +76,8 @@ def parse_args():
     p.add_argument("--open-loop", action="store_true",
                    help="C4 open loop: jobs submitted at their Eq. (4) arrival times; p50/p99 latency per "
                    "priority class, LAS+GUF vs arrival-order GMin+FIFO; not the driver line")
+    p.add_argument("--open-loop-config", default="C4", choices=["C4", "C4c"],
+                   help="C4c: the admission-contention variant (rho = 2, c_t = 4, M = 4)")
     p.add_argument("--open-loop-dilate", type=float, default=0.0,
                    help="arrival-time dilation (0 = logical devices per physical GPU, so the offered load "
                    "per physical host link is the config's rho)")
@@ -1253,7 +1255,7 @@ def open_loop(args) -> None:
     ngpu = torch.cuda.device_count()
     peaks = measured_peaks()
     link = host_link_peaks(torch)
-    base = W.CONFIGS["C4"]()
+    base = W.CONFIGS[args.open_loop_config]()
     lpg = max(1, (base.config.num_gpus + ngpu - 1) // ngpu)
     dil = args.open_loop_dilate or float(lpg)
     wl = dataclasses.replace(base, jobs=[dataclasses.replace(j, arrival_ns=int(j.arrival_ns * dil))
@@ -1315,11 +1317,18 @@ def open_loop(args) -> None:
                     f.write(json.dumps({"tenant": sp.tenant, "cls": W.CLASS_NAMES[sp.kclass], "gid": inf.gid,
                                         "arr": inf.t_arrival, "place": inf.t_place, "start": list(inf.t_start),
                                         "done": list(inf.t_done)}) + "\n")
-        lat = {}
+        lat, slow = {}, {}
         for sp, inf in zip(run_wl.jobs, infos):
             lat.setdefault(weight_of[sp.tenant], []).append((inf.t_done[2] - inf.t_arrival) / 1e6)
+            # slowdown: latency / the job's nominal solo chain (H2D + KL + D2H at the injected
+            # rates), so classes with different job mixes compare
+            solo = max(1, sp.inj_h2d_ns + sp.inj_kl_ns + sp.inj_d2h_ns)
+            slow.setdefault(weight_of[sp.tenant], []).append((inf.t_done[2] - inf.t_arrival) / solo)
         per_class = {f"w={w}": {"jobs": len(v), "p50_ms": round(_pct(v, 0.5), 3), "p99_ms": round(_pct(v, 0.99), 3),
-                                "mean_ms": round(sum(v) / len(v), 3)} for w, v in sorted(lat.items(), reverse=True)}
+                                "mean_ms": round(sum(v) / len(v), 3),
+                                "slowdown_mean": round(sum(slow[w]) / len(slow[w]), 2),
+                                "slowdown_p99": round(_pct(slow[w], 0.99), 2)}
+                     for w, v in sorted(lat.items(), reverse=True)}
         busy, first, last = {}, {}, {}
         for inf in infos:
             busy[inf.tenant] = busy.get(inf.tenant, 0) + sum(inf.t_done[x] - inf.t_start[x] for x in range(3))
@@ -1328,7 +1337,7 @@ def open_loop(args) -> None:
         xs = [busy[t] / max(1, last[t] - first[t]) / wl.tenants[t].weight for t in busy]
         jain = sum(xs) ** 2 / (len(xs) * sum(x * x for x in xs))
         span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
-        print(json.dumps({"config": "C4 open loop", "scheduler": name, "status": st,
+        print(json.dumps({"config": f"{args.open_loop_config} open loop", "scheduler": name, "status": st,
                           "failed_jobs": sum(1 for i in infos if i.status != S.OK),
                           "jobs": len(wl.jobs), "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
                           "timing": "INJECTED (virtual)" if injected else "MEASURED",

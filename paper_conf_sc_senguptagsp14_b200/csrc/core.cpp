@@ -509,7 +509,7 @@ void Core::complete(const Completion& c) {
 void Core::feedback(uint64_t t, Job* j) {
   // Request Monitor -> Feedback Engine -> SFT (R-14)
   uint64_t smp[3];
-  for (int x = 0; x < 3; ++x) smp[x] = j->done[x] - j->start[x];
+  for (int x = 0; x < 3; ++x) smp[x] = j->measured[x] ? j->measured[x] : j->done[x] - j->start[x];
   uint64_t span = t - j->t_place;
   uint64_t util = span ? (smp[ENG_KL] * 65536) / span : 0;
   SftRow& r = sft_[j->tenant * K_NCLASS + j->kclass];

@@ -46,6 +46,11 @@ struct Job {
   uint64_t arrival = 0;
   uint64_t h2d_bytes = 0, d2h_bytes = 0, hbm_bytes = 0, flop = 0;
   uint64_t dur[3] = {0, 0, 0};        // injected durations
+  // MEASURED mode: a phase's busy time measured on the device (KL: the
+  // dispatcher's %globaltimer claim -> last CTA), fed to the SFT instead of the
+  // host-observed DONE - START, which adds the publish and completion-observation
+  // latency; 0 = not measured (the host-observed time is used)
+  uint64_t measured[3] = {0, 0, 0};
   // decision state
   bool arrived = false, placed = false;
   int gid = -1;

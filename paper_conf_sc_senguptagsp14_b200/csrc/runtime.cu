@@ -1326,6 +1326,8 @@ class Runtime : public strings::Hooks {
       jc->kl_t1 = d->t_end;
       jc->kl_exec = d->t_exec;
       jc->kl_observe = real_ns();
+      // MEASURED timing: the SFT learns the KL's device time (R-14 telemetry)
+      if (!virtual_clock() && jc->kl_t1 > jc->kl_t0) jc->job.measured[strings::ENG_KL] = jc->kl_t1 - jc->kl_t0;
       lg.completed += 1;
       jc->phys_done[engine] = true;
       return true;

@@ -356,7 +356,23 @@ def config_c5(seed: int = 1, reps: int = 64, scale: int = 1, jobs_per_tenant: in
     return _closed_loop("C5", cfg, tenants, jobs_per_tenant, mk)
 
 
-CONFIGS = {"C1": config_c1, "C2": config_c2, "C3": config_c3, "C4": config_c4, "C5": config_c5}
+def config_c4c(seed: int = 1, reps: int = 64, scale: int = 1, jobs_per_tenant: int = 32) -> Workload:
+    """C4 under admission contention (not a BASELINE.json config; the variant
+    that exercises LAS at the balancer): the same 64 tenants
+    and skewed weights, offered twice the box's capacity (rho = 2.0), each
+    tenant with c_t = 4 requests in flight, at most M = 4 resident jobs per
+    device -- so admissions queue and the weighted-LAS order decides who goes
+    next."""
+    wl = config_c4(seed=seed, reps=reps, scale=scale, rho=2.0, jobs_per_tenant=jobs_per_tenant)
+    for t in wl.tenants:
+        t.max_inflight = 4
+    wl.config.admit_cap = 4
+    wl.name = "C4c"
+    return wl
+
+
+CONFIGS = {"C1": config_c1, "C2": config_c2, "C3": config_c3, "C4": config_c4, "C5": config_c5,
+           "C4c": config_c4c}
 
 # ----------------------------------------------------------------------------
 # NEXT-2: the paper's pairwise mix (PAPER.md L877: 6 long x 4 short apps -> 24

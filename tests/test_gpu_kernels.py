@@ -11,6 +11,7 @@ import pytest
 
 import strings_workload as W
 from oracle import kernels as K
+from gemm_bounds import gemm_elementwise_ok
 from paper_conf_sc_senguptagsp14_b200 import strings as S
 
 pytestmark = pytest.mark.gpu
@@ -90,6 +91,7 @@ def test_gemm_random_inputs_within_tolerance(m, n, k):
     ref = K.gemm(a, b)
     err = np.max(np.abs(c.astype(np.float64) - ref)) / np.max(np.abs(ref))
     assert err <= 1e-5, err
+    assert gemm_elementwise_ok(c, a, b)
 
 
 def test_gemm_structured_operands_catch_layout_errors():

@@ -157,3 +157,22 @@ def test_sort_segments_sorted_permutation():
         assert np.all(b[1:] >= b[:-1])                        # ascending
         assert sorted(a.tolist()) == b.tolist()               # a permutation of its own segment
     assert K.sort_segments(np.array([3, 1, 2, 0], np.uint32), seg=4).tolist() == [0, 1, 2, 3]
+
+
+def test_gemm_elementwise_bound_accepts_fp32_accumulation_and_rejects_errors():
+    # the GPU tests' element-wise GEMM bound (tests/gemm_bounds.py, R-22): a plain
+    # sequential fp32 accumulation of the exact bf16 products stays inside it; a
+    # result rounded to bf16, or one with a single wrong product, does not
+    from gemm_bounds import gemm_elementwise_ok
+    rng = np.random.default_rng(5)
+    a = W.f32_to_bf16_bits(rng.uniform(-1, 1, (128, 256)).astype(np.float32))
+    b = W.f32_to_bf16_bits(rng.uniform(-1, 1, (256, 256)).astype(np.float32))
+    af, bf = K.bf16_bits_to_f64(a).astype(np.float32), K.bf16_bits_to_f64(b).astype(np.float32)
+    c = np.zeros((128, 256), np.float32)
+    for kk in range(256):
+        c += af[:, kk:kk + 1] * bf[kk:kk + 1, :]
+    assert gemm_elementwise_ok(c, a, b)
+    assert not gemm_elementwise_ok(K.bf16_bits_to_f64(W.f32_to_bf16_bits(c)).astype(np.float32), a, b)
+    bad = c.copy()
+    bad[3, 7] += af[3, 11] * bf[11, 7]           # one product counted twice
+    assert not gemm_elementwise_ok(bad, a, b)

@@ -254,3 +254,66 @@ def test_eq1_partial_epoch_service_splits_at_the_boundary():
     ep = [(int(f[0]), int(f[8]), int(f[9])) for f in (ln.split() for ln in o.trace)
           if f[1] == "EPOCH" and f[5] == "1"]
     assert ep[:2] == [(1_000_000, 600_000, 31_457_280_000), (2_000_000, 600_000, 37_748_736_000)]
+
+
+# ------------------------------------------------- LAS at the balancer (L693)
+def _las_admission_blocks(weights):
+    """Two tenants, 30 identical 100 us KL-only jobs each, all at t = 0, one
+    resident job at a time (M = 1), weighted-LAS admission, Q = 1 ms.  Returns
+    the tenant of each PLACE in order."""
+    cfg = W.SystemConfig(num_gpus=1, partitions=1, awake_budget=1, admit_cap=1, balancer=W.GMIN,
+                         las_admission=1, device_policy=W.FIFO, quantum_ns=1_000_000)
+    jobs = [kl_only(t, 100_000) for _ in range(30) for t in (0, 1)]
+    o = run_oracle(W.Workload("las", cfg, [W.TenantSpec(weight=w) for w in weights], jobs))
+    return [int(f[5]) for f in (ln.split() for ln in o.trace) if f[1] == "PLACE"]
+
+
+def test_las_admission_alternates_whole_epochs_between_equal_tenants():
+    # PAPER.md L693-695 + R-7: the LAS key is the decayed service CGS, which only
+    # changes at epoch boundaries; within an epoch the lower key keeps winning.
+    # Epoch 1: both CGS = 0, tie -> tenant 0 takes all 10 admissions (1 ms / 100 us).
+    # At 1 ms: CGS_0 = 4*(1e6 << 16)/5 = 52,428,800,000 > CGS_1 = 0 -> tenant 1's epoch;
+    # at 2 ms: CGS_0 = 52,428,800,000/5 = 10,485,760,000 < CGS_1 = 52,428,800,000 -> tenant 0 ...
+    seq = _las_admission_blocks((1, 1))
+    assert seq[:40] == [0] * 10 + [1] * 10 + [0] * 10 + [1] * 10
+
+
+def test_las_admission_weights_divide_the_decayed_service():
+    # R-7: a before b iff CGS_a * p_b < CGS_b * p_a.  Weights 8 : 1, per epoch:
+    #   1: tie 0 = 0 -> tenant 0         CGS = (52,428,800,000, 0)
+    #   2: 52.4e9 * 1 > 0 * 8 -> 1       CGS = (10,485,760,000, 52,428,800,000)
+    #   3: 10.5e9 * 1 < 52.4e9 * 8 -> 0  CGS = (54,525,952,000, 10,485,760,000)
+    #   4: 54.5e9 * 1 < 10.5e9 * 8 -> 0  CGS = (63,333,990,400, 2,097,152,000)
+    #   5: 63.3e9 * 1 > 2.1e9 * 8 -> 1
+    # (with k = 0.8 the decay is steep, so a weight of 8 buys 2 epochs of 3, not 8 of 9)
+    seq = _las_admission_blocks((8, 1))
+    assert seq[:50] == [0] * 10 + [1] * 10 + [0] * 20 + [1] * 10
+
+
+def test_c4c_admissions_are_capacity_blocked():
+    # the contention variant exists to exercise LAS at the balancer: jobs that
+    # had arrived wait for a device with room (c_t = 4 x 64 tenants vs M = 4 x 8)
+    wl = W.config_c4c()
+    o = Oracle(wl)
+    blocked = []
+    orig = o.admission
+
+    def counted(t):
+        orig(t)
+        # the admission loop stopped; if an eligible job is left, no device had room
+        elig = [tn for tn in o.tenants if tn.pending and tn.inflight < tn.c and o.jobs[tn.pending[0]].arrived]
+        if elig:
+            blocked.append(t)
+    o.admission = counted
+    o.run()
+    assert len(blocked) > 100
+    base = Oracle(W.config_c4())                 # the BASELINE C4 never blocks on capacity
+    orig_b, blocked_b = base.admission, []
+
+    def counted_b(t):
+        orig_b(t)
+        if any(tn.pending and tn.inflight < tn.c and base.jobs[tn.pending[0]].arrived for tn in base.tenants):
+            blocked_b.append(t)
+    base.admission = counted_b
+    base.run()
+    assert blocked_b == []
