@@ -16,6 +16,7 @@ for task in "$@"; do
     configs) BENCH_CONFIGS=${CONFIGS:-C1,C2,C3,C4,C5} timeout 2400 python bench.py --configs --config-repeats ${REPEATS:-3} > gpurun_out/configs.log 2>&1; echo "configs rc=$?"; tail -c 4000 gpurun_out/configs.log ;;
     ncu_item) timeout 900 ncu --set full --clock-control none --import-source on -k regex:oneshot -c 4 -f -o gpurun_out/prof_xfer_item python tools/kernel_probe.py xfer_item > gpurun_out/ncu_item.log 2>&1; echo "ncu_item rc=$?"; tail -3 gpurun_out/ncu_item.log ;;
     ncu_launches) timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv --log-file gpurun_out/launches_bench.csv python bench.py --steps 2 --warmup 1 --no-static --no-e2e --no-kernels > gpurun_out/ncu_launches.log 2>&1; echo "ncu_launches rc=$?"; tail -c 600 gpurun_out/ncu_launches.log ;;
+    openloop) timeout 1800 python bench.py --open-loop --open-loop-config ${OLCFG:-C4} > gpurun_out/openloop_${OLCFG:-C4}.log 2>&1; echo "openloop rc=$?"; tail -c 1500 gpurun_out/openloop_${OLCFG:-C4}.log ;;
     *) echo "unknown task $task" ;;
   esac
 done
