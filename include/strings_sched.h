@@ -202,6 +202,9 @@ typedef struct {
                                                      STRINGS_SM_COPY_MAX) instead of the copy engines */
     int32_t  kl_mode;                             /* effective KL mode (0 persistent, 1 per-op launches) */
     int32_t  reserved_i32;
+    uint64_t eager_jobs;                          /* MEASURED: jobs whose KL and D2H were queued on the
+                                                     device behind their H2D (eager chaining, DESIGN §2;
+                                                     STRINGS_EAGER=0 disables)                        */
 } strings_stats_t;
 
 /* Initialise the runtime (gPool creation): enumerate the GPUs,

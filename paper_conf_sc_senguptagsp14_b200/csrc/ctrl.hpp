@@ -12,7 +12,11 @@
 
 namespace strings_dev {
 
-constexpr int kRing = 256;            // KL ring entries per logical device
+constexpr int kRing = 256;            // entries per KL ring
+// KL rings per logical device: 0 = entries the host publishes when the scheduler
+// wakes a KL (queue stream), 1 = entries chained on the H2D stream behind the
+// job's input copy when the KL's wake is certain (eager chaining, runtime.cu)
+constexpr int kRings = 2;
 constexpr uint32_t kStop = 0xFFFFFFFFu;
 
 struct __align__(32) KlDone {
@@ -25,7 +29,7 @@ struct __align__(32) KlDone {
 // Host-mapped part (cudaHostAlloc mapped): the completion words the GPU writes.
 struct HostCtrl {
   uint32_t pad[16];
-  // followed by KlDone[L][kRing], then the copy partition's KlDone[kRing] and CopyItem[kRing]
+  // followed by KlDone[L][kRings][kRing], then the copy partition's KlDone[kRing] and CopyItem[kRing]
 };
 
 // Device-memory part: claim counters and per-partition mailboxes.
@@ -124,12 +128,14 @@ __device__ __forceinline__ void copy_body(const CopyItem& c, int rank, int S) {
 }
 
 struct DispatchParams {
-  KlDone* done;                       // [L * kRing] host-mapped completion words
-  uint32_t* heads;                    // [L] device-memory claim counters
+  KlDone* done;                       // [L][kRings][kRing] host-mapped completion words
+  uint32_t* done_dev;                 // [L][kRings][kRing] device copies of the completion seq
+                                      // (an eager D2H waits on them: cuStreamWaitValue32)
+  uint32_t* heads;                    // [L][kRings] device-memory claim counters, [L*kRings] = copy ring
   PartState* parts;                   // [L * P]
   const int* part_start;              // [L * P + 1] first CTA of each partition (device memory)
   const uint32_t* stop;
-  const uint64_t* ring;               // [L * kRing]
+  const uint64_t* ring;               // [L][kRings][kRing]
   const KlItem* items;                // [L * M]
   int L, P, M;                        // logical devices hosted, partitions per device, slots per device
   uint32_t flags;                     // experiment knobs (STRINGS_DISPATCH_FLAGS): bit0 no poll back-off
@@ -137,15 +143,16 @@ struct DispatchParams {
   uint64_t fault_job;                 // fault injection (STRINGS_FAULT_JOB): trap on this job id
   uint32_t help;                      // 1: an idle sibling KL partition joins VSCALE/XFER items
   // copy partition (partition index L*P, CTAs [part_start[L*P], part_start[L*P+1])) when copy_ctas > 0;
-  // its claim counter is heads[L] and its PartState parts[L*P]
+  // its claim counter is heads[L * kRings] and its PartState parts[L*P]
   int copy_ctas;
+  uint32_t* progress;                 // [gridDim.x] per-CTA (generation << 4 | step) for stall dumps
   const uint64_t* cring;              // [kRing] device ring entries (seq << 32) | index
   const CopyItem* citems;             // [kRing] host-mapped copy items (device view)
   KlDone* cdone;                      // [kRing] host-mapped completion words
 };
 
 inline size_t host_ctrl_bytes(int L) {
-  return sizeof(HostCtrl) + sizeof(KlDone) * kRing * (L + 1) + sizeof(CopyItem) * kRing + 128;
+  return sizeof(HostCtrl) + sizeof(KlDone) * kRing * (L * kRings + 1) + sizeof(CopyItem) * kRing + 128;
 }
 
 }  // namespace strings_dev

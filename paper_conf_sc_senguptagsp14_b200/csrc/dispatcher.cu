@@ -29,6 +29,7 @@
 
 namespace strings_dev {
 
+
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -79,10 +80,12 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
   partition_of(blockIdx.x, NP, p.part_start, &q, &start, &S);
   const int rank = blockIdx.x - start;
   const bool cpart = q == NK;
-  const int ld = cpart ? p.L : q / p.P;           // claim counter heads[ld]
+  const int ld = cpart ? p.L : q / p.P;           // logical device (copy partition: L)
+  const int nrings = cpart ? 1 : kRings;         // KL rings of the device (host-published, eager)
   PartState* ps = p.parts + q;
   const KlItem* table = p.items + (size_t)(cpart ? 0 : ld) * p.M;
-  const uint64_t* ring = cpart ? p.cring : p.ring + (size_t)ld * kRing;
+  uint32_t* const heads = cpart ? p.heads + (size_t)p.L * kRings : p.heads + (size_t)ld * kRings;
+  const uint64_t* const rings = cpart ? p.cring : p.ring + (size_t)ld * kRings * kRing;
   // the sibling KL slot of the same logical device that may lend its CTAs (P >= 2)
   const int sib = (!cpart && p.help && (q ^ 1) < NK && (q ^ 1) / p.P == ld) ? (q ^ 1) : -1;
   PartState* sps = sib >= 0 ? p.parts + sib : nullptr;
@@ -107,13 +110,20 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
               break;
             }
           }
-          const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&p.heads[ld]);
-          const uint64_t e = ld_acquire_gpu_u64(&ring[h % kRing]);
-          if ((uint32_t)(e >> 32) == h + 1) {     // entry h published
-            if (sib >= 0 && atomicCAS(&ps->lock, 0u, kLockOwn) != 0u) continue;   // being lent: help first
+          bool retry = false;
+          // ring 0 (entries the host published at the model's wake) first, then the
+          // eager ring: an eager entry waits at most one extra L2 read, ring 0 none
+          for (int r = 0; r < nrings && !claimed; ++r) {
+            const uint32_t h = *reinterpret_cast<volatile uint32_t*>(&heads[r]);
+            const uint64_t e = ld_acquire_gpu_u64(&rings[(size_t)r * kRing + h % kRing]);
+            if ((uint32_t)(e >> 32) != h + 1) continue;            // entry h of ring r not published
+            if (sib >= 0 && atomicCAS(&ps->lock, 0u, kLockOwn) != 0u) {  // being lent: help first
+              retry = true;
+              break;
+            }
             const uint64_t t_seen = globaltimer();
-            if (atomicCAS(&p.heads[ld], h, h + 1) == h) {
-              ps->ring_idx = h % kRing;
+            if (atomicCAS(&heads[r], h, h + 1) == h) {
+              ps->ring_idx = (uint32_t)r * kRing + h % kRing;
               ps->seq = h + 1;
               ps->t_start = t_seen;
               ps->total = 0;                      // decided below, after the CTAs are released
@@ -121,11 +131,14 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
               kc = cpart ? 0xFFu : (((uint32_t)e >> 16) & 0xFFu);
               claimed = true;
               pub = ((uint64_t)slot << 32) | (seen + 1);
+            } else {
+              if (sib >= 0) st_release_gpu(&ps->lock, 0u);
+              retry = true;                       // the other KL slot took it
               break;
             }
-            if (sib >= 0) st_release_gpu(&ps->lock, 0u);
-            continue;                             // the other KL slot took it
           }
+          if (claimed) break;
+          if (retry) continue;
           if (ld_acquire_gpu(p.stop)) {
             pub = kStop;
             break;
@@ -178,6 +191,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     const uint32_t g = s_gen;
     if (g == kStop) break;
     seen = g;
+    if (threadIdx.x == 0) p.progress[blockIdx.x] = (g << 12) | (s_item.kclass << 8) | 1u;     // item read
     const bool lent = s_owner != (uint32_t)q;
     PartState* ops = p.parts + s_owner;          // the partition whose item this is
     // the owner partition's CTAs come first in the item's rank order
@@ -195,6 +209,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     }
     __syncthreads();
     if (threadIdx.x == 0) {
+      p.progress[blockIdx.x] = (seen << 12) | 2u;                     // body done
       // CTAs on this item (own + lent), published by the owner's leader after it
       // released its CTAs (long ago by now: the load overlaps the fence below)
       uint32_t total = ld_acquire_gpu(&ops->total);
@@ -209,10 +224,12 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         total = ld_acquire_gpu(&ops->total);
       }
       const uint32_t old = atomicAdd(&ops->done_cnt, 1u);
+      p.progress[blockIdx.x] = (seen << 12) | 3u;                     // counted in
       if (old == total - 1) {                     // last CTA of the item (own or lent)
         ops->done_cnt = 0;
         ops->sync.chunk_next = 0;                 // streaming chunk counter for the next item
-        KlDone* d = cpart ? &p.cdone[ops->ring_idx] : &p.done[ld * kRing + ops->ring_idx];
+        const size_t di = (size_t)ld * kRings * kRing + ops->ring_idx;
+        KlDone* d = cpart ? &p.cdone[ops->ring_idx] : &p.done[di];
         d->partition = s_owner;
         d->t_start = ops->t_start;
         d->t_exec = ops->t_exec;
@@ -223,6 +240,9 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         // (a sys-scope release costs ~3 us more per item, PCIe-fence round trip).
         __threadfence();
         d->seq = ops->seq;
+        // the device copy an eager D2H's stream waits on (gpu scope: the copy engine
+        // reads the outputs through L2, which every CTA's fence already ordered)
+        if (!cpart) st_release_gpu(&p.done_dev[di], ops->seq);
         const uint32_t og = (uint32_t)*reinterpret_cast<volatile uint64_t*>(&ops->gen);
         if (sib >= 0 || lent) st_release_gpu(&ops->lock, 0u);   // the owner may claim / lend again
         st_release_gpu(&ops->done_gen, og);
@@ -257,9 +277,10 @@ __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_const
   uint32_t tmem = 0, mma_phase = 0;
   GroupSync* gs = it.sync ? reinterpret_cast<GroupSync*>(it.sync) : &g_oneshot_sync;
   const int rank = blockIdx.x, S = gridDim.x;
+  if constexpr (KC != 1) mbar_setup(sm);          // (GEMM: cta_setup below)
   if constexpr (KC == 0) {
     stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n,
-                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, nullptr);
+                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, sm.sphase, gs, nullptr);
   } else if constexpr (KC == 1) {
     tmem = cta_setup(sm);
     gemm_body(it.tmap_a, it.tmap_b, it.tmap_c, false, reinterpret_cast<float*>(it.out0), it.m, it.n, it.k, it.reps,
@@ -267,13 +288,13 @@ __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_const
     cta_teardown(tmem);
   } else if constexpr (KC == 2) {
     stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n,
-                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, nullptr);
+                   it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, sm.sphase, gs, nullptr);
   } else if constexpr (KC == 3) {
     hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
               sm.stage);
   } else if constexpr (KC == 4) {
     scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
-              sm.stage, sm.sbar, sm.scratch);
+              sm.stage, sm.sbar, sm.scratch, sm.sphase);
   } else {
     sort_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
               sm.stage);

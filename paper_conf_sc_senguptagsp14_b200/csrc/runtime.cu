@@ -49,6 +49,7 @@ using strings_dev::KlDone;
 using strings_dev::KlItem;
 using strings_dev::CopyItem;
 using strings_dev::kRing;
+using strings_dev::kRings;
 
 namespace {
 
@@ -86,6 +87,8 @@ typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned i
 WriteValue32Fn g_write_value32 = nullptr;
 typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 WriteValue64Fn g_write_value64 = nullptr;
+typedef CUresult (*WaitValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+WaitValue32Fn g_wait_value32 = nullptr;
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -147,9 +150,10 @@ bool encode_gemm_maps(KlItem& it) {
 // (stream memory operation, ordered after the copy), so the engine thread
 // detects completion with a plain memory read instead of a driver call.
 struct __align__(64) CopyCounters {
-  volatile uint32_t done[3];          // indexed by engine (H2D = 0, D2H = 2)
-  uint32_t pad[13];
+  volatile uint32_t done[4];          // indexed by engine (H2D = 0, D2H = 2); 3 = the eager D2H stream
+  uint32_t pad[12];
 };
+constexpr int kEagerD2H = 3;          // CopyCounters / Logical::issued index of the eager D2H stream
 
 constexpr uint64_t kAlign = 256;
 inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
@@ -181,7 +185,8 @@ struct JobCtx {
   int item_cidx = -1;                              //   (CE-path H2D jobs; STRINGS_ITEM_VIA_COPY), consumed with the H2D
   uint32_t cseq[3] = {0, 0, 0};
   int cidx[3] = {-1, -1, -1};
-  int kl_idx = -1;
+  int kl_idx = -1;                     // ring * kRing + index of the KL's ring entry
+  bool eager = false;                  // KL and D2H chained on the device behind the H2D (issue())
   int kl_partition = -1;
   uint64_t kl_t0 = 0, kl_t1 = 0, kl_exec = 0;     // device %globaltimer: claim, end, body start
   uint64_t kl_issue = 0, kl_observe = 0;          // host CLOCK_REALTIME: published, completion seen
@@ -202,14 +207,16 @@ struct Logical {
   std::vector<int> free_slots;
   KlItem* item_host = nullptr;         // [M] pinned staging of the slots' work items
   CUdeviceptr item_dev = 0;            // [M] device copies (dispatcher reads them)
-  CUdeviceptr ring_dev = 0;            // [kRing] device ring entries (seq << 32 | slot)
-  KlDone* done = nullptr;              // host pointer, kRing entries
-  uint32_t tail = 0;                   // items published
-  uint32_t completed = 0;              // items whose completion was consumed
+  CUdeviceptr ring_dev = 0;            // [kRings][kRing] device ring entries (seq << 32 | kclass << 16 | slot)
+  KlDone* done = nullptr;              // host pointer, [kRings][kRing] entries
+  CUdeviceptr done_dev = 0;            // [kRings][kRing] u32 device copies of the completion seq
+  uint32_t tail[kRings] = {0, 0};      // items published per ring
+  uint32_t completed[kRings] = {0, 0}; // items whose completion was consumed, per ring
+  cudaStream_t d2h_eager = nullptr;    // eager D2H ops: wait for their KL on the device, then copy
   CopyCounters* ctr = nullptr;         // host view
   CUdeviceptr ctr_dev = 0;             // device view
   int ctas = 0;                        // CTAs (SMs) of this logical device's partitions
-  uint32_t issued[3] = {0, 0, 0};      // copy ops issued per engine
+  uint32_t issued[4] = {0, 0, 0, 0};   // copy ops issued per engine (3 = eager D2H stream)
 };
 
 struct Phys {
@@ -230,7 +237,9 @@ struct Phys {
   // stream memory ops on this stream, work items DMA'd by the H2D streams
   cudaStream_t dbstream = nullptr;
   uint8_t* doorbells = nullptr;
-  uint8_t* ring_dev = nullptr;         // [L][kRing] u64
+  uint8_t* ring_dev = nullptr;         // [L][kRings][kRing] u64
+  uint8_t* done_dev = nullptr;         // [L][kRings][kRing] u32
+  uint8_t* progress = nullptr;         // [sms] u32 per-CTA progress words (stall dumps)
   uint8_t* items_dev = nullptr;        // [L][M] KlItem
   KlItem* items_host = nullptr;        // [L][M] pinned staging
   uint64_t items_host_dev = 0;         // device view of items_host (mapped)
@@ -506,6 +515,13 @@ class Runtime : public strings::Hooks {
   uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
   uint64_t decision_ns = 0;            // time inside Core::step (decisions + op issue)
   uint64_t sm_copies = 0;              // H2D/D2H ops served by the copy partition
+  uint64_t eager_jobs = 0;             // jobs whose KL and D2H were chained on the device (eager_ok)
+  uint64_t inflight_cap_sum = 0;       // sum of the registered tenants' in-flight limits c_t
+  // STRINGS_EAGER=0 turns eager chaining off (every phase issued at its wake)
+  const bool eager_enabled = [] {
+    const char* e = getenv("STRINGS_EAGER");
+    return !(e && e[0] == '0');
+  }();
   uint64_t last_progress = 0;
   bool stall_dumped = false;
   const uint64_t stall_dump_ns = [] {
@@ -684,7 +700,7 @@ class Runtime : public strings::Hooks {
       ph->ctrl = static_cast<HostCtrl*>(hp);
       if (!cuda_ok(cudaHostGetDevicePointer(&ph->ctrl_dev, hp, 0))) return STRINGS_ECUDA;
       {
-        uint8_t* cb0 = static_cast<uint8_t*>(hp) + sizeof(HostCtrl) + sizeof(KlDone) * kRing * ph->L;
+        uint8_t* cb0 = static_cast<uint8_t*>(hp) + sizeof(HostCtrl) + sizeof(KlDone) * kRing * kRings * ph->L;
         ph->cdone = reinterpret_cast<KlDone*>(cb0);
         uint8_t* ci = cb0 + sizeof(KlDone) * kRing;
         ci += (128 - reinterpret_cast<uintptr_t>(ci) % 128) % 128;
@@ -704,16 +720,19 @@ class Runtime : public strings::Hooks {
           return STRINGS_ECUDA;
         g_write_value32 = reinterpret_cast<WriteValue32Fn>(fn);
       }
-      // device state: heads[L + 1] (padded; [L] = copy ring) + parts[L*P + 1] + partition
-      // table + doorbells (one 128-B line per logical device's ring tail, one for shutdown)
-      size_t heads_bytes = 128 * (size_t)(ph->L + 1);
+      // device state: heads[L * kRings + 1] ([L * kRings] = copy ring) + parts[L*P + 1] +
+      // partition table + shutdown doorbell + rings + device done words + item table
+      size_t heads_bytes = 128 * (size_t)((ph->L * kRings + 1) * 4 / 128 + 1);
       size_t parts_bytes = sizeof(strings_dev::PartState) * (ph->L * cfg.partitions + 1);
       size_t table_bytes = sizeof(int) * ph->part_start.size();
       size_t db_off = align_up(heads_bytes + parts_bytes + table_bytes);
       size_t db_bytes = 128;                                         // shutdown word
       size_t ring_off = align_up(db_off + db_bytes);
-      size_t ring_bytes = sizeof(uint64_t) * kRing * ph->L;
-      size_t items_off = align_up(ring_off + ring_bytes);
+      size_t ring_bytes = sizeof(uint64_t) * kRing * kRings * ph->L;
+      size_t donedev_off = align_up(ring_off + ring_bytes);
+      size_t donedev_bytes = sizeof(uint32_t) * kRing * kRings * ph->L;
+      size_t prog_off = align_up(donedev_off + donedev_bytes);
+      size_t items_off = align_up(prog_off + sizeof(uint32_t) * 1024);
       size_t items_bytes = sizeof(KlItem) * (size_t)cfg.admit_cap * ph->L;
       size_t cring_off = align_up(items_off + items_bytes);
       size_t cring_bytes = sizeof(uint64_t) * kRing;
@@ -721,6 +740,8 @@ class Runtime : public strings::Hooks {
       if (!cuda_ok(cudaMemset(ph->dev_state, 0, cring_off + cring_bytes))) return STRINGS_ECUDA;
       ph->doorbells = ph->dev_state + db_off;
       ph->ring_dev = ph->dev_state + ring_off;
+      ph->done_dev = ph->dev_state + donedev_off;
+      ph->progress = ph->dev_state + prog_off;
       ph->items_dev = ph->dev_state + items_off;
       ph->cring_dev = ph->dev_state + cring_off;
       {
@@ -741,6 +762,7 @@ class Runtime : public strings::Hooks {
           return STRINGS_ECUDA;
         g_write_value64 = reinterpret_cast<WriteValue64Fn>(fn);
       }
+      if (!driver_entry("cuStreamWaitValue32", &g_wait_value32)) return STRINGS_ECUDA;
       if (!cuda_ok(cudaMemcpy(ph->dev_state + heads_bytes + parts_bytes, ph->part_start.data(), table_bytes,
                               cudaMemcpyHostToDevice)))
         return STRINGS_ECUDA;
@@ -810,8 +832,11 @@ class Runtime : public strings::Hooks {
         for (int s = cfg.admit_cap - 1; s >= 0; --s) lg.free_slots.push_back(s);
         lg.item_host = ph->items_host + (size_t)lg.local * cfg.admit_cap;
         lg.item_dev = reinterpret_cast<CUdeviceptr>(ph->items_dev) + sizeof(KlItem) * (size_t)lg.local * cfg.admit_cap;
-        lg.ring_dev = reinterpret_cast<CUdeviceptr>(ph->ring_dev) + sizeof(uint64_t) * (size_t)kRing * lg.local;
-        lg.done = dones + (size_t)lg.local * kRing;
+        lg.ring_dev = reinterpret_cast<CUdeviceptr>(ph->ring_dev) + sizeof(uint64_t) * (size_t)kRing * kRings * lg.local;
+        lg.done = dones + (size_t)lg.local * kRing * kRings;
+        lg.done_dev = reinterpret_cast<CUdeviceptr>(ph->done_dev) + sizeof(uint32_t) * (size_t)kRing * kRings * lg.local;
+        if (kl_mode == 0 && !cuda_ok(cudaStreamCreateWithFlags(&lg.d2h_eager, cudaStreamNonBlocking)))
+          return STRINGS_ECUDA;
         lg.ctr = ph->ctrs + lg.local;
         lg.ctr_dev = reinterpret_cast<CUdeviceptr>(static_cast<CopyCounters*>(ph->ctrs_dev) + lg.local);
       }
@@ -824,6 +849,8 @@ class Runtime : public strings::Hooks {
         strings_dev::DispatchParams dp;
         uint8_t* dbase = static_cast<uint8_t*>(ph->ctrl_dev);
         dp.done = reinterpret_cast<KlDone*>(dbase + sizeof(HostCtrl));
+        dp.done_dev = reinterpret_cast<uint32_t*>(ph->done_dev);
+        dp.progress = reinterpret_cast<uint32_t*>(ph->progress);
         dp.heads = reinterpret_cast<uint32_t*>(ph->dev_state);
         dp.parts = reinterpret_cast<strings_dev::PartState*>(ph->dev_state + heads_bytes);
         dp.part_start = reinterpret_cast<const int*>(ph->dev_state + heads_bytes + parts_bytes);
@@ -938,6 +965,8 @@ class Runtime : public strings::Hooks {
           if (!lg.d2h_ext) cudaStreamDestroy(lg.d2h);
         }
         for (auto s : lg.kl_streams) cudaStreamSynchronize(s), cudaStreamDestroy(s);
+        if (lg.d2h_eager) cudaStreamSynchronize(lg.d2h_eager), cudaStreamDestroy(lg.d2h_eager);
+        lg.d2h_eager = nullptr;
         lg.h2d = lg.d2h = nullptr;
         lg.kl_streams.clear();
         if (lg.kl_sync) cudaFree(lg.kl_sync);
@@ -1005,11 +1034,49 @@ class Runtime : public strings::Hooks {
     return it.kclass != STRINGS_GEMM || encode_gemm_maps(it);
   }
 
+  // Eager chaining (MEASURED timing): when the scheduler is certain to wake a
+  // job's KL the moment its H2D completes and its D2H the moment its KL
+  // completes, the whole chain is queued on the device at H2D issue -- the KL
+  // ring entry as a stream write behind the input copy (ring 1), the D2H on its
+  // own stream behind a wait on the KL's device done word -- so no phase
+  // boundary waits for the host to observe a completion, decide and issue
+  // (SURVEY §7 hard part 3; three concurrently usable engines).
+  // The decisions and the trace are unchanged: the model still wakes and starts
+  // the KL and D2H at the completions it observes; only the physical issue moved.
+  // Certain means: a wake policy that wakes every candidate while the budget
+  // allows (FIFO, LAS, PS; not TFS) and at most A resident jobs per device
+  // (M <= A, or the tenants' in-flight limits sum to <= A), so every candidate is
+  // woken at once.  Only jobs whose copies both go to the copy engines qualify
+  // (a copy-partition op's completion is not ordered on a stream).
+  bool eager_ok(const JobCtx* jc, const Logical& lg) const {
+    if (!eager_enabled || virtual_clock() || kl_mode != 0 || item_via_copy) return false;
+    if (cfg.device_policy == STRINGS_DEV_TFS) return false;
+    if ((uint64_t)cfg.admit_cap > (uint64_t)cfg.awake_budget && inflight_cap_sum > (uint64_t)cfg.awake_budget)
+      return false;
+    if (jc->job.h2d_bytes <= sm_copy_max || jc->job.d2h_bytes <= sm_copy_max) return false;
+    return lg.tail[1] - lg.completed[1] < (uint32_t)kRing;
+  }
+
   void issue(strings::Job& j, JobCtx* jc, int engine) {
     Logical& lg = logical[j.gid];
     Phys* ph = lg.phys;
+    if (jc->eager && engine != strings::ENG_H2D) {
+      // queued on the device at H2D issue: the model's wake has nothing left to issue
+      if (!virtual_clock()) inflight.push_back({jc, engine});
+      return;
+    }
     set_dev(ph->dev);
     bool ok = true;
+    if (engine == strings::ENG_H2D && eager_ok(jc, lg)) {
+      ok = issue_eager(j, jc, lg);
+      jc->issued[engine] = true;
+      if (!ok) {
+        fail_job(jc);
+        for (int e = 0; e < 3; ++e) jc->phys_done[e] = true;
+      }
+      if (!virtual_clock()) inflight.push_back({jc, engine});
+      return;
+    }
     if (engine == strings::ENG_H2D) {
       if (jc->slot < 0) {
         jc->slot = lg.free_slots.back();
@@ -1097,15 +1164,15 @@ class Runtime : public strings::Hooks {
     } else if (kl_mode == 0) {
       if (!await_item_copy(ph, jc)) {
         ok = false;
-      } else if (!jc->item_ok || lg.tail - lg.completed >= (uint32_t)kRing) {
+      } else if (!jc->item_ok || lg.tail[0] - lg.completed[0] >= (uint32_t)kRing) {
         ok = false;   // bad item (fault localised to this job); a full ring cannot happen with A <= kRing
       } else {
         // one 64-bit stream memory op publishes ring entry (seq, kclass, slot); it is
         // ordered after the item copy issued on the same stream at H2D time.  The
         // class rides along so the claiming leader decides on lending its sibling
         // slot without first reading the item (ctrl.hpp)
-        const uint32_t idx = lg.tail % kRing;
-        const uint32_t seq = lg.tail + 1;
+        const uint32_t idx = lg.tail[0] % kRing;
+        const uint32_t seq = lg.tail[0] + 1;
         jc->kl_issue = real_ns();
         jc->kl_seq = seq;
         jc->kl_idx = (int)idx;
@@ -1116,7 +1183,7 @@ class Runtime : public strings::Hooks {
           g_last_cuda_error.store(10000 + (int32_t)r);
           ok = false;
         } else {
-          lg.tail = seq;
+          lg.tail[0] = seq;
         }
       }
     } else {
@@ -1219,7 +1286,10 @@ class Runtime : public strings::Hooks {
       // publish + item read of the SM path (4 KB job: 11.7 vs 16.6 us)
       bool busy = mono_ns() - ph->last_big_copy_ns < 2000000ull;
       for (const auto& lg : logical)
-        if (lg.phys == ph && lg.ctr && (int32_t)(lg.issued[engine] - lg.ctr->done[engine]) > 0) busy = true;
+        if (lg.phys == ph && lg.ctr &&
+            ((int32_t)(lg.issued[engine] - lg.ctr->done[engine]) > 0 ||
+             (engine == strings::ENG_D2H && (int32_t)(lg.issued[kEagerD2H] - lg.ctr->done[kEagerD2H]) > 0)))
+          busy = true;
       if (!busy) return false;
     }
     uint64_t total = 0;
@@ -1283,11 +1353,75 @@ class Runtime : public strings::Hooks {
     return true;
   }
 
-  // Append "done[engine] = seq" to the copy stream (ordered after the copies).
-  bool signal_copy(Logical& lg, JobCtx* jc, int engine, cudaStream_t s) {
-    const uint32_t seq = ++lg.issued[engine];
+  // The whole H2D -> KL -> D2H chain of an eager job, queued now (see eager_ok).
+  bool issue_eager(strings::Job& j, JobCtx* jc, Logical& lg) {
+    Phys* ph = lg.phys;
+    if (jc->slot < 0) {
+      jc->slot = lg.free_slots.back();
+      lg.free_slots.pop_back();
+      uint8_t* base = lg.arena + (size_t)jc->slot * cfg.slot_bytes;
+      uint64_t off = 0;
+      for (size_t i = 0; i < jc->in.size(); ++i) {
+        jc->dev_in[i] = reinterpret_cast<uint64_t>(base + off);
+        off = align_up(off + jc->in[i].bytes);
+      }
+      jc->dev_out = reinterpret_cast<uint64_t>(base + off);
+    }
+    KlItem& it = lg.item_host[jc->slot];
+    jc->item_ok = build_item(j, jc, it);
+    if (!jc->item_ok) return false;
+    // H2D stream: the work item, the inputs, the H2D counter, then ring 1's entry
+    const size_t ibytes = it.kclass == STRINGS_GEMM ? sizeof(KlItem) : offsetof(KlItem, tmap_a);
+    bool ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(lg.item_dev + sizeof(KlItem) * jc->slot), &it, ibytes,
+                                      cudaMemcpyHostToDevice, lg.h2d));
+    for (size_t i = 0; i < jc->in.size() && ok; ++i)
+      if (jc->in[i].bytes)
+        ok = cuda_ok(cudaMemcpyAsync(reinterpret_cast<void*>(jc->dev_in[i]), jc->in[i].dma, jc->in[i].bytes,
+                                     cudaMemcpyHostToDevice, lg.h2d));
+    ok = ok && signal_copy(lg, jc, strings::ENG_H2D, lg.h2d);
+    if (!ok) return false;
+    const uint32_t idx = lg.tail[1] % kRing;
+    const uint32_t seq = lg.tail[1] + 1;
+    CUresult r = g_write_value64(reinterpret_cast<CUstream>(lg.h2d), lg.ring_dev + sizeof(uint64_t) * (kRing + idx),
+                                 ((uint64_t)seq << 32) | ((uint32_t)jc->desc.kclass << 16) | (uint32_t)jc->slot, 0);
+    if (r != CUDA_SUCCESS) {
+      g_last_cuda_error.store(10000 + (int32_t)r);
+      return false;
+    }
+    lg.tail[1] = seq;
+    jc->kl_seq = seq;
+    jc->kl_idx = kRing + (int)idx;
+    jc->kl_issue = real_ns();
+    jc->eager = true;
+    jc->issued[strings::ENG_KL] = true;
+    // D2H: the eager stream waits for the KL's device done word, then copies out
+    r = g_wait_value32(reinterpret_cast<CUstream>(lg.d2h_eager), lg.done_dev + sizeof(uint32_t) * (kRing + idx), seq,
+                       CU_STREAM_WAIT_VALUE_EQ);
+    if (r != CUDA_SUCCESS) {
+      g_last_cuda_error.store(10000 + (int32_t)r);
+      return false;
+    }
+    uint64_t off = 0;
+    for (size_t i = 0; i < jc->out.size() && ok; ++i) {
+      if (jc->out[i].bytes)
+        ok = cuda_ok(cudaMemcpyAsync(jc->out[i].dma, reinterpret_cast<void*>(jc->dev_out + off), jc->out[i].bytes,
+                                     cudaMemcpyDeviceToHost, lg.d2h_eager));
+      off = align_up(off + jc->out[i].bytes);
+    }
+    ok = ok && signal_copy(lg, jc, strings::ENG_D2H, lg.d2h_eager, kEagerD2H);
+    jc->issued[strings::ENG_D2H] = true;
+    ph->last_big_copy_ns = mono_ns();
+    eager_jobs += 1;
+    return ok;
+  }
+
+  // Append "done[counter] = seq" to the copy stream (ordered after the copies);
+  // counter = the engine, or kEagerD2H for the eager D2H stream.
+  bool signal_copy(Logical& lg, JobCtx* jc, int engine, cudaStream_t s, int counter = -1) {
+    if (counter < 0) counter = engine;
+    const uint32_t seq = ++lg.issued[counter];
     jc->copy_seq[engine] = seq;
-    CUresult r = g_write_value32(reinterpret_cast<CUstream>(s), lg.ctr_dev + engine * sizeof(uint32_t), seq, 0);
+    CUresult r = g_write_value32(reinterpret_cast<CUstream>(s), lg.ctr_dev + counter * sizeof(uint32_t), seq, 0);
     if (r != CUDA_SUCCESS) {
       g_last_cuda_error.store(10000 + (int32_t)r);
       return false;
@@ -1328,7 +1462,7 @@ class Runtime : public strings::Hooks {
       jc->kl_observe = real_ns();
       // MEASURED timing: the SFT learns the KL's device time (R-14 telemetry)
       if (!virtual_clock() && jc->kl_t1 > jc->kl_t0) jc->job.measured[strings::ENG_KL] = jc->kl_t1 - jc->kl_t0;
-      lg.completed += 1;
+      lg.completed[jc->kl_idx / kRing] += 1;
       jc->phys_done[engine] = true;
       return true;
     }
@@ -1338,7 +1472,7 @@ class Runtime : public strings::Hooks {
       return true;
     }
     if (engine != strings::ENG_KL) {
-      const uint32_t d = lg.ctr->done[engine];
+      const uint32_t d = lg.ctr->done[engine == strings::ENG_D2H && jc->eager ? kEagerD2H : engine];
       if ((int32_t)(d - jc->copy_seq[engine]) < 0) return false;
       // an H2D whose KL work item went through the copy partition is complete
       // only once the item landed too (so the KL issue never waits for it)
@@ -1535,9 +1669,57 @@ class Runtime : public strings::Hooks {
       fprintf(stderr, "[strings]  gpu %d: copy ring tail %u completed %u, copy ctas %d\n", ph->dev, ph->ctail,
               ph->ccompleted, ph->copy_ctas);
     for (auto& lg : logical)
-      fprintf(stderr, "[strings]  ld %d: KL tail %u completed %u, copies issued h2d %u d2h %u, done h2d %u d2h %u\n",
-              lg.gid, lg.tail, lg.completed, lg.issued[0], lg.issued[2], lg.ctr ? lg.ctr->done[0] : 0,
-              lg.ctr ? lg.ctr->done[2] : 0);
+      fprintf(stderr,
+              "[strings]  ld %d: KL tail %u/%u completed %u/%u, copies issued h2d %u d2h %u eager %u, done h2d %u "
+              "d2h %u eager %u\n",
+              lg.gid, lg.tail[0], lg.tail[1], lg.completed[0], lg.completed[1], lg.issued[0], lg.issued[2],
+              lg.issued[kEagerD2H], lg.ctr ? lg.ctr->done[0] : 0, lg.ctr ? lg.ctr->done[2] : 0,
+              lg.ctr ? lg.ctr->done[kEagerD2H] : 0);
+    // device side: claim counters, partition mailboxes and the ring entries at the heads
+    for (auto& ph : phys) {
+      if (!ph->L || !ph->dev_state) continue;
+      set_dev(ph->dev);
+      cudaStream_t st;
+      if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) continue;
+      const int nh = ph->L * kRings + 1, np = ph->L * cfg.partitions + (ph->copy_ctas ? 1 : 0);
+      std::vector<uint32_t> heads(nh);
+      std::vector<strings_dev::PartState> parts(np);
+      cudaMemcpyAsync(heads.data(), ph->dp.heads, sizeof(uint32_t) * nh, cudaMemcpyDeviceToHost, st);
+      cudaMemcpyAsync(parts.data(), ph->dp.parts, sizeof(strings_dev::PartState) * np, cudaMemcpyDeviceToHost, st);
+      std::vector<uint64_t> ring((size_t)ph->L * kRings * kRing);
+      cudaMemcpyAsync(ring.data(), ph->ring_dev, sizeof(uint64_t) * ring.size(), cudaMemcpyDeviceToHost, st);
+      std::vector<KlItem> items((size_t)ph->L * cfg.admit_cap);
+      cudaMemcpyAsync(items.data(), ph->items_dev, sizeof(KlItem) * items.size(), cudaMemcpyDeviceToHost, st);
+      std::vector<uint32_t> prog(ph->sms);
+      cudaMemcpyAsync(prog.data(), ph->progress, sizeof(uint32_t) * prog.size(), cudaMemcpyDeviceToHost, st);
+      cudaStreamSynchronize(st);
+      cudaStreamDestroy(st);
+      for (int h = 0; h < nh; ++h) {
+        const uint64_t e = h < ph->L * kRings ? ring[(size_t)h * kRing + heads[h] % kRing] : 0;
+        fprintf(stderr, "[strings]  gpu %d head %d = %u, entry there seq %u word %08x\n", ph->dev, h, heads[h],
+                (uint32_t)(e >> 32), (uint32_t)e);
+      }
+      for (size_t k = 0; k < items.size(); ++k)
+        if (items[k].n || items[k].in0)
+          fprintf(stderr, "[strings]  gpu %d item[%zu] job %llu kclass %u n %llu in0 %llx out0 %llx\n", ph->dev, k,
+                  (unsigned long long)items[k].job, items[k].kclass, (unsigned long long)items[k].n,
+                  (unsigned long long)items[k].in0, (unsigned long long)items[k].out0);
+      for (int q = 0; q < np; ++q) {
+        std::string pr;
+        for (int b = ph->part_start[q]; b < ph->part_start[q + 1]; ++b) {
+          char tmp[24];
+          snprintf(tmp, sizeof tmp, " %x", prog[b]);
+          pr += tmp;
+        }
+        fprintf(stderr, "[strings]  gpu %d part %d CTA progress (gen << 12 | class << 8 | step: 1 item read, 2 body done, 3 counted):%s\n",
+                ph->dev, q, pr.c_str());
+      }
+      for (int q = 0; q < np; ++q)
+        fprintf(stderr, "[strings]  gpu %d part %d gen %llx done_gen %u done_cnt %u lock %x total %u help %llx seq %u "
+                        "ring_idx %u\n",
+                ph->dev, q, (unsigned long long)parts[q].gen, parts[q].done_gen, parts[q].done_cnt, parts[q].lock,
+                parts[q].total, (unsigned long long)parts[q].help, parts[q].seq, parts[q].ring_idx);
+    }
     for (auto& f : ops) {
       JobCtx* jc = f.first;
       const int e = f.second;
@@ -1753,6 +1935,7 @@ strings_status_t strings_register_tenant(uint32_t weight, uint32_t max_inflight,
   t.weight = weight;
   t.c = max_inflight;
   g_rt->tenants.push_back(t);
+  g_rt->inflight_cap_sum += max_inflight;
   int id = g_rt->core->add_tenant(weight, max_inflight);
   *out = (strings_tenant_t)id;
   return STRINGS_OK;
@@ -1870,6 +2053,7 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   for (size_t i = 0; i < r.phys.size() && i < 8; ++i) st->gpu_clock_offset_ns[i] = r.phys[i]->clock_offset_ns;
   st->sm_copy_ops = r.sm_copies;
   st->kl_mode = r.kl_mode;
+  st->eager_jobs = r.eager_jobs;
   for (int g2 = 0; g2 < std::min(8, r.cfg.num_gpus); ++g2)
     for (int x = 0; x < 3; ++x) st->engine_busy_ns[g2][x] = r.core->busy_ns(g2, x);
   st->num_gpus = r.cfg.num_gpus;

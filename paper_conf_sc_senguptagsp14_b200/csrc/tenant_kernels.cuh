@@ -44,9 +44,16 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+// Every mbarrier is initialised ONCE per kernel (mbar_setup at the kernel's
+// start); items that re-use one track its phase parity across items (the stage
+// and fill parities in GemmSmem::sphase, the MMA barrier's in mma_phase).
+// Re-initialising a barrier per item, as round 1 did, was not reliable on
+// sm_100a: the persistent dispatcher's second streaming item on a CTA could
+// wait forever on its first stage (the new phase accounted an arrival twice).
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
 }
+constexpr int kTailBarriers = 14;    // stream/SCAN pipeline stages [0, kStreamStages), GEMM fill [kFillBar0, +4)
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t a = smem_u32(bar);
   asm volatile(
@@ -166,6 +173,8 @@ constexpr int kStreamLead = STRINGS_STREAM_LEAD;
 constexpr int kStreamMinChunks = STRINGS_STREAM_MIN_CHUNKS;
 constexpr int kStreamStoreSlack = kStreamStages - kStreamLead - 1;
 static_assert(kStreamStages >= 3 && kStreamStages <= 12, "stream stages");
+constexpr int kFillBar0 = kStreamStages;   // first GEMM fill barrier in the smem tail (after the stages)
+static_assert(kFillBar0 + 4 <= kTailBarriers, "tail barriers: stages + 4 GEMM fill barriers");
 static_assert(kStreamLead >= 1 && kStreamLead < kStreamStages, "stream lead");
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
@@ -203,11 +212,20 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
 // partial chunk) use the LDG path with a static split over ranks < S (a lent
 // CTA has rank >= S and skips it).
 constexpr uint32_t kNoChunk = 0xFFFFFFFFu;
+// Stage phase parities after `used` more pipeline positions (position i uses
+// stage i mod kStreamStages once).
+__device__ __forceinline__ uint32_t stage_phases_after(uint32_t bits, uint64_t used) {
+  for (int st = 0; st < kStreamStages; ++st) {
+    const uint64_t uses = used > (uint64_t)st ? (used - 1 - st) / kStreamStages + 1 : 0;
+    bits ^= (uint32_t)(uses & 1) << st;
+  }
+  return bits;
+}
 
 template <int KCLASS>
 __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
                             float alpha, uint32_t seed, int rank, int S, uint8_t* stage, uint64_t* sbar,
-                            uint32_t* cid, GroupSync* gs, const uint32_t* total_word) {
+                            uint32_t* cid, uint32_t* sphase, GroupSync* gs, const uint32_t* total_word) {
   const bool aligned = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   const uint64_t bytes = n * 4;
   // items too small to fill the pipeline (fewer than kStreamMinChunks chunks per CTA)
@@ -246,16 +264,18 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       bulk_g2s(stage + st * kStreamChunk, xb + (uint64_t)c * kStreamChunk, kStreamChunk, &sbar[st]);
       next = claim();                             // consumed at the next issue
     };
+    // the stage barriers live for the whole kernel (mbar_setup); their phase
+    // parities carry over from item to item in *sphase (bit st = stage st)
+    const uint32_t ph0 = *reinterpret_cast<volatile uint32_t*>(sphase);
     if (threadIdx.x == 0) {
-      for (int st = 0; st < kStreamStages; ++st) mbar_init(&sbar[st], 1);
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
       next = claim();
       for (int st = 0; st < kStreamLead && claiming; ++st) issue(st);
     }
     __syncthreads();
-    for (uint64_t i = 0;; ++i) {
+    uint64_t i = 0;
+    for (;; ++i) {
       const int st = (int)(i % kStreamStages);
-      const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
+      const uint32_t ph = ((ph0 >> st) & 1u) ^ (uint32_t)((i / kStreamStages) & 1);
       if (threadIdx.x == 0 && claiming) {
         const int s2 = (int)((i + kStreamLead) % kStreamStages);
         // stage s2 was last stored at iteration i + kStreamLead - kStreamStages: that
@@ -282,6 +302,7 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       if (threadIdx.x == 0) bulk_s2g(yb + (uint64_t)c * kStreamChunk, stage + st * kStreamChunk, kStreamChunk);
     }
     if (threadIdx.x == 0) {
+      *sphase = stage_phases_after(ph0, i + 1);   // positions 0..i (the end marker's included) used a phase
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");                   // writes done
       asm volatile("fence.proxy.async.global;" ::: "memory");                     // async -> generic
       // every claim of this CTA has returned (the last one came back empty and was
@@ -412,6 +433,7 @@ struct GemmSmem {
   uint8_t* stage;      // streaming stages (aliases a/b: a CTA runs one item at a time)
   uint64_t* sbar;      // streaming stage mbarriers / GEMM fill mbarriers [4]
   uint32_t* scratch;   // 32 words outside the stages (SCAN warp totals)
+  uint32_t* sphase;    // phase parities of the pipeline stage barriers (bit per stage), kept across items
 };
 
 // Units u = tile * R + rep, tile = (mt, nt); this CTA takes the contiguous
@@ -434,26 +456,27 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, const v
     asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_b) : "memory");
     asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" :: "l"(tmap_c) : "memory");
   }
+  // fill barrier c's phase parity: bit 8 + c of *sm.sphase (only thread 0 uses them)
+  uint32_t fph = threadIdx.x == 0 ? (*sm.sphase >> 8) & 0xFu : 0u;
   uint64_t u = u0;
   while (u < u1) {
     const uint64_t tile = u / R;
     const uint64_t last = min(u1, (tile + 1) * R);        // exclusive end of this tile's run
     const uint64_t mt = tile / tiles_n, nt = tile % tiles_n;
     if (threadIdx.x == 0) {
-      for (int c = 0; c < kchunks; ++c) mbar_init(&sm.sbar[c], 1);
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
       for (int c = 0; c < kchunks; ++c) {
         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
-                     :: "r"(smem_u32(&sm.sbar[c])), "r"(kSlabA + 4 * kChunkB) : "memory");
-        tma_load_2d(sm.a + c * kSlabA, tmap_a, 64 * c, (int)(mt * kTileM), &sm.sbar[c]);
+                     :: "r"(smem_u32(&sm.sbar[kFillBar0 + c])), "r"(kSlabA + 4 * kChunkB) : "memory");
+        tma_load_2d(sm.a + c * kSlabA, tmap_a, 64 * c, (int)(mt * kTileM), &sm.sbar[kFillBar0 + c]);
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          tma_load_2d(sm.b + j * kSlabB + c * kChunkB, tmap_b, (int)(nt * kTileN) + 64 * j, 64 * c, &sm.sbar[c]);
+          tma_load_2d(sm.b + j * kSlabB + c * kChunkB, tmap_b, (int)(nt * kTileN) + 64 * j, 64 * c,
+                      &sm.sbar[kFillBar0 + c]);
       }
       for (uint64_t v = u; v < last; ++v) {
         for (int c = 0; c < kchunks; ++c) {
           if (v == u) {
-            mbar_wait(&sm.sbar[c], 0);
+            mbar_wait(&sm.sbar[kFillBar0 + c], (fph >> c) & 1u);
             tc_fence_after();
           }
 #pragma unroll
@@ -466,6 +489,7 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, const v
         }
       }
       umma_commit(sm.bar);            // arrives when every MMA above has completed
+      fph ^= (1u << kchunks) - 1u;    // each fill barrier completed one phase in this run
     }
     __syncwarp();
     mbar_wait(sm.bar, mma_phase);
@@ -506,6 +530,8 @@ __device__ inline void gemm_body(const void* tmap_a, const void* tmap_b, const v
     __syncthreads();                  // smem and TMEM free for the next run
     u = last;
   }
+  if (threadIdx.x == 0 && u0 < u1) *sm.sphase = (*sm.sphase & ~0xF00u) | (fph << 8);
+  __syncthreads();
 }
 
 // ------------------------------------------------------- group coordination
@@ -613,7 +639,8 @@ __device__ __forceinline__ uint32_t scan_chunk_smem(uint32_t* c, uint32_t carry,
 }
 
 __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
-                                 int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* wsum) {
+                                 int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* wsum,
+                                 uint32_t* sphase) {
   // wsum: 16 words outside the stages ([8] warp totals + [8] broadcast / second buffer)
   constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;
   const uint64_t chunk = ((n + S - 1) / S + kTile - 1) / kTile * kTile;
@@ -667,11 +694,7 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
   if (nch) {
     const uint8_t* xb = reinterpret_cast<const uint8_t*>(x + b0);
     uint8_t* yb = reinterpret_cast<uint8_t*>(y + b0);
-    if (threadIdx.x == 0) {
-      for (int q = 0; q < kStreamStages; ++q) mbar_init(&sbar[q], 1);
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
+    const uint32_t ph0 = *reinterpret_cast<volatile uint32_t*>(sphase);   // (stream_body's stage barriers)
     if (threadIdx.x == 0)
       for (int q = 0; q < kStreamLead && (uint64_t)q < nch; ++q) {
         mbar_expect_tx(&sbar[q], kStreamChunk);
@@ -679,7 +702,7 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
       }
     for (uint64_t i = 0; i < nch; ++i) {
       const int q = (int)(i % kStreamStages);
-      const uint32_t ph = (uint32_t)((i / kStreamStages) & 1);
+      const uint32_t ph = ((ph0 >> q) & 1u) ^ (uint32_t)((i / kStreamStages) & 1);
       if (threadIdx.x == 0 && i + kStreamLead < nch) {
         const int q2 = (int)((i + kStreamLead) % kStreamStages);
         if (i + kStreamLead >= (uint64_t)kStreamStages)
@@ -695,6 +718,7 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
       if (threadIdx.x == 0) bulk_s2g(yb + i * kStreamChunk, stage + q * kStreamChunk, kStreamChunk);
     }
     if (threadIdx.x == 0) {
+      *sphase = stage_phases_after(ph0, nch);
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
       asm volatile("fence.proxy.async.global;" ::: "memory");
     }
@@ -877,7 +901,7 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
       break;
     case 4:
       scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
-                gs, sm.stage, sm.sbar, sm.scratch);
+                gs, sm.stage, sm.sbar, sm.scratch, sm.sphase);
       break;
     case 5:
       sort_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,
@@ -885,11 +909,11 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
       break;
     case 0:
       stream_body<0>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, total_word);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, sm.sphase, gs, total_word);
       break;
     case 2:
       stream_body<2>(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0),
-                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, gs, total_word);
+                     it.n, it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, sm.sphase, gs, total_word);
       break;
     case 1:
       gemm_body(tmaps->tmap_a, tmaps->tmap_b, tmaps->tmap_c, tmap_global, reinterpret_cast<float*>(it.out0), it.m,
@@ -910,16 +934,24 @@ __device__ __forceinline__ GemmSmem carve_smem(uint8_t* base) {
   s.stage = base;
   s.sbar = reinterpret_cast<uint64_t*>(tail + 16);
   s.scratch = reinterpret_cast<uint32_t*>(tail + 128);
+  s.sphase = reinterpret_cast<uint32_t*>(tail + 12);
   return s;
 }
 
 // CTA prologue / epilogue shared by every kernel that may run a GEMM item.
-__device__ __forceinline__ uint32_t cta_setup(const GemmSmem& sm) {
-  if (threadIdx.x / 32 == 0) tmem_alloc(sm.tmem_slot, kTmemCols);
+// Every barrier of the smem tail, once per kernel (items track their phases).
+__device__ __forceinline__ void mbar_setup(const GemmSmem& sm) {
   if (threadIdx.x == 32) {
     mbar_init(sm.bar, 1);
+    for (int b = 0; b < kTailBarriers; ++b) mbar_init(&sm.sbar[b], 1);
+    *sm.sphase = 0;
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  __syncthreads();
+}
+__device__ __forceinline__ uint32_t cta_setup(const GemmSmem& sm) {
+  if (threadIdx.x / 32 == 0) tmem_alloc(sm.tmem_slot, kTmemCols);
+  mbar_setup(sm);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();

@@ -69,7 +69,8 @@ class Stats(C.Structure):
                 ("engine_busy_ns", (C.c_uint64 * 3) * 8), ("num_gpus", C.c_int32),
                 ("physical_gpus", C.c_int32), ("partitions", C.c_int32), ("sms_per_partition", C.c_int32),
                 ("issue_ns", C.c_uint64), ("gpu_clock_offset_ns", C.c_int64 * 8),
-                ("sm_copy_ops", C.c_uint64), ("kl_mode", C.c_int32), ("reserved_i32", C.c_int32)]
+                ("sm_copy_ops", C.c_uint64), ("kl_mode", C.c_int32), ("reserved_i32", C.c_int32),
+                ("eager_jobs", C.c_uint64)]
 
 
 def _load() -> C.CDLL:

@@ -17,6 +17,12 @@ for task in "$@"; do
     ncu_item) timeout 900 ncu --set full --clock-control none --import-source on -k regex:oneshot -c 4 -f -o gpurun_out/prof_xfer_item python tools/kernel_probe.py xfer_item > gpurun_out/ncu_item.log 2>&1; echo "ncu_item rc=$?"; tail -3 gpurun_out/ncu_item.log ;;
     ncu_launches) timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv --log-file gpurun_out/launches_bench.csv python bench.py --steps 2 --warmup 1 --no-static --no-e2e --no-kernels > gpurun_out/ncu_launches.log 2>&1; echo "ncu_launches rc=$?"; tail -c 600 gpurun_out/ncu_launches.log ;;
     openloop) timeout 1800 python bench.py --open-loop --open-loop-config ${OLCFG:-C4} > gpurun_out/openloop_${OLCFG:-C4}.log 2>&1; echo "openloop rc=$?"; tail -c 1500 gpurun_out/openloop_${OLCFG:-C4}.log ;;
+    configs_ab) for e in 1 0 1 0; do STRINGS_EAGER=$e BENCH_CONFIGS=${CONFIGS:-C1,C3} timeout 1200 python bench.py --configs --config-repeats ${REPEATS:-3} > gpurun_out/configs_eager$e.log 2>&1; echo "eager=$e rc=$?"; python -c "
+import json,sys
+for l in open('gpurun_out/configs_eager$e.log'):
+    if l.startswith('{'):
+        d=json.loads(l); print(d['config'], d['jobs_per_s'], d['span_ms'], d['roofline_frac'], d.get('frac_vs_copy_replay'), d['span_ms_min_max'])
+"; done ;;
     *) echo "unknown task $task" ;;
   esac
 done
