@@ -903,12 +903,13 @@ def _kernel_roofline(kl_lat, wl, peaks, krl=None) -> dict:
 
 
 # ncu --set full of the C2 work item's body as a stand-alone launch (XFER 2^24 u32
-# on 74 CTAs, `tools/kernel_probe.py xfer_item`): dram__bytes_read.sum +
-# dram__bytes_write.sum per launch; see profiles/r01_kernels.md.
-# Reads 67.18 MB = the 64 MiB input exactly; writes 21.33 MB of 67.1 MB: at this size
-# most of the output is still in the 126 MB L2 when the launch ends (no re-reads).
-_XFER_ITEM_NCU = {"dram_bytes": 67181056 + 21326336,
-                  "source": "profiles/r01_kernels.md (xfer_item: ncu --set full, XFER 2^24 on 74 CTAs)"}
+# on 144 CTAs -- one KL partition plus its lent sibling -- `tools/kernel_probe.py
+# xfer_item`): dram__bytes_read.sum + dram__bytes_write.sum per launch, mean of two
+# launches; profiles/r02_kernels.md.  Reads 67.14 MB = the 64 MiB input exactly;
+# writes 17.3 MB of 67.1 MB: most of the output is still in the 126 MB L2 when the
+# launch ends (no re-reads).
+_XFER_ITEM_NCU = {"dram_bytes": 67136768 + 17278080,
+                  "source": "profiles/r02_kernels.md (xfer_item: ncu --set full, XFER 2^24 on 144 CTAs)"}
 
 
 def max_over(gloo, x: float) -> float:
