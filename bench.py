@@ -923,85 +923,78 @@ def gloo_barrier(gloo):
 
 
 # --------------------------------------------------------------- baselines
-def cpu_baseline(wl, sample_jobs: int = 16) -> dict:
-    """The oracle (as it stands) on a bounded sample of the workload on the host:
-    per job a host copy in, the oracle kernel, a host copy out; BLAS limited to
-    one thread.  Plus the oracle DES on the whole workload."""
+def _oracle_inputs(specs):
     import numpy as np
-    from threadpoolctl import threadpool_limits
 
     import strings_workload as W
-    from oracle import kernels as K
+    ins = [W.job_inputs(s) for s in specs]
+    outs = [[np.empty(sh, dt) for sh, dt in W.job_output_shapes(s)] for s in specs]
+    return ins, outs
+
+
+def cpu_baseline(wl, threads: int = 0) -> dict:
+    """SURVEY §8(d)'s CPU reference: the oracle's plain C kernels (oracle/c,
+    -O3, no BLAS), the WHOLE workload -- every job's H2D bytes copied in, the
+    kernel (GEMM repeated R times), the D2H bytes copied out -- on a pthread pool
+    of `threads` workers (default: every host core), tenants dealt round-robin
+    to workers and each tenant's jobs run in submission order (c_t = 1).
+    Inputs are generated before timing.  Also the DES speed: the oracle's
+    discrete-event model of the scheduler (plain Python) over the workload."""
+    from oracle import cbind
     from oracle.des import run_oracle
 
-    sample = wl.jobs[:sample_jobs]
-    data = [W.job_inputs(s) for s in sample]
-    with threadpool_limits(limits=1):
-        t = time.perf_counter()
-        for s, ins in zip(sample, data):
-            staged = [np.copy(a) for a in ins]
-            outs = K.run_job(s, staged)
-            _ = [np.copy(o) for o in outs]
-        dt = time.perf_counter() - t
-        t2 = time.perf_counter()
-        run_oracle(wl)
-        des = time.perf_counter() - t2
-    return {"value": round(len(sample) / dt, 3), "unit": "jobs/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {len(sample)} jobs of C2 (one per tenant): copy-in, oracle kernel, copy-out",
-            "des_s_full_workload": round(des, 3)}
-
-
-def _oracle_shard(specs):
-    """One worker: generate its jobs' inputs (untimed), then time the oracle on them."""
-    import numpy as np
-    import strings_workload as W
-    from oracle import kernels as K
-    data = [W.job_inputs(s) for s in specs]
+    threads = threads or (os.cpu_count() or 1)
+    ins, outs = _oracle_inputs(wl.jobs)
+    cbind.lib()
     t = time.perf_counter()
-    for spec, ins in zip(specs, data):
-        outs = K.run_job(spec, [np.copy(a) for a in ins])
-        _ = [np.copy(o) for o in outs]
-    return time.perf_counter() - t
-
-
-def cpu_baseline_all_cores(wl, sample_jobs: int = 64) -> dict:
-    """The same oracle sample spread over every host core (one process per core,
-    BLAS single-threaded inside each): jobs / slowest worker's compute time."""
-    import multiprocessing as mp
-    cores = os.cpu_count() or 1
-    sample = wl.jobs[:sample_jobs]
-    shards = [sample[i::cores] for i in range(cores)]
-    shards = [s for s in shards if s]
-    os.environ.setdefault("OMP_NUM_THREADS", "1")
-    os.environ.setdefault("OPENBLAS_NUM_THREADS", "1")
-    with mp.get_context("fork").Pool(len(shards)) as pool:
-        times = pool.map(_oracle_shard, shards)
-    return {"value": round(len(sample) / max(times), 3), "unit": "jobs/s", "cores": len(shards), "kind": "oracle",
-            "sample": f"first {len(sample)} jobs of C2 split over {len(shards)} processes "
-                      "(inputs generated before timing; value = jobs / slowest worker)"}
+    cbind.run_jobs(wl.jobs, ins, outs, threads)
+    dt = time.perf_counter() - t
+    t2 = time.perf_counter()
+    o = run_oracle(wl)
+    des = time.perf_counter() - t2
+    decisions = sum(1 for ln in o.trace if " PLACE " in ln or " WAKE " in ln)
+    busy = min(threads, len({s.tenant for s in wl.jobs}))
+    return {"value": round(len(wl.jobs) / dt, 3), "unit": "jobs/s", "cores": busy, "kind": "oracle",
+            "sample": f"the whole workload ({len(wl.jobs)} jobs, GEMM R = {max(s.reps for s in wl.jobs)} computed "
+                      f"every repetition) through the oracle's plain C kernels (oracle/c/kernels.c, gcc -O3, no "
+                      f"BLAS) with host copies in and out, {threads} worker threads ({busy} busy: tenants are "
+                      f"dealt to workers, c_t = 1)",
+            "seconds": round(dt, 3),
+            "des": {"seconds": round(des, 3), "decisions": decisions,
+                    "decisions_per_s": round(decisions / des, 1) if des > 0 else None,
+                    "note": "oracle/des.py (plain Python) on the same workload"}}
 
 
 def run_reference(args):
-    """--impl reference: the oracle as it stands on the host cores, same config/metric."""
+    """--impl reference: the oracle as it stands on the host cores, same
+    config/metric.  Each step is a bounded sample of C2: one job per tenant (16
+    jobs, GEMM R = 64 computed every repetition) through the oracle's plain C
+    kernels on a pool of every host core, host copies in and out."""
     import strings_workload as W
+    from oracle import cbind
+
     wl = W.config_c2(jobs_per_tenant=args.jobs_per_tenant)
+    sample = [s for s in wl.jobs if s.arrival_ns == 0][:len(wl.tenants)]
+    ins, outs = _oracle_inputs(sample)
+    threads = os.cpu_count() or 1
+    cbind.lib()
     for _ in range(args.warmup):
-        cpu_baseline(wl, sample_jobs=4)
-    vals = []
+        cbind.run_jobs(sample[:2], ins[:2], outs[:2], threads)
     t = time.perf_counter()
     for _ in range(args.steps):
-        vals.append(cpu_baseline(wl, sample_jobs=16)["value"])
+        cbind.run_jobs(sample, ins, outs, threads)
     dt = time.perf_counter() - t
-    v = statistics.median(vals)
+    v = round(len(sample) * args.steps / dt, 3)
+    busy = min(threads, len(sample))
     line = {"metric": METRIC, "value": v, "unit": "jobs/s", "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64/f32/u32 (numpy)", "data": "synthetic",
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64/f32/u32 (plain C)", "data": "synthetic",
             "impl": "reference",
             "config": arm_config(wl.config.resolved(), len(wl.jobs), args.gpus, args.kl_mode),
-            "reference_note": "the oracle (oracle/, plain numpy, one host core) runs the same C2 jobs: copy-in, "
-                              "CPU kernel, copy-out; each step times a 16-job sample (one job per tenant)",
-            "cpu_baseline": {"value": v, "unit": "jobs/s", "cores": 1, "kind": "oracle",
-                             "sample": "16 jobs of C2 per step (one per tenant)"},
+            "reference_note": "the oracle (oracle/c/kernels.c, plain C, -O3, no BLAS) runs the C2 jobs on the host: "
+                              "copy-in, CPU kernel (GEMM R = 64 times), copy-out; each step is one job per tenant",
+            "cpu_baseline": {"value": v, "unit": "jobs/s", "cores": busy, "kind": "oracle",
+                             "sample": f"16 jobs of C2 per step (one per tenant) on {threads} threads"},
             "e2e": {"value": v, "unit": "jobs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -1443,10 +1436,6 @@ def main():
         res.pop("_mean_latency_s_by_tenant", None)
         if world == 1:
             res["cpu_baseline"] = cpu_baseline(wl)
-            try:
-                res["cpu_baseline_all_cores"] = cpu_baseline_all_cores(wl)
-            except Exception as e:  # pragma: no cover - informational only
-                res["cpu_baseline_all_cores"] = {"error": repr(e)}
         print(json.dumps(res), flush=True)
     if world > 1:
         import torch.distributed as dist
