@@ -24,6 +24,8 @@ for l in open('gpurun_out/configs_eager$e.log'):
         d=json.loads(l); print(d['config'], d['jobs_per_s'], d['span_ms'], d['roofline_frac'], d.get('frac_vs_copy_replay'), d['span_ms_min_max'])
 "; done ;;
     ncu_kernels) for k in vscale xfer gemm scan hist sort; do timeout 900 ncu --set full --clock-control none --import-source on -k regex:oneshot -c 2 -f -o gpurun_out/prof_$k python tools/kernel_probe.py $k > gpurun_out/ncu_$k.log 2>&1; echo "ncu $k rc=$?"; done ;;
+    benchdef) timeout 1200 python bench.py > gpurun_out/benchdef.log 2>&1; echo "benchdef rc=$?"; tail -c 400 gpurun_out/benchdef.log ;;
+    ref) timeout 900 python bench.py --impl reference --steps ${STEPS:-20} --warmup ${WARMUP:-5} > gpurun_out/ref.log 2>&1; echo "ref rc=$?"; tail -c 800 gpurun_out/ref.log ;;
     *) echo "unknown task $task" ;;
   esac
 done
