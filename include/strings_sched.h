@@ -192,7 +192,11 @@ typedef struct {
     int32_t  num_gpus, physical_gpus, partitions, sms_per_partition;
     uint64_t issue_ns;                            /* part of decision_ns spent issuing woken ops
                                                      (cudaMemcpyAsync, stream writes, KL ring
-                                                     publish); decision_ns - issue_ns = decisions */
+                                                     publish); decision_ns - issue_ns = decisions.
+                                                     With one issuer thread per GPU
+                                                     (STRINGS_ISSUE_THREADS, default when the
+                                                     process drives >= 4 GPUs) the issuing runs
+                                                     on those threads, off the engine thread */
     int64_t  gpu_clock_offset_ns[8];              /* per physical GPU (first 8): %globaltimer minus
                                                      CLOCK_REALTIME, calibrated at init (kl_gpu_*
                                                      stamps - offset = host clock); 0 if unknown */

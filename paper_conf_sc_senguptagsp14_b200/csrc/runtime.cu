@@ -175,8 +175,10 @@ struct JobCtx {
   int slot = -1;                       // resident slot on the logical device
   uint64_t dev_in[2] = {0, 0}, dev_out = 0;
   cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
-  bool issued[3] = {false, false, false};
-  bool phys_done[3] = {false, false, false};
+  // set by whichever thread issues the op (the engine thread, or the GPU's issuer
+  // thread: STRINGS_ISSUE_THREADS); phys_done before issued on a failed issue
+  std::atomic<bool> issued[3]{};
+  std::atomic<bool> phys_done[3]{};
   uint32_t kl_seq = 0;
   bool item_ok = false;                // KL work item built (and staged) at H2D issue
   uint32_t copy_seq[3] = {0, 0, 0};
@@ -211,7 +213,9 @@ struct Logical {
   KlDone* done = nullptr;              // host pointer, [kRings][kRing] entries
   CUdeviceptr done_dev = 0;            // [kRings][kRing] u32 device copies of the completion seq
   uint32_t tail[kRings] = {0, 0};      // items published per ring
-  uint32_t completed[kRings] = {0, 0}; // items whose completion was consumed, per ring
+  // items whose completion was consumed, per ring: written by the engine thread,
+  // read by the issuing thread (ring-room checks) -- accessed with __atomic builtins
+  uint32_t completed[kRings] = {0, 0};
   cudaStream_t d2h_eager = nullptr;    // eager D2H ops: wait for their KL on the device, then copy
   CopyCounters* ctr = nullptr;         // host view
   CUdeviceptr ctr_dev = 0;             // device view
@@ -254,7 +258,7 @@ struct Phys {
   // ops of different logical devices / directions are consumed out of ring order
   // (in INJECTED timing an op may be issued long before its virtual DONE), so an
   // index is reused only after its own op was observed, never by count alone
-  std::vector<uint8_t> cbusy = std::vector<uint8_t>(kRing, 0);
+  std::vector<std::atomic<uint8_t>> cbusy = std::vector<std::atomic<uint8_t>>(kRing);
   cudaStream_t cpstream = nullptr;     // stream memory ops publishing copy ring entries
   int64_t clock_offset_ns = 0;         // %globaltimer - CLOCK_REALTIME (ping-pong, min RTT)
   uint64_t clock_rtt_ns = 0;
@@ -263,6 +267,15 @@ struct Phys {
   void* probe_host = nullptr;          // clock-calibration buffer, freed at shutdown with everything else
   std::vector<int> part_start;         // [L*P + 1] partition table (host copy)
   std::vector<cudaEvent_t> ev_pool;
+  std::mutex ev_mu;                    // ev_pool: taken by the issuing thread, returned by the engine
+  // Issuer thread (STRINGS_ISSUE_THREADS): the engine thread hands this GPU's woken
+  // ops over in wake order; this thread makes the driver calls
+  std::mutex iq_mu;
+  std::condition_variable iq_cv;
+  std::deque<std::pair<JobCtx*, int>> iq;
+  std::atomic<uint32_t> iq_len{0};
+  bool iq_stop = false;
+  std::thread issuer;
 };
 
 // One part of a PMT staging copy.  Large parts use non-temporal stores
@@ -514,9 +527,10 @@ class Runtime : public strings::Hooks {
   uint64_t first_submit = 0, last_done = 0;
   uint64_t h2d_total = 0, d2h_total = 0, kbytes_total = 0, kflop_total = 0;
   uint64_t decision_ns = 0;            // time inside Core::step (decisions + op issue)
-  uint64_t sm_copies = 0;              // H2D/D2H ops served by the copy partition
-  uint64_t eager_jobs = 0;             // jobs whose KL and D2H were chained on the device (eager_ok)
-  uint64_t inflight_cap_sum = 0;       // sum of the registered tenants' in-flight limits c_t
+  std::atomic<uint64_t> sm_copies{0};  // H2D/D2H ops served by the copy partition
+  std::atomic<uint64_t> eager_jobs{0}; // jobs whose KL and D2H were chained on the device (eager_ok)
+  std::atomic<uint64_t> inflight_cap_sum{0};  // sum of the registered tenants' in-flight limits c_t
+  bool issue_threads = false;          // one issuer thread per GPU (init: STRINGS_ISSUE_THREADS)
   // STRINGS_EAGER=0 turns eager chaining off (every phase issued at its wake)
   const bool eager_enabled = [] {
     const char* e = getenv("STRINGS_EAGER");
@@ -543,7 +557,7 @@ class Runtime : public strings::Hooks {
     const char* e = getenv("STRINGS_ITEM_VIA_COPY");
     return e && e[0] == '1';
   }();
-  uint64_t issue_ns = 0;               // of which: issuing woken ops (on_wake)
+  std::atomic<uint64_t> issue_ns{0};   // issuing woken ops (driver calls), whichever thread does it
   // in-flight physical ops (measured mode): (job, engine)
   std::vector<std::pair<JobCtx*, int>> inflight;
   // virtual DONE events (injected / decisions-only)
@@ -634,6 +648,24 @@ class Runtime : public strings::Hooks {
         teardown_gpus();
         return s;
       }
+    }
+    // one issuer thread per GPU: default from 4 GPUs on.  The engine thread spends
+    // ~3-5 us per job deciding and ~6-8 us issuing (driver calls); alone it would
+    // saturate near 90k jobs/s, i.e. at 5-6 GPUs of small (C3-class) jobs.  The
+    // hand-over costs a chain of dependent phases some latency (one B200: C1 2.5 ->
+    // 3.0 ms, C2/C3 within noise), so fewer GPUs issue inline.
+    // STRINGS_ISSUE_THREADS=1 forces it on, =0 off.
+    if (has_gpu()) {
+      int used = 0;
+      for (auto& ph : phys) used += ph->L > 0;
+      const char* it = getenv("STRINGS_ISSUE_THREADS");
+      issue_threads = it ? it[0] == '1' : used >= 4;
+      if (issue_threads)
+        for (auto& ph : phys)
+          if (ph->L) {
+            Phys* p = ph.get();
+            p->issuer = std::thread([this, p] { issuer_main(p); });
+          }
     }
     t0 = mono_ns();
     engine = std::thread([this] { engine_main(); });
@@ -1012,9 +1044,68 @@ class Runtime : public strings::Hooks {
       jc->phys_done[engine] = true;
       return;
     }
+    Logical& lg = logical[j.gid];
+    if (engine == strings::ENG_H2D && jc->slot < 0) assign_slot(lg, jc);   // engine-thread state
+    if (!virtual_clock()) inflight.push_back({jc, engine});
+    if (issue_threads) {
+      // hand the op to its GPU's issuer thread (FIFO: ops issue in wake order)
+      Phys* ph = lg.phys;
+      {
+        std::lock_guard<std::mutex> g(ph->iq_mu);
+        ph->iq.push_back({jc, engine});
+      }
+      ph->iq_len.fetch_add(1, std::memory_order_release);
+      ph->iq_cv.notify_one();
+      return;
+    }
     const uint64_t i0 = mono_ns();
     issue(j, jc, engine);
     issue_ns += mono_ns() - i0;
+  }
+
+  // Issuer thread of one GPU: drain its queue of woken ops in order.  Spins
+  // (yielding) while ops keep coming, sleeps on the condition after ~200 us idle.
+  void issuer_main(Phys* ph) {
+    uint64_t idle_since = mono_ns();
+    for (;;) {
+      if (ph->iq_len.load(std::memory_order_acquire) == 0) {
+        if (mono_ns() - idle_since < 200000ull) {
+          std::this_thread::yield();
+          continue;
+        }
+        std::unique_lock<std::mutex> lk(ph->iq_mu);
+        ph->iq_cv.wait_for(lk, std::chrono::milliseconds(1), [ph] { return ph->iq_stop || !ph->iq.empty(); });
+        if (ph->iq.empty()) {
+          if (ph->iq_stop) return;
+          continue;
+        }
+      }
+      std::pair<JobCtx*, int> op;
+      {
+        std::lock_guard<std::mutex> g(ph->iq_mu);
+        if (ph->iq.empty()) continue;
+        op = ph->iq.front();
+        ph->iq.pop_front();
+      }
+      ph->iq_len.fetch_sub(1, std::memory_order_relaxed);
+      const uint64_t i0 = mono_ns();
+      issue(op.first->job, op.first, op.second);
+      issue_ns += mono_ns() - i0;
+      idle_since = mono_ns();
+    }
+  }
+
+  // The job's resident slot and its device pointers (at its H2D wake).
+  void assign_slot(Logical& lg, JobCtx* jc) {
+    jc->slot = lg.free_slots.back();
+    lg.free_slots.pop_back();
+    uint8_t* base = lg.arena + (size_t)jc->slot * cfg.slot_bytes;
+    uint64_t off = 0;
+    for (size_t i = 0; i < jc->in.size(); ++i) {
+      jc->dev_in[i] = reinterpret_cast<uint64_t>(base + off);
+      off = align_up(off + jc->in[i].bytes);
+    }
+    jc->dev_out = reinterpret_cast<uint64_t>(base + off);
   }
 
   // The job's KL work item (device pointers of its slot; GEMM tensor maps).
@@ -1054,41 +1145,25 @@ class Runtime : public strings::Hooks {
     if ((uint64_t)cfg.admit_cap > (uint64_t)cfg.awake_budget && inflight_cap_sum > (uint64_t)cfg.awake_budget)
       return false;
     if (jc->job.h2d_bytes <= sm_copy_max || jc->job.d2h_bytes <= sm_copy_max) return false;
-    return lg.tail[1] - lg.completed[1] < (uint32_t)kRing;
+    return lg.tail[1] - __atomic_load_n(&lg.completed[1], __ATOMIC_ACQUIRE) < (uint32_t)kRing;
   }
 
   void issue(strings::Job& j, JobCtx* jc, int engine) {
     Logical& lg = logical[j.gid];
     Phys* ph = lg.phys;
-    if (jc->eager && engine != strings::ENG_H2D) {
-      // queued on the device at H2D issue: the model's wake has nothing left to issue
-      if (!virtual_clock()) inflight.push_back({jc, engine});
-      return;
-    }
+    if (jc->eager && engine != strings::ENG_H2D) return;   // queued on the device at H2D issue
     set_dev(ph->dev);
     bool ok = true;
     if (engine == strings::ENG_H2D && eager_ok(jc, lg)) {
       ok = issue_eager(j, jc, lg);
-      jc->issued[engine] = true;
       if (!ok) {
         fail_job(jc);
         for (int e = 0; e < 3; ++e) jc->phys_done[e] = true;
       }
-      if (!virtual_clock()) inflight.push_back({jc, engine});
+      jc->issued[engine] = true;
       return;
     }
     if (engine == strings::ENG_H2D) {
-      if (jc->slot < 0) {
-        jc->slot = lg.free_slots.back();
-        lg.free_slots.pop_back();
-        uint8_t* base = lg.arena + (size_t)jc->slot * cfg.slot_bytes;
-        uint64_t off = 0;
-        for (size_t i = 0; i < jc->in.size(); ++i) {
-          jc->dev_in[i] = reinterpret_cast<uint64_t>(base + off);
-          off = align_up(off + jc->in[i].bytes);
-        }
-        jc->dev_out = reinterpret_cast<uint64_t>(base + off);
-      }
       if (sm_copy_eligible(jc->in, ph, engine)) {
         // small inputs (+ the KL work item) as one zero-copy item on the copy partition
         CopyItem ci;
@@ -1104,12 +1179,11 @@ class Runtime : public strings::Hooks {
                                it.kclass == STRINGS_GEMM ? sizeof(KlItem) : offsetof(KlItem, tmap_a)};
         }
         ok = publish_copy(ph, jc, engine, ci);
-        jc->issued[engine] = true;
         if (!ok) {
           fail_job(jc);
           jc->phys_done[engine] = true;
         }
-        if (!virtual_clock()) inflight.push_back({jc, engine});
+        jc->issued[engine] = true;
         return;
       }
       for (size_t i = 0; i < jc->in.size() && ok; ++i)
@@ -1164,7 +1238,7 @@ class Runtime : public strings::Hooks {
     } else if (kl_mode == 0) {
       if (!await_item_copy(ph, jc)) {
         ok = false;
-      } else if (!jc->item_ok || lg.tail[0] - lg.completed[0] >= (uint32_t)kRing) {
+      } else if (!jc->item_ok || lg.tail[0] - __atomic_load_n(&lg.completed[0], __ATOMIC_ACQUIRE) >= (uint32_t)kRing) {
         ok = false;   // bad item (fault localised to this job); a full ring cannot happen with A <= kRing
       } else {
         // one 64-bit stream memory op publishes ring entry (seq, kclass, slot); it is
@@ -1200,12 +1274,11 @@ class Runtime : public strings::Hooks {
         ok = ok && jc->ev[engine] && cuda_ok(cudaEventRecord(jc->ev[engine], s));
       }
     }
-    jc->issued[engine] = true;
     if (!ok) {
       fail_job(jc);
       jc->phys_done[engine] = true;   // a failed op completes immediately (fault localised)
     }
-    if (!virtual_clock()) inflight.push_back({jc, engine});
+    jc->issued[engine] = true;
   }
 
   void on_start(strings::Job& j, int engine, int slot, uint64_t t) override {
@@ -1334,7 +1407,7 @@ class Runtime : public strings::Hooks {
     volatile KlDone* d = &ph->cdone[idx];
     if (d->seq != seq) return false;
     std::atomic_thread_fence(std::memory_order_acquire);
-    ph->ccompleted += 1;
+    __atomic_fetch_add(&ph->ccompleted, 1u, __ATOMIC_RELAXED);
     ph->cbusy[idx] = 0;
     return true;
   }
@@ -1356,17 +1429,6 @@ class Runtime : public strings::Hooks {
   // The whole H2D -> KL -> D2H chain of an eager job, queued now (see eager_ok).
   bool issue_eager(strings::Job& j, JobCtx* jc, Logical& lg) {
     Phys* ph = lg.phys;
-    if (jc->slot < 0) {
-      jc->slot = lg.free_slots.back();
-      lg.free_slots.pop_back();
-      uint8_t* base = lg.arena + (size_t)jc->slot * cfg.slot_bytes;
-      uint64_t off = 0;
-      for (size_t i = 0; i < jc->in.size(); ++i) {
-        jc->dev_in[i] = reinterpret_cast<uint64_t>(base + off);
-        off = align_up(off + jc->in[i].bytes);
-      }
-      jc->dev_out = reinterpret_cast<uint64_t>(base + off);
-    }
     KlItem& it = lg.item_host[jc->slot];
     jc->item_ok = build_item(j, jc, it);
     if (!jc->item_ok) return false;
@@ -1430,6 +1492,7 @@ class Runtime : public strings::Hooks {
   }
 
   cudaEvent_t take_event(Phys* ph) {
+    std::lock_guard<std::mutex> g(ph->ev_mu);
     if (ph->ev_pool.empty()) {
       cudaEvent_t e;
       if (!cuda_ok(cudaEventCreateWithFlags(&e, cudaEventDisableTiming))) return nullptr;
@@ -1441,7 +1504,9 @@ class Runtime : public strings::Hooks {
   }
   void give_event(JobCtx* jc, int engine) {
     if (jc->ev[engine]) {
-      logical[jc->job.gid].phys->ev_pool.push_back(jc->ev[engine]);
+      Phys* ph = logical[jc->job.gid].phys;
+      std::lock_guard<std::mutex> g(ph->ev_mu);
+      ph->ev_pool.push_back(jc->ev[engine]);
       jc->ev[engine] = nullptr;
     }
   }
@@ -1462,7 +1527,7 @@ class Runtime : public strings::Hooks {
       jc->kl_observe = real_ns();
       // MEASURED timing: the SFT learns the KL's device time (R-14 telemetry)
       if (!virtual_clock() && jc->kl_t1 > jc->kl_t0) jc->job.measured[strings::ENG_KL] = jc->kl_t1 - jc->kl_t0;
-      lg.completed[jc->kl_idx / kRing] += 1;
+      __atomic_fetch_add(&lg.completed[jc->kl_idx / kRing], 1u, __ATOMIC_RELEASE);
       jc->phys_done[engine] = true;
       return true;
     }
@@ -1893,6 +1958,15 @@ class Runtime : public strings::Hooks {
       cv_engine.notify_all();
     }
     if (engine.joinable()) engine.join();
+    for (auto& ph : phys) {                 // the engine is gone: no more wakes to hand over
+      if (!ph->issuer.joinable()) continue;
+      {
+        std::lock_guard<std::mutex> g(ph->iq_mu);
+        ph->iq_stop = true;
+      }
+      ph->iq_cv.notify_all();
+      ph->issuer.join();
+    }
     {
       std::lock_guard<std::mutex> g(mu);
       stop_final = true;
@@ -2050,6 +2124,9 @@ strings_status_t strings_get_stats(strings_stats_t* st) {
   st->decisions = r.core->decisions();
   st->decision_ns = r.decision_ns;
   st->issue_ns = r.issue_ns;
+  // with issuer threads the driver calls run outside the engine's decision time: add
+  // them so that decision_ns - issue_ns stays the decision core's own time
+  if (r.issue_threads) st->decision_ns += st->issue_ns;
   for (size_t i = 0; i < r.phys.size() && i < 8; ++i) st->gpu_clock_offset_ns[i] = r.phys[i]->clock_offset_ns;
   st->sm_copy_ops = r.sm_copies;
   st->kl_mode = r.kl_mode;

@@ -454,3 +454,19 @@ def test_ext_streams_rejects_a_duplicate_handle():
         S.init_from_config(wl.config.resolved(), timing_mode=S.INJECTED, physical_gpus=1,
                            streams=[s, s, None, None])
     assert e.value.status == S.EINVAL
+
+
+@pytest.mark.parametrize("timing", [S.INJECTED, S.MEASURED])
+def test_issuer_threads(monkeypatch, timing):
+    # one issuer thread per GPU (the default with >= 2 GPUs; forced here on one):
+    # the engine thread hands woken ops over in wake order; decisions and
+    # outputs must not change
+    monkeypatch.setenv("STRINGS_ISSUE_THREADS", "1")
+    for wl in (W.config_c1(reps=4), W.config_c3(scale=8), W.config_c5(scale=64, jobs_per_tenant=4)):
+        r = run_workload(wl, timing_mode=timing)
+        assert r.status == S.OK
+        if timing == S.INJECTED:
+            assert r.trace == run_oracle(wl).trace
+        else:
+            assert invariants.check(r.trace, wl) == []
+        check_outputs(wl, r)

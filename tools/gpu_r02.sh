@@ -26,6 +26,12 @@ for l in open('gpurun_out/configs_eager$e.log'):
     ncu_kernels) for k in vscale xfer gemm scan hist sort; do timeout 900 ncu --set full --clock-control none --import-source on -k regex:oneshot -c 2 -f -o gpurun_out/prof_$k python tools/kernel_probe.py $k > gpurun_out/ncu_$k.log 2>&1; echo "ncu $k rc=$?"; done ;;
     benchdef) timeout 1200 python bench.py > gpurun_out/benchdef.log 2>&1; echo "benchdef rc=$?"; tail -c 400 gpurun_out/benchdef.log ;;
     ref) timeout 900 python bench.py --impl reference --steps ${STEPS:-20} --warmup ${WARMUP:-5} > gpurun_out/ref.log 2>&1; echo "ref rc=$?"; tail -c 800 gpurun_out/ref.log ;;
+    configs_it) for e in 1 0; do STRINGS_ISSUE_THREADS=$e BENCH_CONFIGS=${CONFIGS:-C1,C3,C5,C2} timeout 1800 python bench.py --configs --config-repeats ${REPEATS:-3} > gpurun_out/configs_it$e.log 2>&1; echo "issue_threads=$e rc=$?"; python -c "
+import json
+for l in open('gpurun_out/configs_it$e.log'):
+    if l.startswith('{'):
+        d=json.loads(l); print(d['config'], d['jobs_per_s'], d['span_ms'], d['roofline_frac'], d['span_ms_min_max'], 'dec', d['decision_us_per_job'], 'iss', d['issue_us_per_job'])
+"; done ;;
     *) echo "unknown task $task" ;;
   esac
 done
