@@ -67,6 +67,8 @@ def parse_args():
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
     p.add_argument("--config-repeats", type=int, default=3, help="timed runs per config in --configs")
     p.add_argument("--config-static", action="store_true", help="--configs: add static baselines")
+    p.add_argument("--baseline-config-static", action="store_true",
+                   help="N > 1: also time static provisioning on the BASELINE config")
     p.add_argument("--no-baseline-config", action="store_true",
                    help="N > 1: skip the BASELINE config whose G equals N (C1/C3/C5)")
     p.add_argument("--configs", action="store_true",
@@ -729,16 +731,28 @@ def run_node(args, torch, gloo, world):
     for _ in range(args.warmup):
         one_step()
     stream.synchronize()
+    timed_ids = []
     with ClockSampler(list(range(phys))) as clk:
         ev0.record(stream)
         t_wall = time.perf_counter()
         for _ in range(args.steps):
             one_step()
+            timed_ids.extend(ids)
         ev1.record(stream)
         ev1.synchronize()
         t_wall = time.perf_counter() - t_wall
     dt = max_over(gloo, ev0.elapsed_time(ev1) / 1e3)
     infos = [S.job_info(i) for i in ids]            # the last timed step
+    # the dominant kernel: XFER work items of every timed step on every GPU (device stamps)
+    xf = [S.job_info(i) for i, sp in zip(timed_ids, wl.jobs * args.steps) if sp.kclass == W.XFER]
+    dev_us = sorted((r.kl_gpu_end_ns - r.kl_gpu_start_ns) / 1e3 for r in xf if r.kl_gpu_end_ns)
+    body_us = sorted((r.kl_gpu_end_ns - r.kl_gpu_exec_ns) / 1e3 for r in xf if r.kl_gpu_exec_ns)
+    kl_lat = {}
+    if dev_us:
+        kl_lat["XFER"] = {"kl_device_us_p50": round(dev_us[len(dev_us) // 2], 1),
+                          "kl_device_us_mean": round(sum(dev_us) / len(dev_us), 2), "items": len(dev_us),
+                          "kl_body_us_mean": round(sum(body_us) / len(body_us), 2) if body_us else None,
+                          "kl_body_us_p50": round(body_us[len(body_us) // 2], 1) if body_us else None}
     stats = S.stats()
     jobs_step = len(wl.jobs)
     e2e = None
@@ -801,7 +815,9 @@ def run_node(args, torch, gloo, world):
                    "ranks": f"{world} (rank 0 drives the node; other ranks idle: no data-path collective)",
                    "kl_mode": "persistent dispatcher" if stats.kl_mode == 0 else "per-op launches"},
         "placement": {str(g): placed.get(g, 0) for g in range(N)},
-        "roofline": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(agg_peak, 2),
+        # the dominant kernel (the contract's `roofline`): the XFER work items on every GPU
+        "roofline": _kernel_roofline(kl_lat, wl, peaks),
+        "roofline_step": {"bound": "host_link", "achieved": round(link_gbs, 2), "peak": round(agg_peak, 2),
                      "unit": "GB/s", "frac": round(link_gbs / agg_peak, 4), "traffic": None,
                      "resource": f"copy engines H2D+D2H of {phys} GPU(s)",
                      "peak_source": "measured in this run: pinned H2D+D2H 256 MiB copies on every GPU at once"},
@@ -841,8 +857,9 @@ def run_node(args, torch, gloo, world):
     if not args.no_baseline_config:
         name = {2: "C1", 4: "C3", 8: "C5"}.get(N)
         if name:
-            res["baseline_config"] = config_result(torch, name, phys, link, peaks, repeats=3,
-                                                   static=not args.no_static)
+            # (its own static baselines only on request: at N = 8 they spawn 2 x 128 processes)
+            res["baseline_config"] = config_result(torch, name, phys, link, peaks, repeats=2,
+                                                   static=args.baseline_config_static and not args.no_static)
     return res, wl
 
 
