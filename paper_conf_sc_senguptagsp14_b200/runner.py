@@ -32,15 +32,20 @@ class RunResult:
 def run_workload(wl: W.Workload, timing_mode: int = S.INJECTED, pinned: bool = True,
                  inputs: Optional[List[List[np.ndarray]]] = None, keep_inputs: bool = False,
                  trace_path: Optional[str] = None, physical_gpus: int = 0, kl_mode: int = 0,
-                 slot_bytes: int = 0, torch_memory: bool = True, streams=None) -> RunResult:
+                 slot_bytes: int = 0, torch_memory: bool = True, streams=None,
+                 library_defaults: bool = False) -> RunResult:
+    """library_defaults: pass the workload's config as written (A = 0, M = 0,
+    joint_select = -1 ...) and let the library fill in its defaults, instead of
+    the generator's resolved values."""
     cfg = wl.config.resolved()
+    init_cfg = wl.config if library_defaults else cfg
     arenas = None
     if timing_mode != S.DECISIONS_ONLY and torch_memory:
         import torch                       # PyTorch provides the device memory (slot arenas)
         nphys = physical_gpus or torch.cuda.device_count()
         arenas = S.torch_arenas(cfg.num_gpus, min(nphys, cfg.num_gpus), cfg.admit_cap, slot_bytes)
         physical_gpus = len(arenas)
-    S.init_from_config(cfg, timing_mode=timing_mode, trace_path=trace_path, physical_gpus=physical_gpus,
+    S.init_from_config(init_cfg, timing_mode=timing_mode, trace_path=trace_path, physical_gpus=physical_gpus,
                        kl_mode=kl_mode, slot_bytes=slot_bytes, arenas=arenas, streams=streams)
     pinned_arrays = []
     try:

@@ -249,3 +249,13 @@ def test_binding_structs_match_the_header_layout(pyname, cname, tmp_path):
     out = [int(v) for v in subprocess.run([str(exe)], check=True, capture_output=True, text=True).stdout.split()]
     assert out[0] == ctypes.sizeof(st), (cname, out[0], ctypes.sizeof(st))
     assert out[1:] == [getattr(st, n).offset for n in names], cname
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4c", "C5"])
+def test_library_defaults_match_the_readings(name):
+    # A = 2 + P (R-11), M = 2A (R-12), joint selection on for DTF/MBF/DYNAMIC (R-16):
+    # the library's own defaulting (strings_init with 0 / -1) gives the oracle's trace
+    wl = W.CONFIGS[name]()
+    assert wl.config.awake_budget == 0 and wl.config.joint_select == -1
+    r = run_workload(wl, timing_mode=S.DECISIONS_ONLY, library_defaults=True)
+    assert r.trace == run_oracle(wl).trace
