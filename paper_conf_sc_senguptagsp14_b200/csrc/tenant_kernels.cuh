@@ -238,13 +238,18 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
     uint32_t next = kNoChunk;                     // thread 0: the claim for the next load
     bool claiming = true;                         // thread 0: the counter may still hold chunks
     // The first kStreamLead rounds are dealt statically to the group's own CTAs
-    // (chunk rank + j*S): their loads go out at once, with no atomic round trip
-    // on the item's start-up path; the counter hands out the chunks after them.
-    const uint64_t dealt = nchunks < (uint64_t)kStreamLead * S ? nchunks : (uint64_t)kStreamLead * S;
+    // (chunk r + j*D over D dealt ranks): their loads go out at once, with no atomic
+    // round trip on the item's start-up path; the counter hands out the chunks after
+    // them.  Inside the dispatcher (total_word set) rank 0 hosts the partition
+    // leader, which starts its own share last (claim, release, lending decision), so
+    // it takes counter chunks only.
+    const int d0 = total_word ? 1 : 0;            // first dealt rank
+    const int D = S - d0;                         // dealt ranks
+    const uint64_t dealt = D <= 0 ? 0 : (nchunks < (uint64_t)kStreamLead * D ? nchunks : (uint64_t)kStreamLead * D);
     int pre = 0;                                  // thread 0: statically dealt chunks used so far
     auto claim = [&]() -> uint32_t {
-      if (rank < S && pre < kStreamLead) {
-        const uint64_t c = (uint64_t)rank + (uint64_t)(pre++) * S;
+      if (rank >= d0 && rank < S && pre < kStreamLead) {
+        const uint64_t c = (uint64_t)(rank - d0) + (uint64_t)(pre++) * D;
         if (c < dealt) return (uint32_t)c;
         pre = kStreamLead;                        // this CTA's static share is used up
       }
