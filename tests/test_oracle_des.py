@@ -443,3 +443,54 @@ def test_invariant_checker_catches_las_wake_order():
             if any(e.startswith("I2") for e in invariants.check(m, wl)):
                 return
     pytest.fail("no LAS wake-order mutation detected")
+
+
+# ------------------------------------------------ invariant checker, check by check
+def _relabel(trace, a, b):
+    """Swap jobs a and b (same tenant) in every record: their admissions and
+    phase starts then happen in the opposite of submission order."""
+    out = []
+    for ln in trace:
+        f = ln.split()
+        if f[7] in (str(a), str(b)):
+            ja, jb = (a, b) if f[7] == str(a) else (b, a)
+            f[7] = str(jb)
+            f[6] = str(_relabel.seq[jb])
+        out.append(" ".join(f))
+    return out
+
+
+def test_invariant_checker_each_check_fires():
+    # every check of oracle/invariants.py must flag a trace that breaks exactly its rule
+    # I4 (P:L299): swap two jobs of one tenant (c_t = 1): admitted and started out of order
+    wl = W.config_c1(reps=2)
+    o = run_oracle(wl)
+    t0 = [j for j in o.jobs if j.tenant == 0]
+    _relabel.seq = {j.id: j.seq for j in o.jobs}
+    errs = invariants.check(_relabel(o.trace, t0[0].id, t0[1].id), wl)
+    assert any("placed job" in e and e.startswith("I4") for e in errs)
+    assert any("started after a later job" in e for e in errs)
+    # I3: the trace of M = 2 checked against M = 1
+    wl2 = W.config_c2(scale=256, jobs_per_tenant=2)
+    wl2.config.admit_cap = 2
+    tr = run_oracle(wl2).trace
+    wl2.config.admit_cap = 1
+    assert any(e.startswith("I3") and "> M=1" in e for e in invariants.check(tr, wl2))
+    # I5 (budget): the trace of A = 1 checked against A = 3
+    wl3 = W.config_c3(scale=16)
+    wl3.config.awake_budget, wl3.config.admit_cap = 1, 8
+    tr = run_oracle(wl3).trace
+    wl3.config.awake_budget = 3
+    assert any("candidates unwoken with budget" in e for e in invariants.check(tr, wl3))
+    # I5 (idle engine): the trace of P = 1 checked against P = 2 (a woken KL waits beside a free slot)
+    cfg4 = W.SystemConfig(num_gpus=1, partitions=1, awake_budget=4, admit_cap=8, device_policy=W.PS)
+    wl4 = W.Workload("p1", cfg4, [W.TenantSpec() for _ in range(4)],
+                     [kl_only_job(t, 10_000) for _ in range(2) for t in range(4)])
+    tr = run_oracle(wl4).trace
+    wl4.config.partitions = 2
+    assert any("idle with woken op" in e for e in invariants.check(tr, wl4))
+    # I7 (TFS, P:L699): a PS trace checked as TFS wakes several tenants at once
+    wl5 = W.config_c2(scale=256, jobs_per_tenant=2)
+    tr = run_oracle(wl5).trace
+    wl5.config.device_policy = W.TFS
+    assert any(e.startswith("I7") for e in invariants.check(tr, wl5))

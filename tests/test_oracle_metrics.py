@@ -31,6 +31,13 @@ def test_roofline_terms():
     assert metrics.roofline_tstar([j, dict(j)], pk) == pytest.approx(3e-3)
     # two tenants: link bound 2 ms
     assert metrics.roofline_tstar([j, dict(j, tenant=1)], pk) == pytest.approx(2e-3)
+    # HBM carries the copies too: 1 GB/s of HBM, 1 + 0.5 MB copied -> 1.5 ms (> the 1 ms link term)
+    slow_hbm = dict(pk, B_hbm=1e9)
+    k = dict(h2d=1e6, d2h=5e5, hbm=0.0, flop=0.0, tenant=0)
+    assert metrics.roofline_tstar([k, dict(k, tenant=1)], slow_hbm) == pytest.approx(3e-3)
+    # open-loop arrival bound: a job arriving at 10 ms finishes no earlier than 10 ms + its chain
+    late = dict(j, arrival=10e-3)
+    assert metrics.roofline_tstar([dict(j, tenant=1), late], pk, t0=0.0) == pytest.approx(10e-3 + 1.5e-3)
 
 
 # ---------------------------------------------------------------- Eq. (4)

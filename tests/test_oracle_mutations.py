@@ -75,6 +75,28 @@ MUTATIONS = [
      "return (a.astype(np.float32) @ b.astype(np.float32)).astype(np.float32)"),
     ("jain_unsquared_sum", "oracle/metrics.py",
      "return sum(xs) ** 2 / (n * s2)", "return sum(xs) / (n * s2)"),
+    ("ws_inverted", "oracle/metrics.py",
+     "return sum(b / p for b, p in zip(base_lat, policy_lat)) / len(base_lat)",
+     "return sum(p / b for b, p in zip(base_lat, policy_lat)) / len(base_lat)"),
+    ("tstar_no_chain", "oracle/metrics.py",
+     "terms.append(max(v / inflight.get(t, 1) for t, v in chains.items()))", "pass"),
+    ("tstar_hbm_only", "oracle/metrics.py",
+     'sum(j["hbm"] + j["h2d"] + j["d2h"] for j in jobs) / bm,', 'sum(j["hbm"] for j in jobs) / bm,'),
+    ("tstar_no_arrival", "oracle/metrics.py",
+     'terms.append(max(j.get("arrival", 0.0) + j["h2d"] / bh + klstar(j) + j["d2h"] / bd for j in jobs) - t0)',
+     "pass"),
+    ("bruteforce_max", "oracle/bruteforce.py", "if best is None or v < best:", "if best is None or v > best:"),
+    ("inv_no_I4_admission", "oracle/invariants.py",
+     'errs.append(f"I4 tenant {tn} placed job {j} before {pending[tn][0]}")', "pass"),
+    ("inv_M_off_by_one", "oracle/invariants.py", "if len(resident[g]) > M:", "if len(resident[g]) > M + 1:"),
+    ("inv_no_I5_budget", "oracle/invariants.py",
+     'errs.append(f"I5 t={t} gid={g} {len(c)} candidates unwoken with budget {A - woken_unf[g]}")', "pass"),
+    ("inv_no_I5_idle", "oracle/invariants.py",
+     'errs.append(f"I5 t={t} gid={g} engine {x} idle with woken op")', "pass"),
+    ("inv_no_I4_start", "oracle/invariants.py",
+     'errs.append(f"I4 tenant {ten_of[j]} engine {x} job {j} started after a later job")', "pass"),
+    ("inv_no_I7", "oracle/invariants.py",
+     'errs.append(f"I7 t={r.t} gid={g} TFS woke tenant {ten_of[j]} while {others} awake")', "pass"),
 ]
 
 PIN_FILES = ["test_oracle_pins.py", "test_oracle_des.py", "test_golden.py",
@@ -86,7 +108,7 @@ def _stage(dst):
         shutil.copytree(os.path.join(ROOT, d), os.path.join(dst, d),
                         ignore=shutil.ignore_patterns("__pycache__"))
     os.makedirs(os.path.join(dst, "tests"))
-    for f in ["conftest.py"] + PIN_FILES:
+    for f in ["conftest.py", "gemm_bounds.py"] + PIN_FILES:
         shutil.copy(os.path.join(ROOT, "tests", f), os.path.join(dst, "tests", f))
     shutil.copytree(os.path.join(ROOT, "tests", "golden"), os.path.join(dst, "tests", "golden"))
     shutil.copy(os.path.join(ROOT, "pytest.ini"), os.path.join(dst, "pytest.ini"))
@@ -102,11 +124,9 @@ def _run_pins(dst):
 def test_every_mutation_is_caught_by_a_pin(tmp_path):
     base = tmp_path / "base"
     _stage(str(base))
-    # the unmutated copy must pass its pins (so a failure below is the mutation's)
-    r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
-                        os.path.join("tests", "test_oracle_pins.py")],
-                       cwd=str(base), env=dict(os.environ, PYTHONPATH=str(base)),
-                       capture_output=True, text=True, timeout=600)
+    # the unmutated copy must pass every pin file (so a failure below is the
+    # mutation's, never the harness's)
+    r = _run_pins(str(base))
     assert r.returncode == 0, r.stdout[-2000:]
 
     def one(m):
@@ -121,7 +141,7 @@ def test_every_mutation_is_caught_by_a_pin(tmp_path):
         return name, r.returncode, r.stdout[-1500:]
 
     muts = MUTATIONS
-    assert len(muts) >= 20
+    assert len(muts) >= 30
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:
         results = list(ex.map(one, muts))
     survivors = [(n, rc, out) for n, rc, out in results if rc != 1]
