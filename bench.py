@@ -1167,6 +1167,10 @@ def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, st
     from paper_conf_sc_senguptagsp14_b200 import strings as S
 
     wl = W.CONFIGS[name]()
+    if os.environ.get("BENCH_AWAKE_BUDGET"):       # experiments: override A (M follows unless set)
+        wl.config.awake_budget = int(os.environ["BENCH_AWAKE_BUDGET"])
+    if os.environ.get("BENCH_ADMIT_CAP"):
+        wl.config.admit_cap = int(os.environ["BENCH_ADMIT_CAP"])
     # arrivals are submit times in MEASURED mode: the whole config is offered at t = 0
     wl = dataclasses.replace(wl, jobs=[dataclasses.replace(j, arrival_ns=0) for j in wl.jobs])
     cfg = wl.config.resolved()
