@@ -613,16 +613,24 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
 // CTA's loads stay 16-B aligned when the buffers are.
 constexpr int kScanPT = 32;
 // One 32 KB chunk (8192 u32) scanned in place in shared memory: warp w owns
-// elements [1024w, 1024w + 1024) and walks them in 32 rounds of 32 consecutive
-// words (lane l reads word 32r + l: conflict-free), carrying its running sum;
-// the warps' offsets come from their chunk totals (phase A).  Returns the
-// chunk total; `carry` is the sum of everything before the chunk.
+// elements [1024w, 1024w + 1024) as 256 16-B vectors; lane l takes vector
+// 32m + l in round m = 0..7 (consecutive lanes, consecutive 16 B: conflict-free
+// 128-bit shared loads).  A round scans its 128 elements as four in-thread adds
+// plus one 5-step warp scan over the lanes' vector sums, so a chunk costs 8 x 6
+// shuffles per warp (a scan per 32 words cost 32 x 6).  The eight vectors stay
+// in registers between the warp-total pass and the scan pass; the warps'
+// offsets come from their totals.  Returns the chunk total; `carry` is the sum
+// of everything before the chunk.
 __device__ __forceinline__ uint32_t scan_chunk_smem(uint32_t* c, uint32_t carry, uint32_t* wtot) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t* mine = c + warp * 1024;
+  uint4* mine = reinterpret_cast<uint4*>(c) + warp * 256;
+  uint4 q[8];
   uint32_t s = 0;
-#pragma unroll 8
-  for (int r = 0; r < 32; ++r) s += mine[r * 32 + lane];
+#pragma unroll
+  for (int m = 0; m < 8; ++m) {
+    q[m] = mine[32 * m + lane];
+    s += q[m].x + q[m].y + q[m].z + q[m].w;
+  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   if (lane == 0) wtot[warp] = s;
@@ -633,11 +641,12 @@ __device__ __forceinline__ uint32_t scan_chunk_smem(uint32_t* c, uint32_t carry,
     if (w < warp) run += t;
     total += t;
   }
-#pragma unroll 4
-  for (int r = 0; r < 32; ++r) {
-    const uint32_t v = mine[r * 32 + lane];
-    const uint32_t incl = warp_incl_scan(v);
-    mine[r * 32 + lane] = run + incl;
+#pragma unroll
+  for (int m = 0; m < 8; ++m) {
+    const uint32_t a = q[m].x, b = a + q[m].y, d3 = b + q[m].z, d = d3 + q[m].w;
+    const uint32_t incl = warp_incl_scan(d);
+    const uint32_t e = run + incl - d;                             // sum before this lane's vector
+    mine[32 * m + lane] = make_uint4(e + a, e + b, e + d3, e + d);
     run += __shfl_sync(0xffffffffu, incl, 31);
   }
   return total;
