@@ -67,13 +67,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 // A "group" is the S CTAs running one item (an SM partition of the dispatcher,
 // or a stand-alone grid).  All of them are co-resident (one CTA per SM), so a
 // counter/generation barrier in global memory is safe.
+constexpr int kScanRing = 8;          // SCAN: rows of GroupSync::wave (wave k uses row k mod 8)
 struct __align__(128) GroupSync {
   uint32_t bar_cnt;
   uint32_t bar_gen;
   uint32_t chunk_next;                 // streaming items: next unclaimed 32 KB chunk (dynamic claiming)
   uint32_t chunk_done;                 // streaming items: CTAs finished claiming (the last one resets both)
-  uint32_t pad[28];
+  uint32_t scan_epoch;                 // SCAN items finished on this group (tags the wave table)
+  uint32_t scan_done;                  // CTAs finished with the current SCAN item (the last one bumps the epoch)
+  uint32_t pad[26];
   uint32_t partial[256];               // per-CTA partial results (S <= 256)
+  uint64_t wave[kScanRing * 256];      // SCAN: (tag << 32) | sum of rank r's part of wave k, at [(k % 8) * 256 + r]
 };
 
 // ---------------------------------------------------------------- streaming
@@ -652,9 +656,12 @@ __device__ __forceinline__ uint32_t scan_chunk_smem(uint32_t* c, uint32_t carry,
   return total;
 }
 
-__device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
-                                 int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* wsum,
-                                 uint32_t* sphase) {
+// Reduce-then-scan over the whole group (unaligned buffers; STRINGS_SCAN_TWOPASS=1
+// for every buffer): per-CTA chunk sums -> group barrier -> chunk offsets -> the
+// chunk again through the pipeline.  Reads the input twice (12n bytes).
+__device__ inline void scan_body_twopass(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
+                                         int rank, int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar,
+                                         uint32_t* wsum, uint32_t* sphase) {
   // wsum: 16 words outside the stages ([8] warp totals + [8] broadcast / second buffer)
   constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;
   const uint64_t chunk = ((n + S - 1) / S + kTile - 1) / kTile * kTile;
@@ -792,6 +799,293 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
     carry += tile;
     __syncthreads();
   }
+}
+
+// L2 eviction-priority policies for the cache_hint forms of loads and bulk copies.
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                              uint64_t pol) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void bulk_s2g_hint(void* dst, const void* src, uint32_t bytes, uint64_t pol) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;"
+               :: "l"(dst), "r"(smem_u32(src)), "r"(bytes), "l"(pol) : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+
+// Target bytes of one SCAN wave: about three waves of input must stay in L2 (a
+// wave's input is read from HBM two waves before it is scanned).  Measured on the
+// B200 at 2^28 on 148 CTAs (profiles/r02_scan.md): 16 MB (19 MB waves) reads 1.05x
+// the input from DRAM, 22 MB 1.31x; smaller waves add per-wave overhead.
+#ifndef STRINGS_SCAN_WAVE_MB
+#define STRINGS_SCAN_WAVE_MB 16
+#endif
+
+// y = inclusive prefix sum of x (u32, mod 2^32) reading the input from HBM once
+// (8n bytes, the algorithmic traffic).  The buffer is cut into waves of S
+// sub-blocks (sub-block r of wave k = CTA r's, a whole number of 32 KB chunks,
+// about STRINGS_SCAN_WAVE_MB per wave).  CTA r first sums its sub-blocks of
+// waves 0 and 1; then for k = 0, 1, ...:
+//   lookup(k)  the S tagged words of wave k (published a whole wave earlier, so
+//              normally there is no wait): offset = sum of the waves < k + the
+//              ranks < r of wave k;
+//   scan(k)    its sub-block of wave k, an L2 hit now, through the TMA bulk
+//              pipeline: each 32 KB chunk scanned in shared memory and
+//              bulk-stored, loads and stores with an evict-first hint (the last
+//              use of x; y must not push later waves' x out of L2);
+//   sum(k+2)   interleaved with scan(k) chunk by chunk in the same bulk
+//              pipeline: one 32 KB chunk of its sub-block of wave k+2 per
+//              scanned chunk, summed from shared memory, loaded with the default
+//              L2 policy so the lines stay for scan(k+2); published at the end.
+// So HBM sees a steady mix of x reads and y writes, and the bulk pipeline runs
+// across wave boundaries (a position's load does not depend on any offset).
+// No group barrier: the words carry a tag (item epoch, wave index); wave k uses
+// row k mod 8, which no CTA can overwrite while another still needs it (a CTA
+// writing wave k+2's row has seen every CTA's sum(k), so every CTA is at
+// lookup(k-1) or later).  The epoch moves when the item's last CTA finishes.
+// Ragged last sub-blocks end in the register tile path.
+__device__ inline void scan_regs(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t r0, uint64_t b1,
+                                 uint32_t carry, bool vec, uint32_t* wsum) {
+  constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  auto load_tile = [&](uint64_t base, uint32_t* w) {
+    const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
+    if (vec && e0 + kScanPT <= b1) {
+#pragma unroll
+      for (int u = 0; u < kScanPT / 4; ++u) {
+        const uint4 q = reinterpret_cast<const uint4*>(x + e0)[u];
+        w[4 * u] = q.x; w[4 * u + 1] = q.y; w[4 * u + 2] = q.z; w[4 * u + 3] = q.w;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < kScanPT; ++i) w[i] = (e0 + i < b1) ? x[e0 + i] : 0u;
+    }
+  };
+  uint32_t nxt[kScanPT];
+  if (r0 < b1) load_tile(r0, nxt);
+  for (uint64_t base = r0; base < b1; base += kTile) {
+    const uint64_t e0 = base + (uint64_t)threadIdx.x * kScanPT;
+    const bool full = vec && e0 + kScanPT <= b1;
+    uint32_t v[kScanPT];
+#pragma unroll
+    for (int i = 0; i < kScanPT; ++i) v[i] = nxt[i];
+    if (base + kTile < b1) load_tile(base + kTile, nxt);
+    uint32_t run = 0;
+#pragma unroll
+    for (int i = 0; i < kScanPT; ++i) {
+      run += v[i];
+      v[i] = run;
+    }
+    const uint32_t incl = warp_incl_scan(run);
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    uint32_t wpre = 0, tile = 0;
+    for (int w = 0; w < 8; ++w) {
+      const uint32_t t = wsum[w];
+      if (w < warp) wpre += t;
+      tile += t;
+    }
+    const uint32_t excl = carry + wpre + incl - run;
+    if (full) {
+#pragma unroll
+      for (int u = 0; u < kScanPT / 4; ++u)
+        reinterpret_cast<uint4*>(y + e0)[u] =
+            make_uint4(excl + v[4 * u], excl + v[4 * u + 1], excl + v[4 * u + 2], excl + v[4 * u + 3]);
+    } else {
+#pragma unroll
+      for (int i = 0; i < kScanPT; ++i)
+        if (e0 + i < b1) y[e0 + i] = excl + v[i];
+    }
+    carry += tile;
+    __syncthreads();
+  }
+}
+
+__device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
+                                 int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* wsum,
+                                 uint32_t* sphase) {
+  const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
+#if defined(STRINGS_SCAN_TWOPASS) && STRINGS_SCAN_TWOPASS
+  if (true) {
+#else
+  if (!vec) {
+#endif
+    scan_body_twopass(x, y, n, rank, S, gs, stage, sbar, wsum, sphase);
+    return;
+  }
+  // wsum: 32 scratch words: [0, 16) chunk scans (two alternating sets of warp
+  // totals), [16, 24) sum / lookup partials, [24, 32) lookup totals
+  constexpr uint64_t kTile = (uint64_t)kThreads * kScanPT;       // one 32 KB chunk
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t target = (uint64_t)STRINGS_SCAN_WAVE_MB * (1u << 20) / 4 / (uint64_t)S;
+  const uint64_t sb = (target + kTile - 1) / kTile * kTile;        // sub-block elements (>= one chunk)
+  const uint64_t W = sb * (uint64_t)S;
+  const uint64_t K = (n + W - 1) / W;
+  const uint32_t etag = (2u * *reinterpret_cast<volatile uint32_t*>(&gs->scan_epoch) + 1u) << 8;
+  const uint64_t pol = l2_policy_evict_first();
+  auto lo_of = [&](uint64_t k) { return min(n, k * W + (uint64_t)rank * sb); };
+  auto hi_of = [&](uint64_t k) { return min(n, k * W + (uint64_t)(rank + 1) * sb); };
+  auto word = [&](uint64_t k, int r) { return &gs->wave[(k % kScanRing) * 256 + r]; };
+  // block sum of s, published as wave k's word of this rank
+  auto publish = [&](uint64_t k, uint32_t s) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) wsum[16 + warp] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t t = 0;
+      for (int w = 0; w < 8; ++w) t += wsum[16 + w];
+      st_relaxed_u64(word(k, rank), ((uint64_t)(etag | (uint32_t)(k & 0xFF)) << 32) | t);
+    }
+    __syncthreads();
+  };
+  // this thread's share of x[a, b) (a 16-B aligned)
+  auto sum_range = [&](uint64_t a, uint64_t b) -> uint32_t {
+    uint32_t s = 0;
+    if (a >= b) return s;
+    const uint4* x4 = reinterpret_cast<const uint4*>(x + a);
+    const uint64_t n4 = (b - a) / 4;
+    uint64_t i = threadIdx.x;
+    for (; i + 7 * kThreads < n4; i += 8 * kThreads) {
+      uint4 q[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) q[u] = ld_stream(x4 + i + u * kThreads);
+#pragma unroll
+      for (int u = 0; u < 8; ++u) s += q[u].x + q[u].y + q[u].z + q[u].w;
+    }
+    for (; i < n4; i += kThreads) {
+      const uint4 q = ld_stream(x4 + i);
+      s += q.x + q.y + q.z + q.w;
+    }
+    for (uint64_t e = a + n4 * 4 + threadIdx.x; e < b; e += kThreads) s += x[e];
+    return s;
+  };
+  for (uint64_t k = 0; k < 2 && k < K; ++k) publish(k, sum_range(lo_of(k), hi_of(k)));
+  // One bulk pipeline carries two kinds of 32 KB ops, in this order for every
+  // wave k: scan(k, i) for i < nch(k), each followed by sum(k+2, i) while sub-block
+  // k+2 has a whole chunk i.  Positions run across waves (no op's load depends on
+  // an offset).  A sum op's stage is read by every thread and then reused only
+  // after the next op, a scan op, whose __syncthreads orders those reads.
+  auto nch_of = [&](uint64_t k) { return k < K ? (hi_of(k) - lo_of(k)) / kTile : 0; };
+  const uint32_t ph0 = *reinterpret_cast<volatile uint32_t*>(sphase);   // (stream_body's stage barriers)
+  uint64_t pk = 0, pi = 0, issued = 0;                              // thread 0: the next op to load
+  bool psum = false;
+  auto produce = [&]() {                                            // thread 0: load the next op, if any
+    if (pk >= K || pi >= nch_of(pk)) return;
+    const int st = (int)(issued % kStreamStages);
+    if (issued >= (uint64_t)kStreamStages)                          // the store that last read stage st
+      asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kStreamStoreSlack) : "memory");
+    mbar_expect_tx(&sbar[st], kStreamChunk);
+    if (!psum) {
+      bulk_g2s_hint(stage + st * kStreamChunk, x + lo_of(pk) + pi * kTile, kStreamChunk, &sbar[st], pol);
+      psum = pi < nch_of(pk + 2);
+    } else {
+      bulk_g2s(stage + st * kStreamChunk, x + lo_of(pk + 2) + pi * kTile, kStreamChunk, &sbar[st]);
+      psum = false;
+    }
+    ++issued;
+    if (!psum && ++pi >= nch_of(pk)) {
+      ++pk;
+      pi = 0;
+    }
+  };
+  if (threadIdx.x == 0)
+    for (int j = 0; j < kStreamLead; ++j) produce();
+  uint32_t base = 0;                                                // sum of the waves before k
+  uint64_t pos = 0;                                                 // ops consumed
+  uint64_t e = threadIdx.x < S && K ? ld_relaxed_u64(word(0, threadIdx.x)) : 0;
+  for (uint64_t k = 0; k < K; ++k) {
+    // lookup(k)
+    const uint32_t want = etag | (uint32_t)(k & 0xFF);
+    if (threadIdx.x < S)
+      while ((uint32_t)(e >> 32) != want) {
+        __nanosleep(32);
+        e = ld_relaxed_u64(word(k, threadIdx.x));
+      }
+    uint32_t v = threadIdx.x < S ? (uint32_t)e : 0u;
+    uint32_t a = threadIdx.x < rank ? v : 0u;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      v += __shfl_xor_sync(0xffffffffu, v, o);
+      a += __shfl_xor_sync(0xffffffffu, a, o);
+    }
+    if (lane == 0) {
+      wsum[16 + warp] = a;
+      wsum[24 + warp] = v;
+    }
+    __syncthreads();
+    uint32_t pre = 0, tot = 0;
+    for (int w = 0; w < 8; ++w) {
+      pre += wsum[16 + w];
+      tot += wsum[24 + w];
+    }
+    __syncthreads();
+    uint32_t carry = base + pre;
+    base += tot;
+    // next wave's words: loaded now, checked at the next lookup
+    if (k + 1 < K) e = threadIdx.x < S ? ld_relaxed_u64(word(k + 1, threadIdx.x)) : 0;
+    const uint64_t lo = lo_of(k), hi = hi_of(k);
+    const uint64_t nch = nch_of(k), nfull2 = nch_of(k + 2);
+    uint8_t* yb = reinterpret_cast<uint8_t*>(y + lo);
+    uint32_t s2 = 0;
+    for (uint64_t i = 0; i < nch; ++i) {
+      {                                                             // scan(k, i)
+        const int st = (int)(pos % kStreamStages);
+        const uint32_t ph = ((ph0 >> st) & 1u) ^ (uint32_t)((pos / kStreamStages) & 1);
+        if (threadIdx.x == 0) produce();
+        mbar_wait(&sbar[st], ph);
+        carry += scan_chunk_smem(reinterpret_cast<uint32_t*>(stage + st * kStreamChunk), carry,
+                                 wsum + 8 * (int)(pos & 1));
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncthreads();
+        if (threadIdx.x == 0) bulk_s2g_hint(yb + i * kStreamChunk, stage + st * kStreamChunk, kStreamChunk, pol);
+        ++pos;
+      }
+      if (i < nfull2) {                                             // sum(k+2, i)
+        const int st = (int)(pos % kStreamStages);
+        const uint32_t ph = ((ph0 >> st) & 1u) ^ (uint32_t)((pos / kStreamStages) & 1);
+        if (threadIdx.x == 0) produce();
+        mbar_wait(&sbar[st], ph);
+        const uint4* c4 = reinterpret_cast<const uint4*>(stage + st * kStreamChunk);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const uint4 q = c4[threadIdx.x + u * kThreads];
+          s2 += q.x + q.y + q.z + q.w;
+        }
+        ++pos;
+      }
+    }
+    if (k + 2 < K) {
+      const uint64_t lo2 = lo_of(k + 2);
+      s2 += sum_range(lo2 + (nch < nfull2 ? nch : nfull2) * kTile, hi_of(k + 2));
+      publish(k + 2, s2);
+    }
+    if (lo + nch * kTile < hi) scan_regs(x, y, lo + nch * kTile, hi, carry, true, wsum);
+  }
+  if (threadIdx.x == 0) {
+    *sphase = stage_phases_after(ph0, pos);
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+    __threadfence();
+    if (atomicAdd(&gs->scan_done, 1u) == (uint32_t)S - 1) {         // the item's last CTA: next tag
+      gs->scan_done = 0;
+      atomicAdd(&gs->scan_epoch, 1u);
+    }
+  }
+  __syncthreads();
 }
 
 // ------------------------------------------- SORT (Table I: SN, batch sort)

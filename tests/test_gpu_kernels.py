@@ -142,6 +142,50 @@ def test_scan_bit_exact(n, ctas):
     assert np.array_equal(y, K.scan(x))
 
 
+# The aligned SCAN body works in waves of about STRINGS_SCAN_WAVE_MB (16 MB) split
+# over the CTAs, with a wave's sums published two waves ahead: these sizes give
+# 3-5 waves (so the interleaved sum(k+2) path and the 8-row tag ring both run),
+# ragged last sub-blocks and CTAs with nothing in the last wave.
+@pytest.mark.parametrize("n,ctas", [(3 * (1 << 22) + 5, 1), ((1 << 24) + 9, 5), ((1 << 25) + 3, 37),
+                                    ((1 << 25) - 4, 148), (5 * (1 << 22), 1)])
+def test_scan_bit_exact_multi_wave(n, ctas):
+    x = np.random.default_rng(n).integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    (y,) = _launch(S.make_desc(S.SCAN, n=n), [x], [np.zeros(n, np.uint32)], ctas)
+    assert np.array_equal(y, K.scan(x))
+
+
+def test_scan_back_to_back_items_reuse_the_wave_table():
+    # consecutive launches on the same group state: each item's wave words carry
+    # a fresh tag, so a small item never reads a big item's stale words
+    torch = _torch()
+    st = torch.cuda.current_stream()
+    sizes = [(1 << 24) + 3, 100, 1 << 22, 8193, (1 << 24) + 3, 0, 5 * (1 << 22) + 1]
+    xs, ys = [], []
+    for i, n in enumerate(sizes):
+        x = np.random.default_rng(100 + i).integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+        dx = torch.from_numpy(x).cuda()
+        dy = torch.zeros(max(n, 1), dtype=torch.int32, device="cuda")
+        S.kernel_launch(0, S.make_desc(S.SCAN, n=n), [dx.data_ptr()], [dy.data_ptr()], ctas=5, stream=st.cuda_stream)
+        xs.append(x)
+        ys.append(dy)
+    torch.cuda.synchronize()
+    for x, dy in zip(xs, ys):
+        y = dy.cpu().numpy().view(np.uint32)[:x.size]
+        assert np.array_equal(y, K.scan(x))
+
+
+def test_scan_unaligned_buffers_take_the_two_pass_body():
+    torch = _torch()
+    n = 3 * (1 << 20) + 11
+    x = np.random.default_rng(5).integers(0, 1 << 32, n + 1, dtype=np.uint64).astype(np.uint32)
+    dx = torch.from_numpy(x).cuda()
+    dy = torch.zeros(n + 1, dtype=torch.int32, device="cuda")
+    S.kernel_launch(0, S.make_desc(S.SCAN, n=n), [dx.data_ptr() + 4], [dy.data_ptr() + 4], ctas=37,
+                    stream=torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    assert np.array_equal(dy.cpu().numpy().view(np.uint32)[1:], K.scan(x[1:]))
+
+
 @pytest.mark.parametrize("segs", [0, 1, 3, 150, 2048])
 @pytest.mark.parametrize("ctas", [0, 7])
 def test_sort_bit_exact(segs, ctas):

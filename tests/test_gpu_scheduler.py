@@ -146,6 +146,19 @@ def test_pairwise_mix_on_hardware(pair):
         check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("kl_mode", [0, 1])
+def test_multi_wave_scan_items_in_the_dispatcher(kl_mode):
+    # SCAN-XFER pair at full size: 2^24-element SCAN items span 4 waves on a KL
+    # partition (interleaved sums, tagged wave words, consecutive items per group)
+    wl = W.config_pair(7, balancer=W.MBF, instances=2, jobs_per_tenant=3, scale=1)
+    for timing in (S.INJECTED, S.MEASURED):
+        r = run_workload(wl, timing_mode=timing, kl_mode=kl_mode)
+        assert r.status == S.OK
+        if timing == S.INJECTED:
+            assert r.trace == run_oracle(wl).trace
+        check_outputs(wl, r)
+
+
 @pytest.mark.parametrize("seed", [3, 8, 21])
 def test_kl_launch_mode(seed):
     # kl_mode 1 (per-job launches of the same bodies, for profilers): same decisions in
