@@ -300,7 +300,8 @@ def kernel_rooflines(torch, S, peaks) -> list:
                     **({"note": "bitonic network, 66 compare-exchange stages per segment, 2 segments per CTA at once: "
                                 "ALU/shuffle bound; "
                                 "frac is of the HBM peak, for context"} if name == "SORT" else
-                       {"note": "reduce-then-scan: reads the input twice (12n bytes moved for 8n algorithmic)"})})
+                       {"note": "waves scanned from L2 with sums published two waves ahead: the input is read "
+                                "from HBM once (8n bytes; 1.05x in ncu)"})})
     del xs, ys
     torch.cuda.empty_cache()
     return out

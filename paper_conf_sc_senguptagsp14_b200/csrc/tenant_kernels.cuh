@@ -601,13 +601,21 @@ __device__ inline void hist_body(const uint8_t* __restrict__ x, uint32_t* __rest
 // ---------------------------------------------------- SCAN (Table I: SC)
 // y = inclusive prefix sum of x (u32, mod 2^32) over the whole group:
 // per-CTA chunk sums -> group barrier -> chunk offset -> tiled block scan.
+template <int O>
+__device__ __forceinline__ void shfl_up_add(uint32_t& v) {
+  asm("{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+      "shfl.sync.up.b32 t|p, %0, %1, 0, 0xffffffff;\n\t"
+      "@p add.u32 %0, %0, t;\n\t}"
+      : "+r"(v) : "n"(O));
+}
+// shfl.up's predicate output says whether the source lane exists: one SHFL and
+// one predicated add per step (the C form compiled to SHFL + SEL + IADD)
 __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
-  const int lane = threadIdx.x & 31;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t u = __shfl_up_sync(0xffffffffu, v, o);
-    if (lane >= o) v += u;
-  }
+  shfl_up_add<1>(v);
+  shfl_up_add<2>(v);
+  shfl_up_add<4>(v);
+  shfl_up_add<8>(v);
+  shfl_up_add<16>(v);
   return v;
 }
 
