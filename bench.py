@@ -65,7 +65,8 @@ def parse_args():
     p.add_argument("--partitions", type=int, default=0, help="P (0 = config default)")
     p.add_argument("--device-policy", type=int, default=-1, help="0 FIFO, 1 LAS, 2 PS (-1 = config)")
     p.add_argument("--balancer", type=int, default=-1, help="balancer id (-1 = config)")
-    p.add_argument("--config-repeats", type=int, default=3, help="timed runs per config in --configs")
+    p.add_argument("--config-repeats", type=int, default=5, help="timed runs per config and seed in --configs")
+    p.add_argument("--config-seeds", default="1", help="--configs: workload seeds, comma-separated (SURVEY: 1-5)")
     p.add_argument("--config-static", action="store_true", help="--configs: add static baselines")
     p.add_argument("--baseline-config-static", action="store_true",
                    help="N > 1: also time static provisioning on the BASELINE config")
@@ -859,7 +860,7 @@ def run_node(args, torch, gloo, world):
         name = {2: "C1", 4: "C3", 8: "C5"}.get(N)
         if name:
             # (its own static baselines only on request: at N = 8 they spawn 2 x 128 processes)
-            res["baseline_config"] = config_result(torch, name, phys, link, peaks, repeats=2,
+            res["baseline_config"] = config_result(torch, name, phys, link, peaks, repeats=2, warmups=1,
                                                    static=args.baseline_config_static and not args.no_static)
     return res, wl
 
@@ -967,6 +968,15 @@ def cpu_baseline(wl, threads: int = 0) -> dict:
     t = time.perf_counter()
     cbind.run_jobs(wl.jobs, ins, outs, threads)
     dt = time.perf_counter() - t
+    # one core (SURVEY §8(d) asks for both): one job of each class of the workload
+    # in submission order, on one worker
+    firsts = {}
+    for i, spec in enumerate(wl.jobs):
+        firsts.setdefault(spec.kclass, i)
+    pick = sorted(firsts.values())
+    t1 = time.perf_counter()
+    cbind.run_jobs([wl.jobs[i] for i in pick], [ins[i] for i in pick], [outs[i] for i in pick], 1)
+    dt1 = time.perf_counter() - t1
     t2 = time.perf_counter()
     o = run_oracle(wl)
     des = time.perf_counter() - t2
@@ -978,6 +988,9 @@ def cpu_baseline(wl, threads: int = 0) -> dict:
                       f"BLAS) with host copies in and out, {threads} worker threads ({busy} busy: tenants are "
                       f"dealt to workers, c_t = 1)",
             "seconds": round(dt, 3),
+            "one_core": {"value": round(len(pick) / dt1, 3), "unit": "jobs/s", "cores": 1,
+                         "sample": f"{len(pick)} jobs, the first of each class in the workload, one worker",
+                         "seconds": round(dt1, 3)},
             "des": {"seconds": round(des, 3), "decisions": decisions,
                     "decisions_per_s": round(decisions / des, 1) if des > 0 else None,
                     "note": "oracle/des.py (plain Python) on the same workload"}}
@@ -1156,18 +1169,19 @@ def copy_replay_s(torch, wl, streams_per_dir: int, reps: int = 2) -> float:
     return best
 
 
-def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, static: bool = False,
-                  replay: bool = False) -> dict:
+def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 5, static: bool = False,
+                  replay: bool = False, seed: int = 1, warmups: int = 2) -> dict:
     """One BASELINE configuration at full size, MEASURED timing, node mode (one
-    process, G logical devices mapped round-robin onto `ngpu` GPUs).  One
-    untimed warm-up run, then `repeats` timed runs; the median jobs/s and span,
+    process, G logical devices mapped round-robin onto `ngpu` GPUs), workload
+    seed `seed`.  `warmups` untimed runs, then `repeats` timed runs (SURVEY
+    §8(d): 2 warm-up, 5 timed per seed); the median jobs/s and span,
     the overlapped roofline T*/span per physical GPU over the jobs placed there
     (SURVEY §8(d)), Jain per R-2 (alone runs), optionally static provisioning
     (tenant mod GPUs, and device 0) and the plain-copy replay."""
     import strings_workload as W
     from paper_conf_sc_senguptagsp14_b200 import strings as S
 
-    wl = W.CONFIGS[name]()
+    wl = W.CONFIGS[name](seed=seed)
     if os.environ.get("BENCH_AWAKE_BUDGET"):       # experiments: override A (M follows unless set)
         wl.config.awake_budget = int(os.environ["BENCH_AWAKE_BUDGET"])
     if os.environ.get("BENCH_ADMIT_CAP"):
@@ -1178,7 +1192,7 @@ def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, st
     lpg = max(1, -(-cfg.num_gpus // ngpu))       # logical devices per GPU
     ins_of, outs_of, bufs = tenant_buffers(torch, wl)
     runs = []
-    for rep in range(1 + repeats):
+    for rep in range(warmups + repeats):
         S.init_from_config(cfg, timing_mode=S.MEASURED, physical_gpus=ngpu, trace_in_memory=False)
         ts = [S.register_tenant(t.weight, t.max_inflight) for t in wl.tenants]
         t0 = time.perf_counter()
@@ -1188,7 +1202,7 @@ def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, st
         infos = [S.job_info(i) for i in ids]
         stats = S.stats()
         S.shutdown()
-        if rep == 0:
+        if rep < warmups:
             continue                    # warm-up
         span = (max(i.t_done[2] for i in infos) - min(i.t_arrival for i in infos)) / 1e9
         runs.append({"span": span, "wall": wall, "status": st, "infos": infos, "sm_copy_ops": stats.sm_copy_ops,
@@ -1204,7 +1218,7 @@ def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, st
     shared = mean_latency_by_tenant(mid["infos"])
     alone = alone_mean_latency(S, wl, ins_of, outs_of)
     jain, _ = jain_r2(wl, shared, alone)
-    out = {"config": name, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
+    out = {"config": name, "seed": seed, "jobs": len(wl.jobs), "tenants": len(wl.tenants),
            "logical_gpus": cfg.num_gpus, "physical_gpus": ngpu,
            "balancer": W.BALANCER_NAMES[cfg.balancer], "las_admission": cfg.las_admission,
            "device_policy": W.DEVICE_POLICY_NAMES[cfg.device_policy],
@@ -1213,7 +1227,7 @@ def config_result(torch, name: str, ngpu: int, link, peaks, repeats: int = 3, st
            "jobs_per_s": round(len(wl.jobs) / span, 1),
            "span_ms": round(span * 1e3, 2), "span_ms_min_max": [round(runs[0]["span"] * 1e3, 2),
                                                              round(runs[-1]["span"] * 1e3, 2)],
-           "runs": len(runs), "sm_copy_ops": mid["sm_copy_ops"],
+           "runs": len(runs), "warmup_runs": warmups, "sm_copy_ops": mid["sm_copy_ops"],
            "tstar_ms": round(tstar * 1e3, 3) if ngpu == 1 else None,
            "roofline_frac": round(tstar / span, 4) if ngpu == 1 else None,
            "tstar_terms_ms": {k: round(v * 1e3, 3) for k, v in terms.items()} if ngpu == 1 else None,
@@ -1254,8 +1268,9 @@ def run_configs(args) -> None:
     link1 = host_link_peaks(torch)
     link = scaled_link(link1, host_link_concurrent(torch, ngpu)) if ngpu > 1 else link1
     for name in os.environ.get("BENCH_CONFIGS", "C1,C2,C3,C4,C5").split(","):
-        print(json.dumps(config_result(torch, name, ngpu, link, peaks, repeats=args.config_repeats,
-                                       static=args.config_static, replay=True)), flush=True)
+        for seed in (int(x) for x in args.config_seeds.split(",")):
+            print(json.dumps(config_result(torch, name, ngpu, link, peaks, repeats=args.config_repeats,
+                                           static=args.config_static, replay=True, seed=seed)), flush=True)
 
 
 def _pct(xs, q):
