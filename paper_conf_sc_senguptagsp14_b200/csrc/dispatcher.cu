@@ -291,7 +291,7 @@ __global__ void __launch_bounds__(kThreads, 1) oneshot_kernel(const __grid_const
                    it.alpha, it.seed, rank, S, sm.stage, sm.sbar, sm.scratch, sm.sphase, gs, nullptr);
   } else if constexpr (KC == 3) {
     hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
-              sm.stage);
+              sm.stage, sm.sbar, sm.sphase);
   } else if constexpr (KC == 4) {
     scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
               sm.stage, sm.sbar, sm.scratch, sm.sphase);

@@ -566,35 +566,108 @@ __device__ __forceinline__ void group_barrier(GroupSync* gs, int S) {
 }
 
 // ---------------------------------------------------- HIST (Table I: HI)
-// bins[256] (u32) = byte histogram of x[n].  Per-warp shared-memory
-// sub-histograms (smem atomics), merged per CTA, then one global atomicAdd per
-// non-zero bin; rank 0 zeroes the output before the group barrier.
+// bins[256] (u32) = byte histogram of x[n].  Counting is bound by the SM's
+// shared-memory atomic rate, not by HBM (one ATOMS per byte;
+// tools/hist_probe.cu, profiles/r02_hist.md).  Counters are lane-private,
+// [bin][lane] u32, so a warp's 32 atomics hit 32 different banks whatever
+// the bytes are, and there are two copies (even / odd warps) so fewer warps
+// contend for one word; each copy is 32 KB at the front of the stage area.
+// Whole 32 KB chunks stream through a 4-stage TMA bulk pipeline (chunks dealt
+// statically, chunk c to rank c mod S) once there is at least
+// kHistBulkMinChunks per CTA; the rest (the tail, or buffers too small for
+// one chunk per CTA) use 16-B LDGs, 8 in flight per thread, and unaligned
+// buffers byte loads.  From cold L2 the pipeline wins at every size measured
+// (2^26 bytes on 148 / 72 CTAs: 0.40 / 0.25 of the HBM peak vs 0.31 / 0.21
+// with LDGs; tools/hist_ab.sh).  Then each
+// thread sums one bin over both copies and the 32 lanes, rank 0 zeroes the
+// output before the group barrier, and one global atomicAdd per non-zero bin.
+constexpr int kHistCopies = 2;
+constexpr uint32_t kHistCounterBytes = kHistCopies * 256 * 32 * 4;      // 64 KB
+constexpr int kHistStages = 4;
+constexpr uint32_t kHistChunk = 32768;
+#ifndef STRINGS_HIST_BULK_MIN_CHUNKS
+#define STRINGS_HIST_BULK_MIN_CHUNKS 1
+#endif
+constexpr uint64_t kHistBulkMinChunks = STRINGS_HIST_BULK_MIN_CHUNKS;
+static_assert(kHistCounterBytes + kHistStages * kHistChunk <= kSmemMain, "HIST smem");
+static_assert(kHistStages <= kStreamStages, "HIST uses the first stage barriers");
+
+__device__ __forceinline__ void hist_word(uint32_t* mine, uint32_t w) {
+#pragma unroll
+  for (int b = 0; b < 4; ++b) atomicAdd(&mine[((w >> (8 * b)) & 0xFF) * 32], 1u);
+}
+__device__ __forceinline__ void hist_vec(uint32_t* mine, uint4 q) {
+  hist_word(mine, q.x);
+  hist_word(mine, q.y);
+  hist_word(mine, q.z);
+  hist_word(mine, q.w);
+}
+
 __device__ inline void hist_body(const uint8_t* __restrict__ x, uint32_t* __restrict__ bins, uint64_t n,
-                                 int rank, int S, GroupSync* gs, uint8_t* stage) {
-  uint32_t* sh = reinterpret_cast<uint32_t*>(stage);            // [8 warps][256]
-  const int warp = threadIdx.x >> 5;
-  for (int i = threadIdx.x; i < 8 * 256; i += kThreads) sh[i] = 0;
+                                 int rank, int S, GroupSync* gs, uint8_t* stage, uint64_t* sbar, uint32_t* sphase) {
+  uint32_t* sh = reinterpret_cast<uint32_t*>(stage);            // [kHistCopies][256 bins][32 lanes]
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < (int)(kHistCounterBytes / 16); i += kThreads)
+    reinterpret_cast<uint4*>(sh)[i] = make_uint4(0, 0, 0, 0);
   if (rank == 0)
     for (int i = threadIdx.x; i < 256; i += kThreads) bins[i] = 0;
   __syncthreads();
-  uint32_t* mine = sh + warp * 256;
-  const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x, nt = (uint64_t)S * kThreads;
+  uint32_t* mine = sh + (warp % kHistCopies) * (256 * 32) + lane;
   const bool aligned = (reinterpret_cast<uintptr_t>(x) & 15) == 0;
-  const uint64_t nv = aligned ? n / 16 : 0;
-  const uint4* x4 = reinterpret_cast<const uint4*>(x);
-  for (uint64_t v = tid; v < nv; v += nt) {
-    const uint4 q = ld_stream(x4 + v);
-    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-    for (int a = 0; a < 4; ++a)
-#pragma unroll
-      for (int b = 0; b < 4; ++b) atomicAdd(&mine[(w[a] >> (8 * b)) & 0xFF], 1u);
+  const uint64_t nch = aligned ? n / kHistChunk : 0;
+  const uint64_t my_ch = nch > (uint64_t)rank ? (nch - 1 - rank) / S + 1 : 0;
+  uint64_t done_bytes = 0;                                      // bytes [0, done_bytes) counted by the bulk path
+  if (nch >= (uint64_t)S * kHistBulkMinChunks) {
+    uint8_t* st = stage + kHistCounterBytes;
+    const uint32_t ph0 = *reinterpret_cast<volatile uint32_t*>(sphase);
+    if (threadIdx.x == 0)
+      for (int s = 0; s < kHistStages && (uint64_t)s < my_ch; ++s) {
+        mbar_expect_tx(&sbar[s], kHistChunk);
+        bulk_g2s(st + s * kHistChunk, x + (rank + (uint64_t)s * S) * kHistChunk, kHistChunk, &sbar[s]);
+      }
+    for (uint64_t i = 0; i < my_ch; ++i) {
+      const int s = (int)(i % kHistStages);
+      mbar_wait(&sbar[s], ((ph0 >> s) & 1u) ^ (uint32_t)((i / kHistStages) & 1));
+      const uint4* b4 = reinterpret_cast<const uint4*>(st + s * kHistChunk);
+#pragma unroll 4
+      for (int j = threadIdx.x; j < (int)(kHistChunk / 16); j += kThreads) hist_vec(mine, b4[j]);
+      __syncthreads();                                          // stage s read by every thread
+      if (threadIdx.x == 0 && i + kHistStages < my_ch) {
+        mbar_expect_tx(&sbar[s], kHistChunk);
+        bulk_g2s(st + s * kHistChunk, x + (rank + (i + kHistStages) * S) * kHistChunk, kHistChunk, &sbar[s]);
+      }
+    }
+    if (threadIdx.x == 0) {                                     // barrier s completed ceil((my_ch - s) / 4) phases
+      uint32_t bits = ph0;
+      for (int s = 0; s < kHistStages; ++s) {
+        const uint64_t uses = my_ch > (uint64_t)s ? (my_ch - 1 - s) / kHistStages + 1 : 0;
+        bits ^= (uint32_t)(uses & 1) << s;
+      }
+      *sphase = bits;
+    }
+    done_bytes = nch * kHistChunk;
   }
-  for (uint64_t e = nv * 16 + tid; e < n; e += nt) atomicAdd(&mine[x[e]], 1u);
+  // LDG path over [done_bytes, n): 16-B vectors (8 in flight per thread), then bytes
+  const uint64_t tid = (uint64_t)rank * kThreads + threadIdx.x, nt = (uint64_t)S * kThreads;
+  const uint64_t nv = aligned ? (n - done_bytes) / 16 : 0;
+  const uint4* x4 = reinterpret_cast<const uint4*>(x + done_bytes);
+  constexpr int U = 8;
+  uint64_t v = tid;
+  for (; v + (U - 1) * nt < nv; v += U * nt) {
+    uint4 q[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) q[u] = ld_stream(x4 + v + u * nt);
+#pragma unroll
+    for (int u = 0; u < U; ++u) hist_vec(mine, q[u]);
+  }
+  for (; v < nv; v += nt) hist_vec(mine, ld_stream(x4 + v));
+  for (uint64_t e = done_bytes + nv * 16 + tid; e < n; e += nt) atomicAdd(&mine[(uint32_t)x[e] * 32], 1u);
   __syncthreads();
-  uint32_t total = 0;                                              // thread t owns bin t
-  for (int w = 0; w < 8; ++w) total += sh[w * 256 + threadIdx.x];
-  group_barrier(gs, S);                                            // output zeroed by rank 0
+  uint32_t total = 0;                                           // thread t owns bin t
+#pragma unroll
+  for (int c = 0; c < kHistCopies; ++c)
+    for (int l = 0; l < 32; ++l) total += sh[c * (256 * 32) + threadIdx.x * 32 + ((l + threadIdx.x) & 31)];
+  group_barrier(gs, S);                                         // output zeroed by rank 0
   if (total) atomicAdd(&bins[threadIdx.x], total);
 }
 
@@ -1213,7 +1286,7 @@ __device__ __forceinline__ void run_item(const KlItem& it, const KlItem* tmaps, 
   switch (it.kclass) {
     case 3:
       hist_body(reinterpret_cast<const uint8_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S, gs,
-                sm.stage);
+                sm.stage, sm.sbar, sm.sphase);
       break;
     case 4:
       scan_body(reinterpret_cast<const uint32_t*>(it.in0), reinterpret_cast<uint32_t*>(it.out0), it.n, rank, S,

@@ -124,14 +124,33 @@ def test_hist_single_bin_contention():
 
 
 @pytest.mark.parametrize("ctas", [1, 3])
-def test_hist_counter_flush_one_bin(ctas):
-    # one CTA sees > 65535 copies of one byte per lane: the 16-bit lane counters
-    # must be flushed before they wrap (every 4095 16-B loads)
+def test_hist_one_bin_large_share(ctas):
+    # one CTA counts > 2^24 copies of one byte (per-lane counters far past 16 bits)
+    # through the bulk pipeline, plus a ragged tail on the LDG / byte paths
     n = (1 << 24) * 2 // ctas + 77
     x = np.full(n, 200, np.uint8)
     x[::4097] = 3
     (h,) = _launch(S.make_desc(S.HIST, n=n), [x], [np.zeros(256, np.uint32)], ctas)
     assert np.array_equal(h, K.hist(x))
+
+
+@pytest.mark.parametrize("ctas", [2, 37])
+@pytest.mark.parametrize("offset", [0, 3])
+def test_hist_bulk_path(ctas, offset):
+    # 41 whole 32 KB chunks per CTA through the TMA bulk pipeline (chunks dealt
+    # round-robin over the CTAs, 4 stages cycling several times); 4099 tail bytes
+    # go through the 16-B and byte loads.  offset 3: the same bytes from an
+    # unaligned start (byte loads only)
+    torch = _torch()
+    n = ctas * 41 * 32768 + 4099
+    spec = W.JobSpec(tenant=0, kclass=W.HIST, n=n + offset, data_seed=ctas + offset)
+    (x,) = W.job_inputs(spec)
+    dx = torch.from_numpy(x).cuda()
+    out = torch.zeros(256, dtype=torch.int32, device="cuda")
+    S.kernel_launch(0, S.make_desc(S.HIST, n=n), [dx.data_ptr() + offset], [out.data_ptr()], ctas=ctas,
+                    stream=torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), K.hist(x[offset:]))
 
 
 @pytest.mark.parametrize("n", [0, 1, 7, 8, 2047, 2049, 100_003, (1 << 22) + 5])

@@ -159,6 +159,23 @@ def test_multi_wave_scan_items_in_the_dispatcher(kl_mode):
         check_outputs(wl, r)
 
 
+def test_bulk_hist_items_between_streaming_items():
+    # HIST-XFER pair with 2^27 + 4099-byte HIST items (57 chunks per CTA of a KL
+    # partition): HIST's TMA bulk pipeline uses the first 4 stage barriers
+    # while XFER items use all 6 on the same CTAs; the barriers' phase parities carry
+    # from item to item (a wrong parity hangs or reads a stale stage)
+    import dataclasses
+    wl = W.config_pair(4, balancer=W.MBF, instances=2, jobs_per_tenant=3, scale=1)
+    wl.jobs = [W.with_nominal_durations(dataclasses.replace(j, n=(1 << 27) + 4099)) if j.kclass == W.HIST else j
+               for j in wl.jobs]
+    for timing in (S.INJECTED, S.MEASURED):
+        r = run_workload(wl, timing_mode=timing)
+        assert r.status == S.OK
+        if timing == S.INJECTED:
+            assert r.trace == run_oracle(wl).trace
+        check_outputs(wl, r)
+
+
 @pytest.mark.parametrize("seed", [3, 8, 21])
 def test_kl_launch_mode(seed):
     # kl_mode 1 (per-job launches of the same bodies, for profilers): same decisions in

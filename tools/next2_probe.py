@@ -21,13 +21,15 @@ def main():
     peaks = bench.measured_peaks()
     st = torch.cuda.current_stream()
 
-    def timed(desc, ins, outs, iters=10):
-        S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], stream=st.cuda_stream)
+    def timed(desc, ins, outs, iters=10, ctas=0):
+        S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], ctas=ctas,
+                        stream=st.cuda_stream)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(st)
         for _ in range(iters):
-            S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], stream=st.cuda_stream)
+            S.kernel_launch(0, desc, [a.data_ptr() for a in ins], [a.data_ptr() for a in outs], ctas=ctas,
+                            stream=st.cuda_stream)
         e1.record(st)
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / 1e3 / iters
@@ -38,6 +40,16 @@ def main():
     t = timed(S.make_desc(S.HIST, n=n), [x], [h])
     rows = [("HIST", n + 1024, t, f"n=2^30 bytes")]
     del x
+    # the pairwise mix's HIST job (2^26 image-like bytes) on all SMs and on one 72-SM KL
+    # slot; 8 rotating inputs (512 MiB > L2)
+    import strings_workload as W
+    xs = [torch.from_numpy(W.job_inputs(W.JobSpec(tenant=0, kclass=W.HIST, n=1 << 26, data_seed=s))[0]).cuda()
+          for s in range(8)]
+    for ctas in (0, 72):
+        ts = [timed(S.make_desc(S.HIST, n=1 << 26), [xs[i]], [h], iters=4, ctas=ctas) for i in range(8)]
+        rows.append(("HIST", (1 << 26) + 1024, sum(ts) / len(ts), f"n=2^26 image-like bytes, {ctas or 'all'} CTAs"))
+    assert torch.equal(h.long(), torch.bincount(xs[7].long(), minlength=256))
+    del xs
     n = 1 << 28
     x = torch.randint(0, 1 << 20, (n,), dtype=torch.int32, device="cuda")
     y = torch.empty_like(x)
