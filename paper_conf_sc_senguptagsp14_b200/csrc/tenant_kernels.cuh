@@ -1175,9 +1175,17 @@ __device__ inline void scan_body(const uint32_t* __restrict__ x, uint32_t* __res
 // keeps keys [8t, 8t + 8) of the segment in registers for the whole network:
 // compare-exchange distance j < 8 is inside the thread, 8 <= j < 256 between
 // lanes of one warp (shuffles), and only j >= 256 (6 of the 66 stages) goes
-// through shared memory (padded one word per 32: conflict-free).  The element
-// at index a with partner a ^ j keeps min(v, p) when it is the lower index of
-// an ascending block ((a & k) == 0) or the higher index of a descending one.
+// through shared memory (padded one word per 32: conflict-free).
+// The body is bound by the integer ALU pipe, so each compare-exchange costs one
+// min/max per key.  In merge phase k >= 8 the keys of a descending block (index
+// bit k set: bit k - 3 of t, the same for the thread's 8 keys) are held
+// complemented; ~ reverses unsigned order, so every compare-exchange of the
+// phase is ascending in the held form: in-thread the lower register takes the
+// min and the higher the max (no direction select), across lanes or warps the
+// lower index takes min(v, p) and the higher max(v, p) (one predicated VIMNMX).
+// Between phases one XOR per key moves to the next phase's form; phase 2048
+// has no descending block, so the keys end uncomplemented.  Phases 2 and 4
+// (k < 8) run on the plain keys with compile-time directions.
 constexpr int kSortSeg = 2048;
 constexpr int kSortPar = 2;                                       // segments sorted at once per CTA (ILP)
 __device__ __forceinline__ int sort_pad(int a) { return a + (a >> 5); }
@@ -1188,7 +1196,7 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
   constexpr int kPadSeg = kSortSeg + kSortSeg / 32;
   uint32_t* key = reinterpret_cast<uint32_t*>(stage);            // [kSortPar][2048 + 64] padded
   const uint64_t nseg = n / kSortSeg;
-  const int t = threadIdx.x;
+  const uint32_t t = threadIdx.x;
   const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
   auto load8 = [&](uint64_t seg, uint32_t* w) {
     if (seg >= nseg) return;                                      // idle lane of the pair: garbage, never stored
@@ -1218,10 +1226,20 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
 #pragma unroll
     for (int lk = 1; lk <= 11; ++lk) {
       const int k = 1 << lk;
+      if (lk >= 3) {                                               // complement for phase k (held form)
+        const uint32_t now = lk < 11 ? (t >> (lk - 3)) & 1u : 0u;  // index bit k
+        const uint32_t before = lk > 3 ? (t >> (lk - 4)) & 1u : 0u;
+        const uint32_t m = 0u - (now ^ before);
+#pragma unroll
+        for (int h = 0; h < kSortPar; ++h)
+#pragma unroll
+          for (int r = 0; r < 8; ++r) v[h][r] ^= m;
+      }
 #pragma unroll
       for (int lj = lk - 1; lj >= 0; --lj) {
         const int j = 1 << lj;
-        if (j >= 256) {                                              // across warps
+        if (j >= 256) {                                              // across warps (k >= 512: held form)
+          const bool lower = (t & (uint32_t)(j >> 3)) == 0;
 #pragma unroll
           for (int h = 0; h < kSortPar; ++h)
 #pragma unroll
@@ -1231,19 +1249,18 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
           for (int h = 0; h < kSortPar; ++h)
 #pragma unroll
             for (int r = 0; r < 8; ++r) {
-              const int a = 8 * t + r;
-              const uint32_t p = key[h * kPadSeg + sort_pad(a ^ j)];
-              v[h][r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[h][r], p) : max(v[h][r], p);
+              const uint32_t p = key[h * kPadSeg + sort_pad((8 * t + r) ^ j)];
+              v[h][r] = lower ? min(v[h][r], p) : max(v[h][r], p);
             }
           __syncthreads();
-        } else if (j >= 8) {                                         // lanes t and t ^ (j / 8)
+        } else if (j >= 8) {                                         // lanes t and t ^ (j / 8) (k >= 16: held form)
+          const bool lower = (t & (uint32_t)(j >> 3)) == 0;
 #pragma unroll
           for (int h = 0; h < kSortPar; ++h)
 #pragma unroll
             for (int r = 0; r < 8; ++r) {
-              const int a = 8 * t + r;
               const uint32_t p = __shfl_xor_sync(0xffffffffu, v[h][r], j >> 3);
-              v[h][r] = (((a & k) == 0) == ((a & j) == 0)) ? min(v[h][r], p) : max(v[h][r], p);
+              v[h][r] = lower ? min(v[h][r], p) : max(v[h][r], p);
             }
         } else {                                                     // registers r and r + j
 #pragma unroll
@@ -1251,7 +1268,8 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
 #pragma unroll
             for (int r = 0; r < 8; ++r) {
               if (r & j) continue;
-              const bool asc = ((8 * t + r) & k) == 0;
+              // k >= 8: held form, ascending; k < 8: plain keys, direction from r
+              const bool asc = k >= 8 || (r & k) == 0;
               const uint32_t lo = v[h][r], hi = v[h][r + j];
               v[h][r] = asc ? min(lo, hi) : max(lo, hi);
               v[h][r + j] = asc ? max(lo, hi) : min(lo, hi);
