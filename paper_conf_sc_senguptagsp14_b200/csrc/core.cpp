@@ -273,6 +273,19 @@ void Core::admission(uint64_t t) {
   std::vector<Job*>& elig = scratch_elig_;
   std::vector<int>& adm = scratch_adm_;
   std::vector<Agg>& aggs = scratch_aggs_;
+  // Cheap exits first: most calls (a completion that freed no resident slot
+  // the pending jobs can use) find no device with room or no eligible job.
+  adm.clear();
+  for (auto& d : devs_)
+    if ((int)d.resident.size() < cfg_.M) adm.push_back(d.gid);
+  if (adm.empty()) return;
+  // Eligible jobs: each tenant's oldest pending job while the tenant is below c_t.
+  // Built once per call; a placement changes only the placed job's tenant.
+  elig.clear();
+  for (auto& tn : tenants_)
+    if (!tn.pending.empty() && tn.inflight < tn.c && tn.pending.front()->arrived)
+      elig.push_back(tn.pending.front());
+  if (elig.empty()) return;
   aggs.resize(devs_.size());
   const bool need_aggs = cfg_.balancer != B_GRR && cfg_.balancer != B_GMIN && cfg_.balancer != B_GWTMIN;
   // Aggregates depend only on the resident jobs' phases and the SFT, neither of
@@ -284,15 +297,6 @@ void Core::admission(uint64_t t) {
     else aggs[d.gid].n = d.resident.size();
   }
   for (;;) {
-    elig.clear();
-    adm.clear();
-    for (auto& d : devs_)
-      if ((int)d.resident.size() < cfg_.M) adm.push_back(d.gid);
-    if (adm.empty()) return;
-    for (auto& tn : tenants_)
-      if (!tn.pending.empty() && tn.inflight < tn.c && tn.pending.front()->arrived)
-        elig.push_back(tn.pending.front());
-    if (elig.empty()) return;
     Job* pick = nullptr;
     int gid = -1, pol = B_GMIN;
     uint64_t sc = 0;
@@ -327,6 +331,21 @@ void Core::admission(uint64_t t) {
     place(t, pick, gid, pol, sc);
     if (need_aggs) aggs[gid] = aggregate(devs_[gid]);
     else aggs[gid].n = devs_[gid].resident.size();
+    if ((int)devs_[gid].resident.size() >= cfg_.M) {
+      adm.erase(std::find(adm.begin(), adm.end(), gid));
+      if (adm.empty()) return;
+    }
+    // the placed job's tenant: its next pending job replaces it if the tenant
+    // is still below c_t (elig keeps no particular order: every scan is a min)
+    Tenant& tn = tenants_[pick->tenant];
+    auto pos = std::find(elig.begin(), elig.end(), pick);
+    if (!tn.pending.empty() && tn.inflight < tn.c && tn.pending.front()->arrived) {
+      *pos = tn.pending.front();
+    } else {
+      *pos = elig.back();
+      elig.pop_back();
+      if (elig.empty()) return;
+    }
   }
 }
 
