@@ -155,14 +155,28 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
           uint32_t total = (uint32_t)S;
           if (sib >= 0 && (kc == 0 || kc == 2) && atomicCAS(&sps->lock, 0u, (uint32_t)q + 1) == 0u) {
             total += (uint32_t)S_sib;
-            st_release_gpu_u64(&sps->help, (uint64_t)(kHelpGen | ((uint32_t)q << 16) | slot) << 32);
+            const uint64_t hw = (uint64_t)(kHelpGen | ((uint32_t)q << 16) | slot) << 32;
+            st_release_gpu_u64(&sps->help, hw);
+            // Start the sibling's CTAs at once rather than through its leader's
+            // back-off poll of `help` (item 24.0 -> 23.7 us on C2, tools/item_ab.sh):
+            // only when the sibling is fully idle -- its last item's done_gen
+            // published (its completion step reads its gen word, and it releases the
+            // lock before done_gen) -- which stays so while we hold its lock.  Its
+            // leader, on seeing `help`, writes the same gen word again.
+            const uint64_t sg = ld_acquire_gpu_u64(&sps->gen);
+            if ((uint32_t)sg != kStop && ld_acquire_gpu(&sps->done_gen) == (uint32_t)sg)
+              st_release_gpu_u64(&sps->gen, hw | (uint32_t)((uint32_t)sg + 1));
           }
           st_release_gpu(&ps->total, total);
         }
       }
       uint64_t gw = 0;
       if (lane == 0)                              // one poller per CTA
-        while ((uint32_t)(gw = ld_acquire_gpu_u64(&ps->gen)) == seen) __nanosleep(32);
+        while ((uint32_t)(gw = ld_acquire_gpu_u64(&ps->gen)) == seen) {
+#ifndef STRINGS_GEN_SPIN
+          __nanosleep(32);
+#endif
+        }
       __syncwarp();                               // orders lane 0's acquire before the item loads
       gw = __shfl_sync(0xffffffffu, gw, 0);
       const uint32_t g = (uint32_t)gw, slot_word = (uint32_t)(gw >> 32);
@@ -196,7 +210,12 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
     PartState* ops = p.parts + s_owner;          // the partition whose item this is
     // the owner partition's CTAs come first in the item's rank order
     const int S_owner = lent ? p.part_start[s_owner + 1] - p.part_start[s_owner] : S;
+#ifdef STRINGS_TEXEC_FIRST
+    // experiment: t_exec = the FIRST CTA (own or lent) to start the body
+    if (!cpart && threadIdx.x == 0) atomicMin(reinterpret_cast<unsigned long long*>(&ops->t_exec), globaltimer());
+#else
     if (!lent && rank == 0 && threadIdx.x == 0) ps->t_exec = globaltimer();
+#endif
     if (cpart) {
       copy_body(s_citem, rank, S);
     } else {
@@ -233,6 +252,9 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
         d->partition = s_owner;
         d->t_start = ops->t_start;
         d->t_exec = ops->t_exec;
+#ifdef STRINGS_TEXEC_FIRST
+        ops->t_exec = ~0ull;
+#endif
         d->t_end = globaltimer();
         // Every CTA fenced its output writes at gpu scope before counting in, so the
         // outputs are in L2/HBM; the host reacts to this word only by issuing a D2H
