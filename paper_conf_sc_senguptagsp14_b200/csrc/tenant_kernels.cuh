@@ -173,6 +173,10 @@ constexpr uint32_t kStreamChunk = STRINGS_STREAM_CHUNK_KB * 1024;    // bytes pe
 #ifndef STRINGS_STREAM_MIN_CHUNKS
 #define STRINGS_STREAM_MIN_CHUNKS 0
 #endif
+#ifndef STRINGS_STREAM_TAIL_SPLIT
+#define STRINGS_STREAM_TAIL_SPLIT 1
+#endif
+constexpr int kStreamTailSplit = STRINGS_STREAM_TAIL_SPLIT;
 constexpr int kStreamLead = STRINGS_STREAM_LEAD;
 constexpr int kStreamMinChunks = STRINGS_STREAM_MIN_CHUNKS;
 constexpr int kStreamStoreSlack = kStreamStages - kStreamLead - 1;
@@ -249,7 +253,16 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
     // it takes counter chunks only.
     const int d0 = total_word ? 1 : 0;            // first dealt rank
     const int D = S - d0;                         // dealt ranks
-    const uint64_t dealt = D <= 0 ? 0 : (nchunks < (uint64_t)kStreamLead * D ? nchunks : (uint64_t)kStreamLead * D);
+    // The last `split` whole chunks are handed out as half chunks, so the CTAs
+    // (own and lent) run out of work closer together at the item's end.  Units
+    // [0, nfull) are whole chunks, [nfull, nunits) halves of the rest.
+    const uint64_t split = kStreamTailSplit ? (nchunks / 4 < 2ull * S ? nchunks / 4 : 2ull * S) : 0;
+    const uint64_t nfull = nchunks - split, nunits = nfull + 2 * split;
+    auto unit_off = [&](uint32_t u) -> uint64_t {
+      return u < nfull ? (uint64_t)u * kStreamChunk : nfull * kStreamChunk + (u - nfull) * (uint64_t)(kStreamChunk / 2);
+    };
+    auto unit_bytes = [&](uint32_t u) -> uint32_t { return u < nfull ? kStreamChunk : kStreamChunk / 2; };
+    const uint64_t dealt = D <= 0 ? 0 : (nunits < (uint64_t)kStreamLead * D ? nunits : (uint64_t)kStreamLead * D);
     int pre = 0;                                  // thread 0: statically dealt chunks used so far
     auto claim = [&]() -> uint32_t {
       if (rank >= d0 && rank < S && pre < kStreamLead) {
@@ -258,7 +271,7 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
         pre = kStreamLead;                        // this CTA's static share is used up
       }
       const uint64_t c = dealt + atomicAdd(&gs->chunk_next, 1u);
-      return c < nchunks ? (uint32_t)c : kNoChunk;
+      return c < nunits ? (uint32_t)c : kNoChunk;
     };
     // thread 0: fill stage st with the chunk claimed earlier (or end the CTA's loop there)
     auto issue = [&](int st) {
@@ -269,8 +282,8 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
         asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(&sbar[st])) : "memory");
         return;
       }
-      mbar_expect_tx(&sbar[st], kStreamChunk);
-      bulk_g2s(stage + st * kStreamChunk, xb + (uint64_t)c * kStreamChunk, kStreamChunk, &sbar[st]);
+      mbar_expect_tx(&sbar[st], unit_bytes(c));
+      bulk_g2s(stage + st * kStreamChunk, xb + unit_off(c), unit_bytes(c), &sbar[st]);
       next = claim();                             // consumed at the next issue
     };
     // the stage barriers live for the whole kernel (mbar_setup); their phase
@@ -297,8 +310,9 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       const uint32_t c = *reinterpret_cast<volatile uint32_t*>(&cid[st]);
       if (c == kNoChunk) break;                   // every thread sees the same end stage
       uint4* buf = reinterpret_cast<uint4*>(stage + st * kStreamChunk);
+      const int nv = (int)(unit_bytes(c) / 16);
 #pragma unroll 4
-      for (int j = threadIdx.x; j < (int)(kStreamChunk / 16); j += kThreads) {
+      for (int j = threadIdx.x; j < nv; j += kThreads) {
         uint4 v = buf[j];
         v.x = elem_op<KCLASS>(v.x, alpha, seed);
         v.y = elem_op<KCLASS>(v.y, alpha, seed);
@@ -308,7 +322,7 @@ __device__ void stream_body(const uint32_t* __restrict__ x, uint32_t* __restrict
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // smem writes -> async proxy
       __syncthreads();
-      if (threadIdx.x == 0) bulk_s2g(yb + (uint64_t)c * kStreamChunk, stage + st * kStreamChunk, kStreamChunk);
+      if (threadIdx.x == 0) bulk_s2g(yb + unit_off(c), stage + st * kStreamChunk, unit_bytes(c));
     }
     if (threadIdx.x == 0) {
       *sphase = stage_phases_after(ph0, i + 1);   // positions 0..i (the end marker's included) used a phase
