@@ -1204,7 +1204,7 @@ constexpr int kSortSeg = 2048;
 constexpr int kSortPar = 2;                                       // segments sorted at once per CTA (ILP)
 __device__ __forceinline__ int sort_pad(int a) { return a + (a >> 5); }
 
-__device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
+__device__ inline void sort_body8(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
                                  int S, uint8_t* stage) {
   static_assert(kSortSeg == 8 * kThreads, "8 keys per thread");
   constexpr int kPadSeg = kSortSeg + kSortSeg / 32;
@@ -1304,6 +1304,134 @@ __device__ inline void sort_body(const uint32_t* __restrict__ x, uint32_t* __res
       }
     }
   }
+}
+
+// 32 keys per thread (64 threads = one segment, four segments per CTA at once):
+// index a = 32t + r, so 45 of the 66 stages are inside the thread (one VIMNMX
+// per key), 20 go across lanes and only j = 1024 through shared memory between
+// the group's two warps.  Held-complement form from phase 32 (bit 5 = t bit 0).
+constexpr int kSortKPT = 32;
+constexpr int kSortTPS = kSortSeg / kSortKPT;                     // 64 threads per segment
+constexpr int kSortGroups = kThreads / kSortTPS;                  // 4 segments per CTA
+
+// The network as compile-time stages (template recursion: nvcc does not fully
+// unroll the nested loops at 32 keys per thread, and a partly unrolled network
+// indexes v[] at run time, i.e. through local memory).
+template <int LK, int LJ>
+__device__ __forceinline__ void sort32_stage(uint32_t (&v)[kSortKPT], uint32_t t, uint32_t* key) {
+  constexpr int k = 1 << LK, j = 1 << LJ;
+  if constexpr (j >= 1024) {                                       // the group's two warps
+    const bool lower = (t & 32u) == 0;
+#pragma unroll
+    for (int r = 0; r < kSortKPT; ++r) key[sort_pad(kSortKPT * t + r)] = v[r];
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kSortKPT; ++r) {
+      const uint32_t p = key[sort_pad((kSortKPT * t + r) ^ j)];
+      v[r] = lower ? min(v[r], p) : max(v[r], p);
+    }
+    __syncthreads();
+  } else if constexpr (j >= kSortKPT) {                            // lanes t and t ^ (j / 32)
+    const bool lower = (t & (uint32_t)(j / kSortKPT)) == 0;
+#pragma unroll
+    for (int r = 0; r < kSortKPT; ++r) {
+      const uint32_t p = __shfl_xor_sync(0xffffffffu, v[r], j / kSortKPT);
+      v[r] = lower ? min(v[r], p) : max(v[r], p);
+    }
+  } else {                                                         // registers r and r + j
+#pragma unroll
+    for (int r = 0; r < kSortKPT; ++r) {
+      if (r & j) continue;
+      const bool asc = k >= kSortKPT || (r & k) == 0;              // k >= 32: held form
+      const uint32_t lo = v[r], hi = v[r + j];
+      v[r] = asc ? min(lo, hi) : max(lo, hi);
+      v[r + j] = asc ? max(lo, hi) : min(lo, hi);
+    }
+  }
+}
+template <int LK, int LJ>
+struct Sort32Phase {
+  __device__ __forceinline__ static void run(uint32_t (&v)[kSortKPT], uint32_t t, uint32_t* key) {
+    sort32_stage<LK, LJ>(v, t, key);
+    Sort32Phase<LK, LJ - 1>::run(v, t, key);
+  }
+};
+template <int LK>
+struct Sort32Phase<LK, -1> {
+  __device__ __forceinline__ static void run(uint32_t (&)[kSortKPT], uint32_t, uint32_t*) {}
+};
+template <int LK>
+struct Sort32Net {
+  __device__ __forceinline__ static void run(uint32_t (&v)[kSortKPT], uint32_t t, uint32_t* key) {
+    if constexpr (LK >= 5) {                                       // complement for phase 2^LK (held form)
+      const uint32_t now = LK < 11 ? (t >> (LK - 5)) & 1u : 0u;    // index bit 2^LK
+      const uint32_t before = LK > 5 ? (t >> (LK - 6)) & 1u : 0u;
+      const uint32_t m = 0u - (now ^ before);
+#pragma unroll
+      for (int r = 0; r < kSortKPT; ++r) v[r] ^= m;
+    }
+    Sort32Phase<LK, LK - 1>::run(v, t, key);
+    Sort32Net<LK + 1>::run(v, t, key);
+  }
+};
+template <>
+struct Sort32Net<12> {
+  __device__ __forceinline__ static void run(uint32_t (&)[kSortKPT], uint32_t, uint32_t*) {}
+};
+
+__device__ inline void sort_body32(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n, int rank,
+                                   int S, uint8_t* stage) {
+  constexpr int kPadSeg = kSortSeg + kSortSeg / 32;
+  const uint32_t t = threadIdx.x % kSortTPS, grp = threadIdx.x / kSortTPS;
+  uint32_t* key = reinterpret_cast<uint32_t*>(stage) + grp * kPadSeg;   // this group's padded segment
+  const uint64_t nseg = n / kSortSeg;
+  const bool vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) & 15) == 0;
+  auto load32 = [&](uint64_t seg, uint32_t* w) {
+    if (seg >= nseg) return;                                      // idle group: garbage, never stored
+    const uint32_t* src = x + seg * kSortSeg + kSortKPT * t;
+    if (vec) {
+#pragma unroll
+      for (int q = 0; q < kSortKPT / 4; ++q) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(src) + q);
+        w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
+      }
+    } else {
+#pragma unroll
+      for (int r = 0; r < kSortKPT; ++r) w[r] = src[r];
+    }
+  };
+  const uint64_t step = (uint64_t)kSortGroups * S;
+  uint32_t nxt[kSortKPT];
+  load32((uint64_t)rank + (uint64_t)grp * S, nxt);
+  // every group runs the same number of rounds (the smem stage has block barriers)
+  for (uint64_t base = rank; base < nseg; base += step) {
+    const uint64_t seg = base + (uint64_t)grp * S;
+    uint32_t v[kSortKPT];
+#pragma unroll
+    for (int r = 0; r < kSortKPT; ++r) v[r] = nxt[r];
+    load32(seg + step, nxt);                                      // next round in flight
+    Sort32Net<1>::run(v, t, key);                                 // the 66 stages, fully expanded
+    if (seg < nseg) {
+      uint32_t* dst = y + seg * kSortSeg + kSortKPT * t;
+      if (vec) {
+#pragma unroll
+        for (int q = 0; q < kSortKPT / 4; ++q)
+          reinterpret_cast<uint4*>(dst)[q] = make_uint4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      } else {
+#pragma unroll
+        for (int r = 0; r < kSortKPT; ++r) dst[r] = v[r];
+      }
+    }
+  }
+}
+
+#ifndef STRINGS_SORT_KPT
+#define STRINGS_SORT_KPT 32
+#endif
+__device__ __forceinline__ void sort_body(const uint32_t* __restrict__ x, uint32_t* __restrict__ y, uint64_t n,
+                                          int rank, int S, uint8_t* stage) {
+  if constexpr (STRINGS_SORT_KPT == 32) sort_body32(x, y, n, rank, S, stage);
+  else sort_body8(x, y, n, rank, S, stage);
 }
 
 // Run one work item on this CTA (rank of S).
