@@ -215,3 +215,19 @@ def test_sort_bit_exact(segs, ctas):
         x[:2048] = rng.integers(0, 4, 2048)            # many duplicates in the first segment
     (y,) = _launch(S.make_desc(S.SORT, n=n), [x], [np.zeros(n, np.uint32)], ctas)
     assert np.array_equal(y, K.sort_segments(x))
+
+
+@pytest.mark.parametrize("ctas", [3, 148])
+def test_sort_unaligned_pointers(ctas):
+    # input and output 4 B past a 16-B boundary: the scalar load / store path of the
+    # network (every group of a 4-segment round; several rounds on 3 CTAs)
+    torch = _torch()
+    segs = 37
+    n = 2048 * segs
+    x = np.random.default_rng(5).integers(0, 1 << 32, n + 1, dtype=np.uint64).astype(np.uint32)
+    dx = torch.from_numpy(x.view(np.int32)).cuda()
+    dy = torch.zeros(n + 1, dtype=torch.int32, device="cuda")
+    S.kernel_launch(0, S.make_desc(S.SORT, n=n), [dx.data_ptr() + 4], [dy.data_ptr() + 4], ctas=ctas,
+                    stream=torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    assert np.array_equal(dy.cpu().numpy().view(np.uint32)[1:], K.sort_segments(x[1:]))
