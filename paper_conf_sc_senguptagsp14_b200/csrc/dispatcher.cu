@@ -125,7 +125,11 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
             if (atomicCAS(&heads[r], h, h + 1) == h) {
               ps->ring_idx = (uint32_t)r * kRing + h % kRing;
               ps->seq = h + 1;
+#ifdef STRINGS_TSTART_AFTER_CAS
+              ps->t_start = globaltimer();      // experiment: how long the claim CAS takes
+#else
               ps->t_start = t_seen;
+#endif
               ps->total = 0;                      // decided below, after the CTAs are released
               slot = cpart ? (uint32_t)e : ((uint32_t)e & 0xFFFFu);
               kc = cpart ? 0xFFu : (((uint32_t)e >> 16) & 0xFFu);
