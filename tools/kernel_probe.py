@@ -5,7 +5,8 @@
 
 Order of launches: VSCALE n=2^28 (x2), XFER n=2^28 (x2), GEMM 18944x256x256 R=64 (x2);
 `xfer_item`: XFER n=2^24 on 72 then 144 CTAs (x2 each), the C2 work item on one P=2 partition;
-`hist` (2^30 bytes), `scan`, `sort` (2^28 u32): the NEXT-2 bodies.
+`hist` (2^30 bytes), `scan`, `sort` (2^28 u32): the NEXT-2 bodies; `gemm_small`: the C2 job's GEMM
+(256^3, R = 64) on 2 CTAs, SURVEY 8(d)'s tensor-pipe check.
 The persistent dispatcher runs exactly these device bodies on its SM partitions.
 """
 import os
@@ -53,6 +54,18 @@ def main():
         for _ in range(2):
             S.kernel_launch(0, S.make_desc(S.GEMM, m=m, n=nn, k=k, reps=reps), [a.data_ptr(), b.data_ptr()],
                             [c.data_ptr()], stream=st)
+        torch.cuda.synchronize()
+        assert torch.equal(c, a.float() @ b.float())
+    if "gemm_small" in which:
+        # SURVEY 8(d)'s kernel check: the C2 job's GEMM (256^3, R = 64) on 2 CTAs, one
+        # 128 x 256 tile each with all 64 repetitions (tensor-pipe activity on its SMs)
+        m, nn, k, reps = 256, 256, 256, 64
+        a = torch.randint(-2, 3, (m, k), device="cuda").to(torch.bfloat16)
+        b = torch.randint(-2, 3, (k, nn), device="cuda").to(torch.bfloat16)
+        c = torch.empty((m, nn), dtype=torch.float32, device="cuda")
+        for _ in range(2):
+            S.kernel_launch(0, S.make_desc(S.GEMM, m=m, n=nn, k=k, reps=reps), [a.data_ptr(), b.data_ptr()],
+                            [c.data_ptr()], ctas=2, stream=st)
         torch.cuda.synchronize()
         assert torch.equal(c, a.float() @ b.float())
     if "hist" in which:
