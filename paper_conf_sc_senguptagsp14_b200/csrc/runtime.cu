@@ -1325,7 +1325,10 @@ class Runtime : public strings::Hooks {
     }
     done_count += 1;
     last_done = std::max(last_done, t);
-    cv_done.notify_all();
+    // waiters (strings_sync of a tenant, strings_drain of all) wait for some tenant's
+    // outstanding count to reach 0: waking them at every job completion made them
+    // contend for the engine's mutex once per job
+    if (tn.outstanding == 0) cv_done.notify_all();
   }
 
   void finalizer_main() {
