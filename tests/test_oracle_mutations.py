@@ -65,6 +65,11 @@ MUTATIONS = [
      "if self.cfg.las_admission:", "if False:"),
     ("las_weight_ignored", "oracle/des.py",
      "lhs, rhs = ca * b.prio, cb * a.prio", "lhs, rhs = ca, cb"),
+    ("arbiter_cold_uses_feedback", "oracle/des.py",
+     "if b in (W.RTF, W.GUF, W.DTF, W.MBF, W.DYNAMIC) and not self.has_sample(j):",
+     "if b in (W.RTF, W.GUF, W.DTF, W.MBF, W.DYNAMIC) and False:"),
+    ("dynamic_means_dtf", "oracle/des.py",
+     "        if b == W.DYNAMIC:\n            return W.MBF", "        if b == W.DYNAMIC:\n            return W.DTF"),
     ("gwtmin_ignores_weight", "oracle/des.py",
      "if best is None or len(d.resident) * best.weight < len(best.resident) * d.weight:",
      "if best is None or len(d.resident) < len(best.resident):"),

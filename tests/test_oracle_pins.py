@@ -317,3 +317,45 @@ def test_c4c_admissions_are_capacity_blocked():
     base.admission = counted_b
     base.run()
     assert blocked_b == []
+
+
+# ------------------------------------------------------- arbiter (L311, L1073; R-15)
+def _placements(o):
+    """(job, gid, tenant, policy, score) of every PLACE record, in order."""
+    return [(int(f[7]), int(f[2]), int(f[5]), int(f[8]), int(f[9]))
+            for f in (ln.split() for ln in o.trace) if f[1] == "PLACE"]
+
+
+def test_arbiter_places_cold_jobs_by_gmin():
+    # PAPER.md L311, L1073 (reading R-15): a feedback policy needs a sample of the
+    # job's (tenant, class) in the SFT; until then the arbiter places it by GMin.
+    # G = 2, RTF, three cold jobs at t = 0: a 64 MiB XFER (tenant 0), then two
+    # tiny VSCALE jobs (tenants 1, 2).  GMin: XFER -> GID0 (0 / 0 resident, tie),
+    # VSCALE -> GID1 (1 / 0), VSCALE -> GID0 (1 / 1, tie -> lowest GID); the
+    # scores are the resident counts 0, 0, 1 and every PLACE records GMIN (1).
+    # (RTF on the class priors would send the third job to GID1, away from the
+    # XFER's ~2.7 ms of predicted remaining transfer time.)
+    cfg = W.SystemConfig(num_gpus=2, balancer=W.RTF, admit_cap=10 ** 6)
+    specs = [W.JobSpec(tenant=0, kclass=W.XFER, n=1 << 24),
+             W.JobSpec(tenant=1, kclass=W.VSCALE, n=1024),
+             W.JobSpec(tenant=2, kclass=W.VSCALE, n=1024)]
+    o = Oracle(W.Workload("pin", cfg, [W.TenantSpec() for _ in specs], specs))
+    for j in o.jobs:
+        j.arrived = True
+    o.admission(0)
+    assert _placements(o) == [(0, 0, 0, W.GMIN, 0), (1, 1, 1, W.GMIN, 0), (2, 0, 2, W.GMIN, 1)]
+
+
+def test_dynamic_is_mbf_once_the_class_has_a_sample():
+    # R-15: DYNAMIC places a (tenant, class) with MBF once the SFT holds a sample
+    # of it, and a class without one by GMin.  G = 2, no joint selection; tenant
+    # 0's GEMM row is warm, tenant 1's cold: PLACE records MBF (6) for tenant 0's
+    # job and GMIN (1) for tenant 1's.
+    cfg = W.SystemConfig(num_gpus=2, balancer=W.DYNAMIC, admit_cap=10 ** 6, joint_select=0)
+    specs = [gemm_job(0), gemm_job(1)]
+    o = Oracle(W.Workload("pin", cfg, [W.TenantSpec() for _ in specs], specs))
+    o.sft[(0, W.GEMM)] = SFTEntry(count=1, h2d=10, kl=20, d2h=10, util=30000)
+    for j in o.jobs:
+        j.arrived = True
+    o.admission(0)
+    assert {t: pol for (_, _, t, pol, _) in _placements(o)} == {0: W.MBF, 1: W.GMIN}
