@@ -70,6 +70,27 @@ MUTATIONS = [
      "if b in (W.RTF, W.GUF, W.DTF, W.MBF, W.DYNAMIC) and False:"),
     ("dynamic_means_dtf", "oracle/des.py",
      "        if b == W.DYNAMIC:\n            return W.MBF", "        if b == W.DYNAMIC:\n            return W.DTF"),
+    ("grr_cursor_not_advanced", "oracle/des.py",
+     "self.grr_cursor = (g + 1) % self.G", "self.grr_cursor = g"),
+    ("ct_off_by_one", "oracle/des.py",
+     "if tn.pending and tn.inflight < tn.c:", "if tn.pending and tn.inflight <= tn.c:"),
+    ("admit_cap_off_by_one", "oracle/des.py",
+     "adm = [d for d in self.devices if len(d.resident) < self.M]",
+     "adm = [d for d in self.devices if len(d.resident) <= self.M]"),
+    ("awake_budget_off_by_one", "oracle/des.py",
+     "free = self.A - d.woken_unfinished", "free = self.A - d.woken_unfinished + 1"),
+    ("fifo_wakes_by_tenant", "oracle/des.py",
+     "for j in sorted(cands, key=lambda j: j.place_order)[:free]:",
+     "for j in sorted(cands, key=lambda j: (j.tenant, j.seq))[:free]:"),
+    ("las_wake_most_service_first", "oracle/des.py",
+     "for j in self.las_sorted(cands)[:free]:", "for j in self.las_sorted(cands)[::-1][:free]:"),
+    ("ps_no_kl_diversity", "oracle/des.py",
+     "if active[KL] == 0 and by[KL] and free > 0:", "if False:"),
+    ("las_tie_highest_tenant", "oracle/des.py",
+     "return -1 if a.tenant < b.tenant else 1", "return -1 if a.tenant > b.tenant else 1"),
+    ("arrival_order_by_tenant_first", "oracle/des.py",
+     "return sorted(js, key=lambda j: (j.arrival, j.tenant, j.seq))",
+     "return sorted(js, key=lambda j: (j.tenant, j.arrival, j.seq))"),
     ("gwtmin_ignores_weight", "oracle/des.py",
      "if best is None or len(d.resident) * best.weight < len(best.resident) * d.weight:",
      "if best is None or len(d.resident) < len(best.resident):"),

@@ -359,3 +359,40 @@ def test_dynamic_is_mbf_once_the_class_has_a_sample():
         j.arrived = True
     o.admission(0)
     assert {t: pol for (_, _, t, pol, _) in _placements(o)} == {0: W.MBF, 1: W.GMIN}
+
+
+# ------------------------------------------ FIFO dispatch and arrival-order admission
+def _records(trace, kind):
+    lines = trace.splitlines() if isinstance(trace, str) else trace
+    return [ln.split() for ln in lines if ln.split()[1] == kind]
+
+
+def test_fifo_wakes_in_placement_order():
+    # The FIFO device policy (the CUDA-runtime-like baseline) wakes ready
+    # phases in the order their jobs were PLACED, not by tenant id.  One GPU, awake
+    # budget A = 1.  Job A (tenant 1) arrives at 0, job B (tenant 0) at 10; every
+    # phase 100 / 50 / 100 ns.  A's H2D holds the one wake until t = 100; then A's
+    # KL and B's H2D are both ready and A, placed first, goes first:
+    #   t=0 A H2D, 100 A KL, 150 A D2H, 250 B H2D, 350 B KL, 400 B D2H.
+    # (Waking by tenant would start B's H2D at t = 100.)
+    cfg = W.SystemConfig(num_gpus=1, balancer=W.GMIN, device_policy=W.FIFO, awake_budget=1, admit_cap=4)
+    jobs = [kl_only(1, 50, arrival=0, h2d_ns=100, d2h_ns=100), kl_only(0, 50, arrival=10, h2d_ns=100, d2h_ns=100)]
+    wl = W.Workload("pin", cfg, [W.TenantSpec(), W.TenantSpec()], jobs)
+    got = [(int(f[0]), int(f[5]), f[3]) for f in _records(run_oracle(wl).trace, "WAKE")]
+    assert got == [(0, 1, "H2D"), (100, 1, "KL"), (150, 1, "D2H"), (250, 0, "H2D"), (350, 0, "KL"), (400, 0, "D2H")]
+
+
+def test_arrival_order_admission_is_by_arrival_then_tenant():
+    # Admission without LAS takes pending jobs in arrival order (DESIGN
+    # §4.4: (arrival, tenant, seq)).  One GPU with room for one job (M = 1): job C
+    # (tenant 2) arrives at 0 and holds the slot until its H2D ends at 100 (KL and
+    # D2H take 0); job D (tenant 1) arrives at 10, job E (tenant 0) at 20.  At 100
+    # D, the earlier arrival, is placed, then E at 200:
+    #   PLACE t=0 tenant 2, t=100 tenant 1, t=200 tenant 0.
+    # (Ordering by tenant first would place E before D.)
+    cfg = W.SystemConfig(num_gpus=1, balancer=W.GMIN, device_policy=W.PS, admit_cap=1)
+    jobs = [kl_only(2, 0, arrival=0, h2d_ns=100), kl_only(1, 0, arrival=10, h2d_ns=100),
+            kl_only(0, 0, arrival=20, h2d_ns=100)]
+    wl = W.Workload("pin", cfg, [W.TenantSpec() for _ in range(3)], jobs)
+    got = [(int(f[0]), int(f[5])) for f in _records(run_oracle(wl).trace, "PLACE")]
+    assert got == [(0, 2), (100, 1), (200, 0)]
