@@ -91,6 +91,19 @@ MUTATIONS = [
     ("arrival_order_by_tenant_first", "oracle/des.py",
      "return sorted(js, key=lambda j: (j.arrival, j.tenant, j.seq))",
      "return sorted(js, key=lambda j: (j.tenant, j.arrival, j.seq))"),
+    ("tfs_slice_ignores_weight", "oracle/des.py",
+     "if d.awake is None or d.awake_used >= self.tenants[d.awake].weight * self.S:",
+     "if d.awake is None or d.awake_used >= self.S:"),
+    ("tfs_pick_most_service", "oracle/des.py",
+     "if best is None or d.svc.get(tid, 0) * self.tenants[best].weight < \\",
+     "if best is None or d.svc.get(tid, 0) * self.tenants[best].weight > \\"),
+    ("sft_first_sample_averaged_with_zero", "oracle/des.py",
+     "        if e.count == 0:\n            e.h2d, e.kl, e.d2h, e.util = smp[0], smp[1], smp[2], util",
+     "        if e.count == 0:\n            e.h2d, e.kl, e.d2h, e.util = (4 * smp[0]) // 5, (4 * smp[1]) // 5, (4 * smp[2]) // 5, (4 * util) // 5"),
+    ("one_kl_slot", "oracle/des.py",
+     "self.busy = [[None], [None] * self.P, [None]]", "self.busy = [[None], [None], [None]]"),
+    ("epoch_service_from_start_not_epoch", "oracle/des.py",
+     "tn.gs_acc += t - max(j.start[x], self.epoch_start)", "tn.gs_acc += t - j.start[x]"),
     ("gwtmin_ignores_weight", "oracle/des.py",
      "if best is None or len(d.resident) * best.weight < len(best.resident) * d.weight:",
      "if best is None or len(d.resident) < len(best.resident):"),
