@@ -146,11 +146,14 @@ def test_pairwise_mix_on_hardware(pair):
         check_outputs(wl, r)
 
 
+@pytest.mark.parametrize("pair", [7, 5])
 @pytest.mark.parametrize("kl_mode", [0, 1])
-def test_multi_wave_scan_items_in_the_dispatcher(kl_mode):
-    # SCAN-XFER pair at full size: 2^24-element SCAN items span 4 waves on a KL
-    # partition (interleaved sums, tagged wave words, consecutive items per group)
-    wl = W.config_pair(7, balancer=W.MBF, instances=2, jobs_per_tenant=3, scale=1)
+def test_full_size_next2_items_in_the_dispatcher(pair, kl_mode):
+    # NEXT-2 pairs at full size.  7 = SCAN-XFER: 2^24-element SCAN items span 4 waves
+    # on a KL partition (interleaved sums, tagged wave words, consecutive items per
+    # group).  5 = HIST-SORT: 2^26-byte HIST items through the bulk pipeline and
+    # 2^20-key SORT items (512 segments, several 4-segment rounds per CTA)
+    wl = W.config_pair(pair, balancer=W.MBF, instances=2, jobs_per_tenant=3, scale=1)
     for timing in (S.INJECTED, S.MEASURED):
         r = run_workload(wl, timing_mode=timing, kl_mode=kl_mode)
         assert r.status == S.OK
