@@ -29,6 +29,10 @@
 
 namespace strings_dev {
 
+#ifndef STRINGS_GEN_POLL_NS
+#define STRINGS_GEN_POLL_NS 32                    // CTAs' back-off between polls of their generation word
+#endif
+
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -178,7 +182,7 @@ __global__ void __launch_bounds__(kThreads, 1) dispatcher_kernel(DispatchParams 
       if (lane == 0)                              // one poller per CTA
         while ((uint32_t)(gw = ld_acquire_gpu_u64(&ps->gen)) == seen) {
 #ifndef STRINGS_GEN_SPIN
-          __nanosleep(32);
+          __nanosleep(STRINGS_GEN_POLL_NS);
 #endif
         }
       __syncwarp();                               // orders lane 0's acquire before the item loads
